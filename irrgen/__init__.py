@@ -1,0 +1,253 @@
+"""Seeded synthetic inputs shared by the oracle side and the CUDA side.
+
+This module holds NO arithmetic of the method (no elimination, no solve, no
+update).  It only draws sizes and values, and builds structured test matrices
+from factors that are *chosen* here (A = P*L*U is assembled by a plain product
+of the chosen factors, which is input construction, not factorization).
+
+Reference: sizes and value distributions follow the paper's workloads
+(§V-A: "one thousand square matrices, whose sizes are randomly
+sampled between 1 and the value shown on the x-axis") and the configs of
+BASELINE.json / SURVEY.md §8(d).  The value generator is the counter-based
+splitmix64 stream of SURVEY.md §8(d):
+
+    a_ij = 2 * ((splitmix64(key + (i + j*m)) >> 11) * 2**-53) - 1
+    key  = splitmix64(seed ^ splitmix64(global_id))
+
+which is an exact dyadic in [-1, 1), independent of the leading dimension.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass
+
+import numpy as np
+
+__all__ = [
+    "splitmix64", "matrix_key", "uniform_values", "hash_stream",
+    "Config", "config", "CONFIG_NAMES",
+    "g1_exact", "g1_singular", "g1_front", "g2_dominant",
+    "front_values",
+]
+
+_M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
+_GOLD = np.uint64(0x9E3779B97F4A7C15)
+_C1 = np.uint64(0xBF58476D1CE4E5B9)
+_C2 = np.uint64(0x94D049BB133111EB)
+_SALT = np.uint64(0xD1B54A32D192ED03)
+
+
+def splitmix64(x):
+    """Standard splitmix64 finalizer, all arithmetic mod 2**64."""
+    with np.errstate(over="ignore"):
+        z = np.asarray(x, dtype=np.uint64) + _GOLD
+        z = (z ^ (z >> np.uint64(30))) * _C1
+        z = (z ^ (z >> np.uint64(27))) * _C2
+        return z ^ (z >> np.uint64(31))
+
+
+def matrix_key(seed: int, gid, salt: int = 0):
+    """Per-matrix stream key. salt=0 is the value stream of SURVEY §8(d);
+    other salts give independent streams for the structured families."""
+    with np.errstate(over="ignore"):
+        s = np.uint64(seed & 0xFFFFFFFFFFFFFFFF)
+        if salt:
+            s = s ^ (np.uint64(salt) * _SALT)
+        return splitmix64(s ^ splitmix64(np.asarray(gid, dtype=np.uint64)))
+
+
+def hash_stream(seed: int, gid: int, salt: int, count: int) -> np.ndarray:
+    """`count` uint64 draws of the stream (seed, gid, salt)."""
+    key = matrix_key(seed, gid, salt)
+    with np.errstate(over="ignore"):
+        return splitmix64(key + np.arange(count, dtype=np.uint64))
+
+
+def uniform_values(seed: int, gid: int, m: int, n: int) -> np.ndarray:
+    """m x n Fortran-ordered matrix with entries exact dyadics in [-1, 1)."""
+    key = matrix_key(seed, gid)
+    with np.errstate(over="ignore"):
+        x = splitmix64(key + np.arange(m * n, dtype=np.uint64))
+    u = (x >> np.uint64(11)).astype(np.float64) * (2.0 ** -53)
+    return (2.0 * u - 1.0).reshape((n, m)).T.copy(order="F") if m * n else np.zeros((m, n), order="F")
+
+
+def front_values(seed: int, gid: int, nf: int) -> np.ndarray:
+    """A frontal matrix is one nf x nf block, values as above."""
+    return uniform_values(seed, gid, nf, nf)
+
+
+# --------------------------------------------------------------------------
+# Workload configurations (BASELINE.json configs)
+# --------------------------------------------------------------------------
+@dataclass
+class Config:
+    name: str
+    kind: str            # "getrf" or "partial"
+    m: np.ndarray        # getrf: rows;  partial: n1
+    n: np.ndarray        # getrf: cols;  partial: n2
+    seed: int
+    description: str
+
+
+CONFIG_NAMES = ("C1", "C1big", "C2", "C3", "C4", "C5", "C5partial")
+
+
+def _sizes_c4c5(rng, count, tail_lo, tail_hi, mid_frac, tail_frac, log_mid):
+    r = rng.random(count)
+    nf = rng.integers(1, 64, size=count)                                  # U{1..63}
+    mid = r >= (1.0 - mid_frac - tail_frac)
+    tail = r >= (1.0 - tail_frac)
+    lm = np.floor(np.exp(rng.uniform(math.log(64), math.log(1025), size=count))).astype(np.int64)
+    lm = np.clip(lm, 64, 1024)
+    nf = np.where(mid, lm, nf)
+    nf = np.where(tail, rng.integers(tail_lo, tail_hi + 1, size=count), nf)
+    return nf.astype(np.int64)
+
+
+def config(name: str, scale: float = 1.0) -> Config:
+    """Return the seeded size lists of a workload.  `scale` < 1 keeps the size
+    distribution and shrinks the count (for tests / bounded CPU samples)."""
+    idx = {"C1": 1, "C1big": 11, "C2": 2, "C3": 3, "C4": 4, "C5": 5, "C5partial": 5}[name]
+    rng = np.random.Generator(np.random.PCG64(1000 + idx))
+    seed = 1000 + idx
+    if name == "C1":
+        cnt = max(1, int(100 * scale))
+        n = rng.integers(1, 33, size=cnt)
+        return Config(name, "getrf", n.copy(), n.copy(), seed, "100 square FP64, n~U{1..32}")
+    if name == "C1big":
+        cnt = max(1, int(1048576 * scale))
+        n = rng.integers(1, 33, size=cnt)
+        return Config(name, "getrf", n.copy(), n.copy(), seed, "1,048,576 square FP64, n~U{1..32}")
+    if name == "C2":
+        cnt = max(1, int(10000 * scale))
+        m = rng.integers(1, 257, size=cnt)
+        n = rng.integers(1, 257, size=cnt)
+        n[0::2] = m[0::2]                       # even i: square
+        odd = np.arange(cnt) % 2 == 1
+        while True:                             # odd i: resample n while n == m
+            bad = odd & (n == m)
+            if not bad.any():
+                break
+            n[bad] = rng.integers(1, 257, size=int(bad.sum()))
+        return Config(name, "getrf", m, n, seed, "10,000 FP64, dims~U{1..256}, even square / odd rectangular m!=n")
+    if name == "C3":
+        cnt = max(1, int(2000 * scale))
+        n = rng.integers(256, 1025, size=cnt)
+        return Config(name, "getrf", n.copy(), n.copy(), seed, "2,000 square FP64, n~U{256..1024}")
+    if name == "C4":
+        cnt = max(1, int(50000 * scale))
+        nf = _sizes_c4c5(rng, cnt, 3072, 4096, 0.099, 0.001, True)
+        f = rng.uniform(0.25, 0.5, size=cnt)
+        n1 = np.maximum(1, np.rint(f * nf)).astype(np.int64)
+        n2 = nf - n1
+        return Config(name, "partial", n1, n2, seed,
+                      "50,000 fronts (90% U{1..63}, 9.9% log-U[64,1024], 0.1% U{3072..4096}); n1=rint(f*nf), f~U[.25,.5]")
+    if name in ("C5", "C5partial"):
+        cnt = max(1, int(200000 * scale))
+        nf = _sizes_c4c5(rng, cnt, 1024, 2048, 0.09, 0.01, True)
+        if name == "C5":
+            return Config(name, "getrf", nf.copy(), nf.copy(), seed,
+                          "200,000 fronts (90% U{1..63}, 9% log-U[64,1024], 1% U{1024..2048}), full DGETRF")
+        f = rng.uniform(0.25, 0.5, size=cnt)
+        n1 = np.maximum(1, np.rint(f * nf)).astype(np.int64)
+        return Config(name, "partial", n1, nf - n1, seed, "C5 fronts, partial factorization (C4 rule)")
+    raise KeyError(name)
+
+
+# --------------------------------------------------------------------------
+# Structured families (SURVEY.md §8(c) "Input families").  Each returns the
+# matrix AND the factors it was assembled from; the expected outputs are the
+# chosen factors, not the result of any elimination.
+# --------------------------------------------------------------------------
+_L_SET = np.array([0.0, 0.25, -0.25, 0.5, -0.5])
+_UD_SET = np.array([1.0, -1.0, 2.0, -2.0])
+
+
+def _apply_swaps_reverse(LU: np.ndarray, ipiv0: np.ndarray) -> np.ndarray:
+    """A = S_0 S_1 ... S_{k-1} (LU): apply row interchanges k-1..0 (input assembly)."""
+    A = LU.copy(order="F")
+    for k in range(len(ipiv0) - 1, -1, -1):
+        p = int(ipiv0[k])
+        if p != k:
+            A[[k, p], :] = A[[p, k], :]
+    return A
+
+
+def g1_exact(seed: int, gid: int, m: int, n: int, singular_col: int | None = None):
+    """G1: exact dyadic family.  L unit lower (m x k) with off-diagonals in
+    {0, +-1/4, +-1/2}; U (k x n) upper with integer off-diagonals in [-8, 8] and
+    diagonal in {+-1, +-2}; 0-based ipiv[k] ~ U[k, m).  Returns
+    (A, L, U, ipiv1based, info).  With singular_col=c (G1-sing): row c of U is
+    zeroed, L(c+1:, c) = 0 and ipiv[c] = c, so info = c+1."""
+    k = min(m, n)
+    h = hash_stream(seed, gid, 1, m * k + k * n + k + 1)
+    hl = h[: m * k].reshape((k, m)).T
+    hu = h[m * k: m * k + k * n].reshape((n, k)).T
+    hp = h[m * k + k * n:]
+    L = np.zeros((m, k))
+    for j in range(k):
+        L[j, j] = 1.0
+        idx = (hl[j + 1:, j] % np.uint64(len(_L_SET))).astype(np.int64)
+        L[j + 1:, j] = _L_SET[idx]
+    U = np.zeros((k, n))
+    for i in range(k):
+        U[i, i] = _UD_SET[int(hu[i, i] % np.uint64(4))]
+        U[i, i + 1:] = (hu[i, i + 1:] % np.uint64(17)).astype(np.int64) - 8
+    ipiv0 = np.array([j + int(hp[j] % np.uint64(m - j)) for j in range(k)], dtype=np.int64)
+    info = 0
+    if singular_col is not None:
+        c = singular_col
+        assert 0 <= c < k
+        U[c, c:] = 0.0
+        L[c + 1:, c] = 0.0
+        ipiv0[c] = c
+        info = c + 1
+    LU = L @ U                 # exact: dyadic products, |entries| << 2**53
+    A = _apply_swaps_reverse(LU, ipiv0)
+    return np.asfortranarray(A), L, U, (ipiv0 + 1).astype(np.int32), info
+
+
+def g1_singular(seed: int, gid: int, m: int, n: int, c: int):
+    return g1_exact(seed, gid, m, n, singular_col=c)
+
+
+def g1_front(seed: int, gid: int, n1: int, n2: int):
+    """G1': exact dyadic front.  F11 from G1; X (n1 x n2), F21 (n2 x n1) and
+    S (n2 x n2) small integers; F12 = F11 X, F22 = S + F21 X.  The partial
+    factorization must return F12 -> X and F22 -> S exactly."""
+    F11, L, U, ipiv, _ = g1_exact(seed, gid, n1, n1)
+    h = hash_stream(seed, gid, 2, n1 * n2 * 2 + n2 * n2)
+    X = ((h[: n1 * n2] % np.uint64(9)).astype(np.int64) - 4).astype(np.float64).reshape((n2, n1)).T
+    F21 = ((h[n1 * n2: 2 * n1 * n2] % np.uint64(9)).astype(np.int64) - 4).astype(np.float64).reshape((n1, n2)).T
+    S = ((h[2 * n1 * n2:] % np.uint64(9)).astype(np.int64) - 4).astype(np.float64).reshape((n2, n2)).T
+    F12 = F11 @ X
+    F22 = S + F21 @ X
+    f = np.asfortranarray
+    return dict(F11=f(F11), F12=f(F12), F21=f(F21), F22=f(F22), X=f(X), S=f(S), L=L, U=U, ipiv=ipiv)
+
+
+def g2_dominant(seed: int, gid: int, m: int, n: int):
+    """G2: permuted column-diagonally-dominant matrix.  Off-diagonals U[-1,1);
+    for j < k: a_jj = +-(2*sum_{i!=j}|a_ij| + 1); rows permuted by pi (row r
+    holds original row pi[r]).  Returns (A, ipiv1based) where ipiv follows from
+    pi alone: cur = pi; for each j, ipiv[j] = position of j in cur; swap."""
+    k = min(m, n)
+    B = uniform_values(seed, gid, m, n).copy()
+    h = hash_stream(seed, gid, 3, m + k)
+    for j in range(k):
+        col = np.abs(B[:, j]).sum() - abs(B[j, j])
+        sgn = 1.0 if (h[m + j] & np.uint64(1)) else -1.0
+        B[j, j] = sgn * (2.0 * col + 1.0)
+    pi = np.arange(m)
+    for t in range(m - 1, 0, -1):            # Fisher-Yates on the hash stream
+        r = int(h[t] % np.uint64(t + 1))
+        pi[t], pi[r] = pi[r], pi[t]
+    A = np.asfortranarray(B[pi, :])
+    cur = list(pi)
+    ipiv = np.zeros(k, dtype=np.int32)
+    for j in range(k):
+        p = cur.index(j, j)
+        ipiv[j] = p + 1
+        cur[j], cur[p] = cur[p], cur[j]
+    return A, ipiv

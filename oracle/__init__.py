@@ -1,0 +1,200 @@
+"""ctypes front-end of the plain CPU oracle (oracle/oracle.c).
+
+TEST INFRASTRUCTURE ONLY: imported by tests/, __graft_entry__.smoke() and the
+cpu_baseline / --impl reference legs of bench.py -- never by the product
+package.  The oracle shares no code with the CUDA path.
+
+Every function here only marshals numpy arrays into the C oracle; the
+arithmetic is in oracle.c (see its header for the PAPER.md citations).
+Matrices are numpy arrays in Fortran (column-major) order.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "oracle.c")
+_lib = None
+
+CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC", "-std=c11"]
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c -> liboracle.so (gcc, no FMA contraction, no fast-math)."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        tmp = _SO + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _SO)
+    return _SO
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = C.CDLL(_SO)
+        P = C.POINTER
+        dp, ip = P(C.c_double), P(C.c_int)
+        L.oracle_getrf.argtypes = [C.c_int, C.c_int, dp, C.c_int, ip, ip, dp]
+        L.oracle_getrf_batch.argtypes = [C.c_int, ip, ip, P(dp), ip, P(ip), ip, dp, C.c_int]
+        L.oracle_getrf_partial.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, dp, C.c_int,
+                                           dp, C.c_int, ip, ip]
+        L.oracle_getrf_partial_batch.argtypes = [C.c_int, ip, ip, P(dp), ip, P(dp), ip, P(dp), ip,
+                                                 P(dp), ip, P(ip), ip, C.c_int]
+        L.oracle_gemm.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_int, C.c_double, dp, C.c_int,
+                                  dp, C.c_int, C.c_double, dp, C.c_int]
+        L.oracle_trsm.argtypes = [C.c_int] * 6 + [C.c_double, dp, C.c_int, dp, C.c_int]
+        L.oracle_laswp.argtypes = [C.c_int, dp, C.c_int, C.c_int, C.c_int, ip]
+        L.oracle_backward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
+        L.oracle_backward_error.restype = C.c_double
+        L.oracle_num_threads.restype = C.c_int
+        _lib = L
+    return _lib
+
+
+def _dp(a):
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _ip(a):
+    return a.ctypes.data_as(C.POINTER(C.c_int))
+
+
+def _fortran(A):
+    A = np.asarray(A, dtype=np.float64)
+    if A.ndim != 2:
+        raise ValueError("matrix must be 2-D")
+    return np.array(A, dtype=np.float64, order="F", copy=True)
+
+
+def _ld(A):
+    return max(1, A.shape[0]) if A.size == 0 else A.strides[1] // 8
+
+
+def getrf(A):
+    """GEPP on a copy of A.  Returns (LU, ipiv (1-based int32), info, min_sep)."""
+    LU = _fortran(A)
+    m, n = LU.shape
+    ipiv = np.zeros(max(1, min(m, n)), dtype=np.int32)
+    info = np.zeros(1, dtype=np.int32)
+    sep = np.zeros(1)
+    buf = LU if LU.size else np.zeros((max(1, m), 1), order="F")
+    r = lib().oracle_getrf(m, n, _dp(buf), max(1, m), _ip(ipiv), _ip(info), _dp(sep))
+    if r < 0:
+        raise ValueError(f"oracle_getrf: bad argument {-r}")
+    return LU, ipiv[: min(m, n)], int(info[0]), float(sep[0])
+
+
+def getrf_batch(mats, nthreads: int = 0):
+    """Batched GEPP in place on a list of Fortran float64 arrays (OpenMP over
+    matrices).  Returns (ipivs, info, min_sep)."""
+    b = len(mats)
+    m = np.array([M.shape[0] for M in mats], dtype=np.int32)
+    n = np.array([M.shape[1] for M in mats], dtype=np.int32)
+    ld = np.array([max(1, M.shape[0]) for M in mats], dtype=np.int32)
+    keep = []
+    ptrs = (C.POINTER(C.c_double) * max(1, b))()
+    ipivs = [np.zeros(max(1, min(M.shape)), dtype=np.int32) for M in mats]
+    iptrs = (C.POINTER(C.c_int) * max(1, b))()
+    for i, M in enumerate(mats):
+        if not (M.flags.f_contiguous and M.dtype == np.float64):
+            raise ValueError("matrices must be Fortran float64")
+        buf = M if M.size else np.zeros(1)
+        keep.append(buf)
+        ptrs[i] = _dp(buf)
+        iptrs[i] = _ip(ipivs[i])
+    info = np.zeros(max(1, b), dtype=np.int32)
+    sep = np.zeros(max(1, b))
+    lib().oracle_getrf_batch(b, _ip(m), _ip(n), ptrs, _ip(ld), iptrs, _ip(info), _dp(sep), nthreads)
+    return [p[: min(M.shape)] for p, M in zip(ipivs, mats)], info[:b], sep[:b]
+
+
+def getrf_partial(F11, F12, F21, F22):
+    """Partial front factorization on copies.
+    Returns (F11 -> L\\U, F12 -> U^-1 L^-1 P^T F12, F22 -> F22 - F21 F12, ipiv, info)."""
+    F11, F12, F21, F22 = (_fortran(X) for X in (F11, F12, F21, F22))
+    n1, n2 = F11.shape[0], F22.shape[0]
+    ipiv = np.zeros(max(1, n1), dtype=np.int32)
+    info = np.zeros(1, dtype=np.int32)
+    bufs = [X if X.size else np.zeros(1) for X in (F11, F12, F21, F22)]
+    r = lib().oracle_getrf_partial(n1, n2, _dp(bufs[0]), max(1, n1), _dp(bufs[1]), max(1, n1),
+                                   _dp(bufs[2]), max(1, n2), _dp(bufs[3]), max(1, n2), _ip(ipiv), _ip(info))
+    if r < 0:
+        raise ValueError(f"oracle_getrf_partial: bad argument {-r}")
+    return F11, F12, F22, ipiv[:n1], int(info[0])
+
+
+def getrf_partial_batch(fronts, nthreads: int = 0):
+    """fronts: list of dicts with Fortran arrays F11, F12, F21, F22 (modified
+    in place).  Returns (ipivs, info)."""
+    b = len(fronts)
+    n1 = np.array([f["F11"].shape[0] for f in fronts], dtype=np.int32)
+    n2 = np.array([f["F22"].shape[0] for f in fronts], dtype=np.int32)
+    P = C.POINTER(C.c_double)
+    arrs = {k: (P * max(1, b))() for k in ("F11", "F12", "F21", "F22")}
+    lds = {k: np.zeros(max(1, b), dtype=np.int32) for k in arrs}
+    keep = []
+    ipivs = [np.zeros(max(1, int(x)), dtype=np.int32) for x in n1]
+    iptrs = (C.POINTER(C.c_int) * max(1, b))()
+    for i, f in enumerate(fronts):
+        for k in arrs:
+            X = f[k]
+            if X.size and not (X.dtype == np.float64 and X.strides[0] == 8):
+                raise ValueError("fronts must be column-major float64")
+            buf = X if X.size else np.zeros(1)
+            keep.append(buf)
+            arrs[k][i] = _dp(buf)
+            lds[k][i] = max(1, X.strides[1] // 8 if X.size else X.shape[0])
+        iptrs[i] = _ip(ipivs[i])
+    info = np.zeros(max(1, b), dtype=np.int32)
+    lib().oracle_getrf_partial_batch(b, _ip(n1), _ip(n2), arrs["F11"], _ip(lds["F11"]), arrs["F12"],
+                                     _ip(lds["F12"]), arrs["F21"], _ip(lds["F21"]), arrs["F22"],
+                                     _ip(lds["F22"]), iptrs, _ip(info), nthreads)
+    return [p[: int(k)] for p, k in zip(ipivs, n1)], info[:b]
+
+
+def gemm(ta, tb, alpha, A, B, beta, C_):
+    A, B, Cm = _fortran(A), _fortran(B), _fortran(C_)
+    m, n = Cm.shape
+    k = A.shape[0] if ta else A.shape[1]
+    bufs = [X if X.size else np.zeros((1, 1), order="F") for X in (A, B, Cm)]
+    lib().oracle_gemm(int(ta), int(tb), m, n, k, float(alpha), _dp(bufs[0]), max(1, A.shape[0]),
+                      _dp(bufs[1]), max(1, B.shape[0]), float(beta), _dp(bufs[2]), max(1, m))
+    return Cm
+
+
+def trsm(side, uplo, trans, diag, alpha, T, B):
+    T, B = _fortran(T), _fortran(B)
+    m, n = B.shape
+    bufs = [X if X.size else np.zeros((1, 1), order="F") for X in (T, B)]
+    lib().oracle_trsm(int(side), int(uplo), int(trans), int(diag), m, n, float(alpha),
+                      _dp(bufs[0]), max(1, T.shape[0]), _dp(bufs[1]), max(1, m))
+    return B
+
+
+def laswp(A, k1, k2, ipiv):
+    A = _fortran(A)
+    ipiv = np.ascontiguousarray(ipiv, dtype=np.int32)
+    buf = A if A.size else np.zeros((1, 1), order="F")
+    lib().oracle_laswp(A.shape[1], _dp(buf), max(1, A.shape[0]), int(k1), int(k2), _ip(ipiv))
+    return A
+
+
+def backward_error(A0, LU, ipiv):
+    A0, LU = _fortran(A0), _fortran(LU)
+    m, n = A0.shape
+    ipiv = np.ascontiguousarray(ipiv, dtype=np.int32)
+    if ipiv.size == 0:
+        ipiv = np.zeros(1, dtype=np.int32)
+    b0 = A0 if A0.size else np.zeros((1, 1), order="F")
+    b1 = LU if LU.size else np.zeros((1, 1), order="F")
+    return lib().oracle_backward_error(m, n, _dp(b0), max(1, m), _dp(b1), max(1, m), _ip(ipiv))
+
+
+def num_threads() -> int:
+    return lib().oracle_num_threads()
