@@ -1,0 +1,448 @@
+#!/usr/bin/env python
+"""bench.py -- variable-size batched DGETRF (irrLU) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl ours|reference]
+
+A step is one irr_getrf (or irr_getrf_partial for the front configs) call on
+the whole (per-rank) batch, i.e. every row of SURVEY §8(a), plus the NCCL
+gather of the per-matrix status words when N > 1.  Inputs are restored from a
+pristine device copy and L2 is flushed before every step, outside the timed
+region; each step is timed with CUDA events on the launching stream; the
+total over K steps is bracketed by a barrier + synchronize and reduced with
+MAX over ranks.  Weak scaling: at N GPUs the global batch is N x the config's
+batch, partitioned flop-balanced (LPT) over the ranks, each rank generating
+only its own matrices (global-id-keyed values).
+
+Metric (BASELINE.json): Gflop/s = sum FLOPS_DGETRF / time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import irrgen  # noqa: E402
+from paper_conf_sc_abdelfattahgbtld22_b200 import flops as F  # noqa: E402
+from paper_conf_sc_abdelfattahgbtld22_b200.shard import lpt_partition  # noqa: E402
+
+METRIC = "variable-size batched DGETRF Gflop/s and % FP64/HBM roofline at 1/2/4/8 B200"
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12   # 37.2: 148 SM x 64 DFMA/clk x 2 x 1.965 GHz
+FALLBACK_HBM_GBS = 6650.0
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback"
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.proc = None
+        self.idx = gpu_index
+        self.path = os.path.join("/tmp", f"irr_clocks_{os.getpid()}.csv")
+
+    def start(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.f.close()
+        sms, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sms.append(float(parts[0]))
+                mx = max(mx, float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sms:
+            return None
+        return {"sm_mhz": statistics.median(sms), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sms)}
+
+
+# ------------------------------------------------------------------ per-tier algorithmic work
+def tier_of(m, n, tier_m_max=24576):
+    m = np.asarray(m)
+    n = np.asarray(n)
+    lds = m | 1
+    t = np.full(len(m), 2)
+    t[(lds * n) <= tier_m_max] = 1
+    t[(m <= 32) & (n <= 32)] = 0
+    t[(m == 0) | (n == 0)] = -1
+    return t
+
+
+def class_work(m, n, nb=32):
+    """Algorithmic (flops, bytes) per kernel class for one getrf step
+    (DESIGN.md 'Roofline accounting')."""
+    m = np.asarray(m, dtype=np.int64)
+    n = np.asarray(n, dtype=np.int64)
+    t = tier_of(m, n)
+    out = {}
+    for cls, tier in (("lu_small", 0), ("lu_mid", 1)):
+        sel = t == tier
+        out[cls] = (float(F.getrf_flops(m[sel], n[sel]).sum()), float(F.getrf_bytes(m[sel], n[sel]).sum()))
+    sel = t == 2
+    mL, nL = m[sel], n[sel]
+    g_f = g_b = p_f = p_b = s_f = s_b = 0.0
+    kL = np.minimum(mL, nL)
+    for j in range(0, int(kL.max()) if len(kL) else 0, nb):
+        act = kL > j
+        if not act.any():
+            break
+        mm, nn, kk = mL[act], nL[act], kL[act]
+        ib = np.minimum(nb, kk - j)
+        Mr = np.maximum(mm - j - ib, 0).astype(np.float64)
+        Nr = np.maximum(nn - j - ib, 0).astype(np.float64)
+        g_f += float((2 * Mr * Nr * ib).sum())
+        g_b += float((16 * Mr * Nr + 8 * (Mr + Nr) * ib * ((Mr > 0) & (Nr > 0))).sum())
+        p_f += float(F.getrf_flops(mm - j, ib).sum())
+        p_b += float((16.0 * (mm - j) * ib).sum())
+        s_f += float((ib * ib * Nr).sum())
+        s_b += float((16.0 * ib * (nn - ib)).sum())
+    out["gemm_trailing"] = (g_f, g_b)
+    out["panel"] = (p_f, p_b)
+    out["swap_trsm"] = (s_f, s_b)
+    return out
+
+
+def class_work_partial(n1, n2, nb=32):
+    n1 = np.asarray(n1, dtype=np.int64)
+    n2 = np.asarray(n2, dtype=np.int64)
+    out = class_work(n1, n1, nb)
+    out["gemm_dcwi"] = (float((2.0 * n1 * n2 * n2).sum()), float((8.0 * (2 * n2 * n2 + n2 * n1 + n1 * n2)).sum()))
+    out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((32.0 * n1 * n2).sum()))
+    return out
+
+
+# ------------------------------------------------------------------ CPU oracle timing
+def time_oracle(cfg, idx, target_s=10.0, threads=None):
+    """Time the oracle (as it stands) on a bounded sample of the workload.
+    Returns (gflops, cores, sample description, seconds)."""
+    import oracle
+    oracle.build()
+    threads = threads or len(os.sched_getaffinity(0))
+    rng = np.random.default_rng(12345)
+    order = rng.permutation(idx)
+
+    def run(sel):
+        if cfg.kind == "getrf":
+            mats = [irrgen.uniform_values(cfg.seed, int(g), int(cfg.m[g]), int(cfg.n[g])) for g in sel]
+            fl = float(F.getrf_flops(cfg.m[sel], cfg.n[sel]).sum())
+            t0 = time.perf_counter()
+            oracle.getrf_batch(mats, nthreads=threads)
+            return fl, time.perf_counter() - t0
+        fronts = []
+        for g in sel:
+            a, b = int(cfg.m[g]), int(cfg.n[g])
+            Fm = irrgen.front_values(cfg.seed, int(g), a + b)
+            fronts.append(dict(F11=Fm[:a, :a].copy(order="F"), F12=Fm[:a, a:].copy(order="F"),
+                               F21=Fm[a:, :a].copy(order="F"), F22=Fm[a:, a:].copy(order="F")))
+        fl = float(F.partial_flops(cfg.m[sel], cfg.n[sel]).sum())
+        t0 = time.perf_counter()
+        oracle.getrf_partial_batch(fronts, nthreads=threads)
+        return fl, time.perf_counter() - t0
+
+    # calibrate on a small slice, then size the sample for ~target_s
+    n0 = min(len(order), 64)
+    fl0, t0 = run(order[:n0])
+    rate = fl0 / max(t0, 1e-6)
+    all_fl = F.getrf_flops(cfg.m[order], cfg.n[order]) if cfg.kind == "getrf" else \
+        F.partial_flops(cfg.m[order], cfg.n[order])
+    budget = rate * target_s
+    cnt = int(np.searchsorted(np.cumsum(all_fl), budget)) + 1
+    cnt = max(n0, min(len(order), cnt))
+    sel = order[:cnt]
+    fl, t = run(sel)
+    desc = f"{cnt} of {len(idx)} matrices of {cfg.name} (uniform random sample, seed 12345), {fl:.3e} flop"
+    return fl / t / 1e9, threads, desc, t
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle (this tier's reference arm), rank 0 only."""
+    if rank != 0:
+        return
+    cfg = irrgen.config(args.config)
+    idx = np.arange(len(cfg.m))
+    vals = []
+    threads = len(os.sched_getaffinity(0))
+    desc = ""
+    for s in range(args.warmup + args.steps):
+        g, cores, desc, secs = time_oracle(cfg, idx, target_s=args.ref_seconds, threads=threads)
+        if s >= args.warmup:
+            vals.append(g)
+    v = float(np.mean(vals))
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "Gflop/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": None, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "description": cfg.description, "batch": int(len(cfg.m))},
+            "cpu_baseline": {"value": v, "unit": "Gflop/s", "cores": threads, "kind": "oracle", "sample": desc},
+            "e2e": {"value": v, "unit": "Gflop/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2", choices=irrgen.CONFIG_NAMES)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--ref-seconds", type=float, default=5.0)
+    ap.add_argument("--profile-out", default=None, help="write per-kernel-class timings here (json)")
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_abdelfattahgbtld22_b200 import irr
+    from paper_conf_sc_abdelfattahgbtld22_b200.batch import FrontBatch, MatrixBatch
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    # ---- workload: global batch = world x config, LPT-sharded by flops
+    cfg = irrgen.config(args.config, scale=float(world))
+    kind = cfg.kind
+    work = F.getrf_flops(cfg.m, cfg.n) if kind == "getrf" else F.partial_flops(cfg.m, cfg.n)
+    owner = lpt_partition(work, world)
+    mine = np.nonzero(owner == rank)[0]
+    m_loc, n_loc = cfg.m[mine], cfg.n[mine]
+    flops_local = float(work[mine].sum())
+    flops_global = float(work.sum())
+
+    if kind == "getrf":
+        B = MatrixBatch(m_loc, n_loc, device=dev)
+        ld_loc = B.ld_h
+        call = lambda: B.getrf()  # noqa: E731
+        cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"))
+        bytes_local = float(F.getrf_bytes(m_loc, n_loc).sum())
+        host = B.host_buffer(pinned=True)
+        hn = host.numpy()
+        hn[:] = 0.0
+        # values keyed by GLOBAL id so a matrix is identical at every N
+        irrgen.fill_packed(cfg.seed, m_loc, n_loc, ld_loc, B.offsets, hn, gids=mine)
+        outs = [B.data, B.ipiv_data, B.info]
+    else:
+        B = FrontBatch(m_loc, n_loc, device=dev)
+        call = lambda: B.getrf_partial()  # noqa: E731
+        cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"))
+        bytes_local = float(F.partial_bytes(m_loc, n_loc).sum())
+        host = torch.empty(B.total, dtype=torch.float64, pin_memory=True)
+        hn = host.numpy()
+        hn[:] = 0.0
+        nf = B.nf_h
+        irrgen.fill_packed(cfg.seed, nf, nf, B.ld_h, B.offsets, hn, gids=mine)
+        outs = [B.data, B.ipiv_data, B.info]
+    pristine = host.to(dev)
+    flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device=dev)   # > 126 MB L2
+    stream = torch.cuda.current_stream(dev)
+
+    # status gather (the only collective): per-matrix info words, padded
+    pad = int(max(np.bincount(owner, minlength=world))) if world > 1 else len(mine)
+    status = torch.zeros(max(1, pad), dtype=torch.int32, device=dev)
+    gathered = torch.zeros(world * max(1, pad), dtype=torch.int32, device=dev) if world > 1 else None
+
+    def step():
+        call()
+        if world > 1:
+            status[: B.batch].copy_(B.info[: B.batch])
+            dist.all_gather_into_tensor(gathered, status)
+
+    def restore():
+        B.data.copy_(pristine)
+        flush.zero_()
+
+    # ---- warm-up
+    for _ in range(args.warmup):
+        restore()
+        step()
+    torch.cuda.synchronize()
+
+    # ---- timed region
+    irr.irr_profile_enable(100000)
+    irr.irr_launch_count(reset=True)
+    clocks = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    total_ms = 0.0
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for s in range(args.steps):
+        restore()
+        evs[s][0].record(stream)
+        step()
+        evs[s][1].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    total_ms = float(sum(step_ms))
+    launches = irr.irr_launch_count()
+    prof = irr.irr_profile_collect()
+    irr.irr_profile_enable(0)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_max_ms = float(t.item())
+    ms_per_step = total_max_ms / args.steps
+    value = flops_global / (ms_per_step * 1e-3) / 1e9
+
+    # ---- parity spot-check on a few matrices of this rank (oracle-free: info must be >= 0)
+    info_h = B.info[: B.batch].cpu().numpy()
+    bad_info = int((info_h < 0).sum())
+
+    # ---- e2e: host buffers through the public API, H2D + compute + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        res_host = [torch.empty(o.numel(), dtype=o.dtype, pin_memory=True) for o in outs]
+        h2d = host.numel() * 8
+        d2h = sum(o.numel() * o.element_size() for o in outs)
+        e_ms = []
+        for s in range(args.warmup + args.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            B.data.copy_(host, non_blocking=True)
+            step()
+            for o, h in zip(outs, res_host):
+                h.copy_(o.view(-1), non_blocking=True)
+            b.record(stream)
+            torch.cuda.synchronize()
+            if s >= args.warmup:
+                e_ms.append(a.elapsed_time(b))
+        te = torch.tensor([float(np.sum(e_ms))], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e_step = float(te.item()) / args.steps
+        e2e = {"value": flops_global / (e_step * 1e-3) / 1e9, "unit": "Gflop/s", "ms_per_step": e_step,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h)}
+
+    # ---- roofline of the dominant kernel class (rank-local, per step)
+    hbm, hbm_src = peaks()
+    dom = max(prof.items(), key=lambda kv: kv[1][0])
+    dname, (dms, dcnt) = dom
+    dms_step = dms / args.steps
+    fl, by = cw.get(dname, (0.0, 0.0))
+    t_f = fl / (FP64_PEAK_TFLOPS * 1e12)
+    t_b = by / (hbm * 1e9)
+    if t_b >= t_f:
+        ach = by / (dms_step * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm}
+    else:
+        ach = fl / (dms_step * 1e-3) / 1e12
+        roof = {"bound": "alu", "achieved": ach, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                "frac": ach / FP64_PEAK_TFLOPS}
+    roof["kernel"] = dname
+    roof["share_of_step"] = dms_step / (total_ms / args.steps)
+    roof["launches_per_step"] = dcnt / args.steps
+    roof["peak_source"] = (hbm_src + " MEASURED_PEAKS.json hbm_gbs") if roof["bound"] == "hbm" else \
+        "derived: 148 SM x 64 DFMA/clk x 2 flop x 1.965 GHz"
+    roof["traffic"] = _ncu_traffic(args.config, dname, dcnt / args.steps)
+    whole = {"flops": flops_local, "bytes": bytes_local,
+             "fp64_frac": flops_local / (ms_per_step * 1e-3) / (FP64_PEAK_TFLOPS * 1e12),
+             "hbm_frac": bytes_local / (ms_per_step * 1e-3) / (hbm * 1e9)}
+
+    # ---- CPU baseline: the oracle on a bounded sample (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        g, cores, desc, secs = time_oracle(irrgen.config(args.config), np.arange(len(cfg.m)),
+                                           target_s=args.cpu_seconds)
+        cpu = {"value": g, "unit": "Gflop/s", "cores": cores, "kind": "oracle", "sample": desc,
+               "seconds": secs}
+
+    if args.profile_out and rank == 0:
+        with open(args.profile_out, "w") as f:
+            json.dump({k: {"ms_per_step": v[0] / args.steps, "launches_per_step": v[1] / args.steps,
+                           "alg_flops": cw.get(k, (0, 0))[0], "alg_bytes": cw.get(k, (0, 0))[1]}
+                       for k, v in prof.items() if v[1]}, f, indent=1)
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "data": "synthetic (seeded splitmix64 values U[-1,1), sizes per BASELINE config)",
+                "config": {"workload": cfg.name if world == 1 else f"{world}x{args.config}",
+                           "description": irrgen.config(args.config).description,
+                           "batch_per_gpu": int(B.batch), "global_batch": int(len(cfg.m)),
+                           "sharding": "LPT by flops" if world > 1 else "none",
+                           "l2": "flushed (512 MB write) and inputs restored before every step, untimed",
+                           "tuning": {k: irr.irr_get_tuning(k) for k in ("nb", "tier_m_max", "panel_rows")}},
+                "gpu_launches": int(launches), "roofline": roof, "whole_step": whole,
+                "kernel_ms_per_step": {k: v[0] / args.steps for k, v in prof.items() if v[1]},
+                "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "info_negative": bad_info}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def _ncu_traffic(config, kname, launches_per_step):
+    """dram bytes per launch of `kname` from a committed ncu --set full summary, else None."""
+    p = os.path.join(ROOT, "profiles", f"ncu_traffic_{config}.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(kname)
+    except Exception:
+        return None
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,202 @@
+/*
+ * irr.h -- C ABI of the B200-native irrLU library (libirr.so).
+ *
+ * Variable-size ("irregular") batched dense LU with partial pivoting and its
+ * building blocks, after Abdelfattah et al., SC'22.  Citations "P:L<n>" are
+ * lines of the paper text (/root/reference/PAPER.md at build time).
+ *
+ * CONVENTIONS (apply to every call)
+ *  - All arrays and pointers are DEVICE memory unless marked (host).  int is
+ *    32-bit.  Matrices are column-major FP64.  Pivot indices are
+ *    1-based (LAPACK), local to each matrix.
+ *  - Required dimensions (host scalars, e.g. max_m) describe the operation for
+ *    the LARGEST matrix of the batch.  Local dimensions (device int
+ *    arrays m[], n[], k[]) describe each matrix and are never modified
+ *    (P:L129).  Pointer offsets (host scalars Xi, Xj) select the submatrix
+ *    X[id] = Xarray[id] + Xj*ldx[id] + Xi of every matrix.
+ *  - Dynamic Compute-Workload Inference, DCWI: every kernel
+ *    infers the actual per-matrix work from required dims, local dims and
+ *    offsets; a matrix with no remaining work does nothing.  There is no
+ *    per-matrix host loop anywhere in the library.
+ *  - Ownership: the caller owns ALL memory (matrices, pointer arrays, size
+ *    arrays, ipiv, info, workspace).  The library never allocates on the hot
+ *    path; its only state is a per-device property cache created on first use.
+ *    The caller-provided workspace keeps the calls asynchronous.
+ *  - Asynchrony: every call enqueues work on `stream` and returns without
+ *    synchronising, except irr_getrf / irr_getrf_partial when a required
+ *    dimension is passed as <= 0: then the library computes it with one device
+ *    reduction and one device-to-host copy (documented synchronisation).
+ *  - Return value: IRR_SUCCESS (0); -p if host argument p (1-based position in
+ *    the C signature) is invalid; IRR_ERR_* (> 0) for a workspace that is too
+ *    small, a launch failure or an unsupported device.  Per-matrix errors are
+ *    reported in info[] (see irr_getrf).
+ *  - Aliasing: matrices, ipiv arrays and workspace must not overlap.
+ *  - Device: compiled for sm_100a only (B200); any other device gives
+ *    IRR_ERR_DEVICE.
+ */
+#ifndef IRR_H
+#define IRR_H
+
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Opaque CUDA stream handle (binary-compatible with cudaStream_t). NULL is the
+ * legacy default stream. */
+typedef struct CUstream_st *irr_stream_t;
+
+typedef enum { IRR_NO_TRANS = 0, IRR_TRANS = 1 } irr_trans_t;
+typedef enum { IRR_LEFT = 0, IRR_RIGHT = 1 } irr_side_t;
+typedef enum { IRR_LOWER = 0, IRR_UPPER = 1 } irr_uplo_t;
+typedef enum { IRR_NON_UNIT = 0, IRR_UNIT = 1 } irr_diag_t;
+
+#define IRR_SUCCESS 0
+#define IRR_ERR_CUDA 1        /* a CUDA launch or API call failed              */
+#define IRR_ERR_WORKSPACE 2   /* work_bytes < the *_workspace_size() query     */
+#define IRR_ERR_UNSUPPORTED 3 /* size or option outside what this build does   */
+#define IRR_ERR_DEVICE 4      /* current device is not sm_100 (B200)           */
+
+/* ------------------------------------------------------------------------
+ * irr_getrf -- batched LU with partial pivoting on matrices of different
+ * sizes: P_i L_i U_i = A_i for every i (§III-B; irrLU).
+ *
+ *  batch        (host) number of matrices, >= 0.
+ *  max_m, max_n (host) required dims = max_i m[i], max_i n[i].
+ *               Must be >= every m[i], n[i]; matrices exceeding them get
+ *               info[i] = -1 / -2.  Pass <= 0 to have them computed (1 sync).
+ *  m, n         local dims, int[batch].
+ *  A            double*[batch]; A[i] points to an m[i] x n[i] column-major
+ *               matrix with leading dimension ld[i].  Overwritten
+ *               by L (unit lower, strictly below the diagonal) and U (upper,
+ *               including the diagonal).
+ *  ld           int[batch], ld[i] >= max(1, m[i]).
+ *  ipiv         int*[batch]; ipiv[i] -> int[min(m[i], n[i])]: row k (1-based
+ *               k+1) was interchanged with row ipiv[i][k] at step k.
+ *  info         int[batch] output.  0: success.  k > 0: U(k,k) (1-based) is an
+ *               exact zero; the factorization still completes (LAPACK).
+ *               -1 / -2 / -3 / -4 / -5: bad m[i] / n[i] / A[i] / ld[i] /
+ *               ipiv[i] (LAPACK argument positions); the matrix is skipped.
+ *  work         device workspace of >= irr_getrf_workspace_size(batch, max_m,
+ *               max_n) bytes, 256-byte aligned, caller-owned.
+ *  stream       CUDA stream; the call is asynchronous on it.
+ * Pivot search picks the largest |a_ik| with the smallest row index on ties
+ * (BLAS idamax).  Results of matrix i depend only on (m[i], n[i], A[i]), not
+ * on the rest of the batch.
+ * ---------------------------------------------------------------------- */
+size_t irr_getrf_workspace_size(int batch, int max_m, int max_n);
+int irr_getrf(int batch, int max_m, int max_n, const int *m, const int *n, double *const *A,
+              const int *ld, int *const *ipiv, int *info, void *work, size_t work_bytes,
+              irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * irr_getrf_partial -- partial factorization of a batch of frontal matrices
+ * F = [F11 F12; F21 F22] (multifrontal step, §III-A):
+ *      P L U <- LU(F11)              pivoting restricted to F11's rows
+ *      F12   <- U^-1 L^-1 P^T F12
+ *      F22   <- F22 - F21 F12        (Schur complement; F21 is NOT modified)
+ *  n1, n2       local dims, int[batch]: F11 n1 x n1, F12 n1 x n2, F21 n2 x n1,
+ *               F22 n2 x n2.  max_n1 / max_n2 (host) their maxima (<= 0: computed).
+ *  F11..F22     double*[batch] with leading dims ld11..ld22 (int[batch]); the
+ *               four blocks may be parts of one nf x nf front (ld = nf).
+ *  ipiv         int*[batch] -> int[n1[i]];  info int[batch] as for irr_getrf
+ *               (bad n1 -> -1, n2 -> -2, ld11 -> -4, ld12 -> -6, ld21 -> -8,
+ *               ld22 -> -10).  A zero pivot (info > 0) still runs the F12/F22
+ *               updates with IEEE inf/NaN semantics.
+ *  work         >= irr_getrf_partial_workspace_size(batch, max_n1, max_n2).
+ * ---------------------------------------------------------------------- */
+size_t irr_getrf_partial_workspace_size(int batch, int max_n1, int max_n2);
+int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const int *n2,
+                      double *const *F11, const int *ld11, double *const *F12, const int *ld12,
+                      const double *const *F21, const int *ld21, double *const *F22, const int *ld22,
+                      int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * irr_gemm -- irrGEMM (§IV-C) with the expanded interface:
+ *      C_i <- alpha op(A_i) op(B_i) + beta C_i      (beta == 0: C not read)
+ * Local dims: C_i is m[i] x n[i]; op(A_i) is m[i] x k[i]; op(B_i) is k[i] x n[i]
+ * (so A_i is stored m x k, or k x m when ta == IRR_TRANS).  Offsets select
+ * submatrices; DCWI clamps the required dims (max_m, max_n, max_k):
+ *   m_eff = min(max_m, m_i - rowoff(op A), m_i - Ci)
+ *   n_eff = min(max_n, n_i - coloff(op B), n_i - Cj)
+ *   k_eff = min(max_k, k_i - coloff(op A), k_i - rowoff(op B))
+ * where for op(A) = A^T the offsets (Ai, Aj) are compared against (k, m)
+ * instead of (m, k).  A matrix with m_eff <= 0 or n_eff <= 0 does
+ * nothing; k_eff <= 0 gives C <- beta C.
+ *  work / work_bytes: optional (may be NULL/0).  With a workspace of
+ *  irr_gemm_workspace_size(batch) bytes the tile schedule is built on the
+ *  device (balanced); without one, a DCWI grid over the required dims is used.
+ * ---------------------------------------------------------------------- */
+size_t irr_gemm_workspace_size(int batch);
+int irr_gemm(irr_trans_t ta, irr_trans_t tb, int max_m, int max_n, int max_k, const int *m, const int *n,
+             const int *k, double alpha, const double *const *A, int Ai, int Aj, const int *lda,
+             const double *const *B, int Bi, int Bj, const int *ldb, double beta, double *const *C, int Ci,
+             int Cj, const int *ldc, int batch, void *work, size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * irr_trsm -- irrTRSM (§IV-D): in-place triangular solve,
+ *      side = LEFT : op(T_i) X = alpha B_i      (T_i is m[i] x m[i])
+ *      side = RIGHT: X op(T_i) = alpha B_i      (T_i is n[i] x n[i])
+ * B_i (m[i] x n[i]) is overwritten by X.  uplo / diag describe the stored T;
+ * only that triangle is read (the diagonal is not read when diag = UNIT).
+ * Recursive on the required dims, the off-diagonal blocks being
+ * irrGEMM calls; DCWI clamps: left m_eff = min(max_m, m_i - Ti, m_i - Tj,
+ * m_i - Bi), n_eff = min(max_n, n_i - Bj); right symmetrically on n.
+ *  work: optional, as for irr_gemm (irr_trsm_workspace_size(batch)).
+ * ---------------------------------------------------------------------- */
+size_t irr_trsm_workspace_size(int batch);
+int irr_trsm(irr_side_t side, irr_uplo_t uplo, irr_trans_t trans, irr_diag_t diag, int max_m, int max_n,
+             const int *m, const int *n, double alpha, const double *const *T, int Ti, int Tj,
+             const int *ldt, double *const *B, int Bi, int Bj, const int *ldb, int batch, void *work,
+             size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * irr_laswp -- irrLASWP (§IV-F): row interchanges
+ *      for k = k1 .. k2-1:  swap rows k and ipiv[i][k]-1 of A_i
+ * (rows relative to the offset Ai), applied to the columns
+ * [Aj, Aj + min(max_n, n_i - Aj)) of A_i; k2 is clamped to kcount[i]
+ * (the length of ipiv[i]).  n[i] is the local column count of A_i; rows must
+ * exist (ipiv entries < lda rows are the caller's contract).  The composite
+ * permutation is "rehearsed" on an index vector first and the rows are then
+ * moved once each.
+ * ---------------------------------------------------------------------- */
+int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
+              const int *kcount, int *const *ipiv, int batch, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
+ * Tuning (tests only; defaults are fixed).  Keys: "nb" (tier-L panel width,
+ * 8..64), "tier_s" (1 = enable warp-per-matrix tier), "tier_m_max" (max m*n
+ * of the shared-memory tier, 0 disables it), "panel_rows" (max panel rows held
+ * in shared memory), "trsm_nb" (TRSM recursion leaf).  Unknown keys are ignored.
+ * irr_get_tuning returns the current value (-1 for an unknown key).
+ * ---------------------------------------------------------------------- */
+void irr_set_tuning(const char *key, int value);
+int irr_get_tuning(const char *key);
+void irr_reset_tuning(void);
+
+/* Number of kernels this library launched on the calling thread since the
+ * last reset (host-side count, used by the benchmark's gpu_launches). */
+long long irr_launch_count(int reset);
+
+/* ------------------------------------------------------------------------
+ * Per-kernel-class device timing (benchmark instrumentation).  While enabled
+ * every kernel the library launches is bracketed by two CUDA events on the
+ * stream it is launched on.  irr_profile_enable(n) creates a pool for n
+ * launches (0 disables and frees it); irr_profile_collect waits for the
+ * recorded events, writes the summed milliseconds and launch counts per class
+ * (arrays of nclass entries) and clears the record; returns the number of
+ * launches read, -1 on a CUDA error.  Class c is named by
+ * irr_profile_class_name(c); irr_profile_num_classes() gives the count.
+ * ---------------------------------------------------------------------- */
+int irr_profile_enable(int max_launches);
+int irr_profile_collect(double *ms, long long *launches, int nclass);
+int irr_profile_num_classes(void);
+const char *irr_profile_class_name(int c);
+
+const char *irr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* IRR_H */

@@ -251,3 +251,57 @@ def g2_dominant(seed: int, gid: int, m: int, n: int):
         ipiv[j] = p + 1
         cur[j], cur[p] = cur[p], cur[j]
     return A, ipiv
+
+
+# --------------------------------------------------------------------------
+# Packed batches: every matrix's values written straight into one flat
+# column-major buffer (matrix g at offsets[g], leading dimension ld[g]).
+# --------------------------------------------------------------------------
+def packed_offsets(ld, n, align: int = 32):
+    """Element offsets of each matrix in a flat buffer, starts aligned to
+    `align` elements (32 doubles = 256 B).  Returns (offsets, total)."""
+    ld = np.asarray(ld, dtype=np.int64)
+    n = np.asarray(n, dtype=np.int64)
+    sizes = ((ld * n + align - 1) // align) * align
+    offsets = np.zeros(len(sizes), dtype=np.int64)
+    if len(sizes) > 1:
+        np.cumsum(sizes[:-1], out=offsets[1:])
+    total = int(offsets[-1] + sizes[-1]) if len(sizes) else 0
+    return offsets, max(total, align)
+
+
+def fill_packed(seed: int, m, n, ld, offsets, out: np.ndarray, gid_base: int = 0, chunk: int = 1 << 24,
+                gids=None):
+    """Write uniform_values(seed, gid(g), m[g], n[g]) for every g into
+    out[offsets[g] + i + j*ld[g]] (vectorised over matrices, chunked), where
+    gid(g) = gids[g] if given, else gid_base + g."""
+    gid_of = (np.arange(len(m), dtype=np.int64) + gid_base) if gids is None else np.asarray(gids, dtype=np.int64)
+    m = np.asarray(m, dtype=np.int64)
+    n = np.asarray(n, dtype=np.int64)
+    ld = np.asarray(ld, dtype=np.int64)
+    offsets = np.asarray(offsets, dtype=np.int64)
+    cnt = m * n
+    g0 = 0
+    B = len(m)
+    while g0 < B:
+        # take matrices until ~chunk elements
+        csum = np.cumsum(cnt[g0:])
+        g1 = g0 + int(np.searchsorted(csum, chunk, side="right")) + 1
+        g1 = min(max(g1, g0 + 1), B)
+        gs = np.arange(g0, g1)
+        c = cnt[gs]
+        tot = int(c.sum())
+        if tot:
+            gid = np.repeat(gs, c)
+            starts = np.repeat(np.cumsum(c) - c, c)
+            e = np.arange(tot, dtype=np.int64) - starts           # i + j*m
+            keys = matrix_key(seed, gid_of[gid].astype(np.uint64))
+            with np.errstate(over="ignore"):
+                x = splitmix64(keys + e.astype(np.uint64))
+            vals = 2.0 * ((x >> np.uint64(11)).astype(np.float64) * (2.0 ** -53)) - 1.0
+            mm = m[gid]
+            j = e // np.maximum(mm, 1)
+            i = e - j * mm
+            out[offsets[gid] + i + j * ld[gid]] = vals
+        g0 = g1
+    return out

@@ -1,0 +1,140 @@
+"""Caller-side device storage for irregular batches (setup, not the method).
+
+The C ABI takes caller-owned device pointer arrays ("the array of
+pointers must exist in the GPU memory before the kernel is launched").  These
+helpers lay a batch out once in HBM and build those arrays:
+
+  * MatrixBatch: one flat float64 buffer, matrix i column-major with leading
+    dimension ld[i], every matrix starting on a 256-byte boundary; a flat int32
+    ipiv buffer; info[batch]; int32 size arrays; int64 pointer arrays.
+  * FrontBatch: one nf x nf block per front (ld = nf) with the four pointer
+    arrays F11 / F12 / F21 / F22 into it (SURVEY §8(d) C4 layout).
+
+Only torch is used here, for device memory and copies.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import irr
+
+ALIGN = 32  # elements (256 B)
+
+
+def _offsets(sizes: np.ndarray, align: int = ALIGN):
+    sizes = ((np.asarray(sizes, dtype=np.int64) + align - 1) // align) * align
+    off = np.zeros(len(sizes), dtype=np.int64)
+    if len(sizes) > 1:
+        np.cumsum(sizes[:-1], out=off[1:])
+    total = int(off[-1] + sizes[-1]) if len(sizes) else 0
+    return off, max(total, align)
+
+
+class MatrixBatch:
+    def __init__(self, m, n, ld=None, device="cuda", with_ipiv=True):
+        self.m_h = np.asarray(m, dtype=np.int64)
+        self.n_h = np.asarray(n, dtype=np.int64)
+        self.batch = len(self.m_h)
+        self.ld_h = np.maximum(1, self.m_h) if ld is None else np.asarray(ld, dtype=np.int64)
+        self.device = torch.device(device)
+        self.offsets, self.total = _offsets(self.ld_h * self.n_h)
+        self.data = torch.empty(self.total, dtype=torch.float64, device=self.device)
+        base = self.data.data_ptr()
+        self.ptr = torch.from_numpy(base + 8 * self.offsets).to(self.device)
+        self.m = torch.from_numpy(self.m_h.astype(np.int32)).to(self.device)
+        self.n = torch.from_numpy(self.n_h.astype(np.int32)).to(self.device)
+        self.ld = torch.from_numpy(self.ld_h.astype(np.int32)).to(self.device)
+        self.max_m = int(self.m_h.max()) if self.batch else 0
+        self.max_n = int(self.n_h.max()) if self.batch else 0
+        self.k_h = np.minimum(self.m_h, self.n_h)
+        if with_ipiv:
+            self.ipiv_off, ipiv_total = _offsets(self.k_h)
+            self.ipiv_data = torch.zeros(ipiv_total, dtype=torch.int32, device=self.device)
+            self.ipiv = torch.from_numpy(self.ipiv_data.data_ptr() + 4 * self.ipiv_off).to(self.device)
+        self.info = torch.zeros(max(1, self.batch), dtype=torch.int32, device=self.device)
+        self.work = None
+
+    # -- host <-> device (setup / verification helpers)
+    def host_buffer(self, pinned=False):
+        return torch.empty(self.total, dtype=torch.float64, pin_memory=pinned)
+
+    def matrix(self, i, flat_host: np.ndarray):
+        """View of matrix i (m x n, Fortran) inside a flat host copy of data."""
+        o, m, n, ld = int(self.offsets[i]), int(self.m_h[i]), int(self.n_h[i]), int(self.ld_h[i])
+        if m * n == 0:
+            return np.zeros((m, n), order="F")
+        return np.lib.stride_tricks.as_strided(flat_host[o:], shape=(m, n), strides=(8, 8 * ld))
+
+    def ipiv_of(self, i, ipiv_host: np.ndarray):
+        o, k = int(self.ipiv_off[i]), int(self.k_h[i])
+        return ipiv_host[o:o + k]
+
+    def workspace(self):
+        if self.work is None:
+            nb = irr.irr_getrf_workspace_size(self.batch, self.max_m, self.max_n)
+            self.work = torch.empty(max(256, nb), dtype=torch.uint8, device=self.device)
+        return self.work
+
+    def getrf(self, stream=None, max_m=None, max_n=None):
+        """irr_getrf on the whole batch (asynchronous on `stream`)."""
+        return irr.irr_getrf(self.batch, self.max_m if max_m is None else max_m,
+                             self.max_n if max_n is None else max_n, self.m, self.n, self.ptr, self.ld,
+                             self.ipiv, self.info, self.workspace(), stream)
+
+
+class FrontBatch:
+    """Fronts F = [F11 F12; F21 F22], one nf x nf block each (ld = nf)."""
+
+    def __init__(self, n1, n2, device="cuda"):
+        self.n1_h = np.asarray(n1, dtype=np.int64)
+        self.n2_h = np.asarray(n2, dtype=np.int64)
+        self.nf_h = self.n1_h + self.n2_h
+        self.batch = len(self.n1_h)
+        self.device = torch.device(device)
+        ldf = np.maximum(1, self.nf_h)
+        self.ld_h = ldf
+        self.offsets, self.total = _offsets(ldf * self.nf_h)
+        self.data = torch.empty(self.total, dtype=torch.float64, device=self.device)
+        base = self.data.data_ptr() + 8 * self.offsets
+        nf, a = self.nf_h, self.n1_h
+
+        def P(x):
+            return torch.from_numpy(np.asarray(x, dtype=np.int64)).to(self.device)
+
+        self.F11 = P(base)
+        self.F12 = P(base + 8 * a * ldf)
+        self.F21 = P(base + 8 * a)
+        self.F22 = P(base + 8 * (a + a * ldf))
+        ld32 = torch.from_numpy(ldf.astype(np.int32)).to(self.device)
+        self.ld11 = self.ld12 = self.ld21 = self.ld22 = ld32
+        self.n1 = torch.from_numpy(self.n1_h.astype(np.int32)).to(self.device)
+        self.n2 = torch.from_numpy(self.n2_h.astype(np.int32)).to(self.device)
+        self.max_n1 = int(self.n1_h.max()) if self.batch else 0
+        self.max_n2 = int(self.n2_h.max()) if self.batch else 0
+        self.ipiv_off, ipiv_total = _offsets(self.n1_h)
+        self.ipiv_data = torch.zeros(ipiv_total, dtype=torch.int32, device=self.device)
+        self.ipiv = P(self.ipiv_data.data_ptr() + 4 * self.ipiv_off)
+        self.info = torch.zeros(max(1, self.batch), dtype=torch.int32, device=self.device)
+        self.work = None
+
+    def front(self, i, flat_host: np.ndarray):
+        o, nf = int(self.offsets[i]), int(self.nf_h[i])
+        if nf == 0:
+            return np.zeros((0, 0), order="F")
+        return np.lib.stride_tricks.as_strided(flat_host[o:], shape=(nf, nf), strides=(8, 8 * max(1, nf)))
+
+    def ipiv_of(self, i, ipiv_host: np.ndarray):
+        o, k = int(self.ipiv_off[i]), int(self.n1_h[i])
+        return ipiv_host[o:o + k]
+
+    def workspace(self):
+        if self.work is None:
+            nb = irr.irr_getrf_partial_workspace_size(self.batch, self.max_n1, self.max_n2)
+            self.work = torch.empty(max(256, nb), dtype=torch.uint8, device=self.device)
+        return self.work
+
+    def getrf_partial(self, stream=None):
+        return irr.irr_getrf_partial(self.batch, self.max_n1, self.max_n2, self.n1, self.n2, self.F11, self.ld11,
+                                     self.F12, self.ld12, self.F21, self.ld21, self.F22, self.ld22, self.ipiv,
+                                     self.info, self.workspace(), stream)

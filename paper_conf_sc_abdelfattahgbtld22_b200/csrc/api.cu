@@ -1,0 +1,421 @@
+// api.cu -- the C ABI entry points (include/irr.h) and the host drivers.
+//
+// The host side only checks scalar arguments, carves the caller's workspace
+// and enqueues kernels; it never touches per-matrix data (the
+// expanded interface exists so that no pointer/size arithmetic runs on the
+// host).  The only host loop is over panel ITERATIONS of the largest matrix
+// (P:L167, L179).
+#include <cstring>
+#include <cstdlib>
+#include <mutex>
+#include <vector>
+
+#include "irr_internal.cuh"
+
+namespace irr {
+
+void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s);
+void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *tile_off, cudaStream_t s);
+void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
+                         const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s);
+size_t laswp_smem(int span);
+
+static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32};
+static Tuning g_tuning = g_default;
+Tuning &tuning() { return g_tuning; }
+
+long long &launch_counter() {
+    static thread_local long long c = 0;
+    return c;
+}
+
+// ---------------------------------------------------------------- profiling
+// Optional per-kernel-class device timing for the benchmark: each launch is
+// bracketed by two CUDA events on its own stream (pool created on enable,
+// never on the hot path).
+static bool g_prof = false;
+struct ProfRec { int cls; int ev0, ev1; };
+static std::vector<cudaEvent_t> g_events;
+static std::vector<ProfRec> g_recs;
+static size_t g_ev_used = 0;
+static std::vector<int> g_open;  // stack of open record indices
+
+bool prof_on() { return g_prof; }
+
+void prof_record(int cls, cudaStream_t s, bool begin) {
+    if (g_ev_used >= g_events.size()) return;  // pool exhausted: stop recording
+    if (begin) {
+        int e = (int)g_ev_used++;
+        cudaEventRecord(g_events[e], s);
+        g_recs.push_back({cls, e, -1});
+        g_open.push_back((int)g_recs.size() - 1);
+    } else {
+        if (g_open.empty()) return;
+        int r = g_open.back();
+        g_open.pop_back();
+        int e = (int)g_ev_used++;
+        cudaEventRecord(g_events[e], s);
+        g_recs[r].ev1 = e;
+    }
+}
+
+static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc"};
+
+struct DeviceInfo {
+    int sms = 0;
+    int major = 0, minor = 0;
+    size_t smem_optin = 0;
+};
+static DeviceInfo g_dev[64];
+static std::mutex g_dev_mu;
+
+static const DeviceInfo *device_info() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    DeviceInfo &d = g_dev[dev];
+    if (d.sms == 0) {
+        cudaDeviceProp p;
+        if (cudaGetDeviceProperties(&p, dev) != cudaSuccess) return nullptr;
+        d.sms = p.multiProcessorCount;
+        d.major = p.major;
+        d.minor = p.minor;
+        d.smem_optin = p.sharedMemPerBlockOptin;
+    }
+    return &d;
+}
+
+int num_sms() {
+    const DeviceInfo *d = device_info();
+    return d ? d->sms : 148;
+}
+
+static int check_device() {
+    const DeviceInfo *d = device_info();
+    if (!d) return IRR_ERR_CUDA;
+    if (d->major != 10 || d->minor != 0) return IRR_ERR_DEVICE;  // built for sm_100a only
+    return IRR_SUCCESS;
+}
+
+// ---------------------------------------------------------------- workspace
+struct Work {
+    int *counters;
+    int *bins;
+    int *tile_off;
+};
+
+static size_t work_bytes_for(int batch) {
+    size_t b = (size_t)(batch > 0 ? batch : 1);
+    return align256(CNT_INTS * sizeof(int)) + align256(NBINS * b * sizeof(int)) + align256((b + 1) * sizeof(int));
+}
+
+static Work carve(void *work, int batch) {
+    size_t b = (size_t)(batch > 0 ? batch : 1);
+    char *p = (char *)work;
+    Work w;
+    w.counters = (int *)p;
+    p += align256(CNT_INTS * sizeof(int));
+    w.bins = (int *)p;
+    p += align256(NBINS * b * sizeof(int));
+    w.tile_off = (int *)p;
+    return w;
+}
+
+static int resolve_max_dims(int batch, int &max_m, int &max_n, const int *m, const int *n, int *counters,
+                            cudaStream_t s) {
+    if (max_m > 0 && max_n > 0) return IRR_SUCCESS;
+    IRR_CUDA_TRY(cudaMemsetAsync(counters, 0, CNT_INTS * sizeof(int), s));
+    launch_max_dims(batch, m, n, counters, s);
+    int h[2];
+    IRR_CUDA_TRY(cudaMemcpyAsync(h, counters + CNT_MAXM, 2 * sizeof(int), cudaMemcpyDeviceToHost, s));
+    IRR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (max_m <= 0) max_m = h[0];
+    if (max_n <= 0) max_n = h[1];
+    return IRR_SUCCESS;
+}
+
+// Enqueue the whole getrf machinery for the (already validated) args.
+static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cudaStream_t s) {
+    IRR_CUDA_TRY(cudaMemsetAsync(w.counters, 0, CNT_INTS * sizeof(int), s));
+    launch_classify(a, w.counters, w.bins, keep_neg_info, s);
+    if (a.max_m <= 0 || a.max_n <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+    const Tuning &t = tuning();
+    // which tiers can be populated, from the required dims alone
+    const long long big = (long long)mid_lds(a.max_m) * a.max_n;
+    const bool only_s = t.tier_s && a.max_m <= 32 && a.max_n <= 32;
+    if (t.tier_s) launch_lu_small(a, w.counters, w.bins, s);
+    if (!only_s) {
+        const long long mmax = t.tier_m_max;
+        if (mmax > 0) {
+            launch_lu_mid(a, w.counters, w.bins, BIN_M1, (int)(mmax < M1_ELEMS ? mmax : M1_ELEMS), s);
+            if (big > M1_ELEMS && mmax > M1_ELEMS)
+                launch_lu_mid(a, w.counters, w.bins, BIN_M2, (int)(mmax < M2_ELEMS ? mmax : M2_ELEMS), s);
+            if (big > M2_ELEMS && mmax > M2_ELEMS) launch_lu_mid(a, w.counters, w.bins, BIN_M3, (int)mmax, s);
+        }
+        if (big > mmax) launch_lu_large(a, w.counters, w.bins, w.tile_off, s);
+    }
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+}  // namespace irr
+
+using namespace irr;
+
+extern "C" {
+
+const char *irr_version(void) { return "irrlu-b200 0.1 (sm_100a)"; }
+
+int irr_profile_enable(int max_launches) {
+    for (cudaEvent_t e : g_events) cudaEventDestroy(e);
+    g_events.clear();
+    g_recs.clear();
+    g_open.clear();
+    g_ev_used = 0;
+    g_prof = max_launches > 0;
+    if (!g_prof) return IRR_SUCCESS;
+    g_events.resize((size_t)max_launches * 2);
+    for (auto &e : g_events)
+        if (cudaEventCreate(&e) != cudaSuccess) { g_prof = false; return IRR_ERR_CUDA; }
+    return IRR_SUCCESS;
+}
+
+int irr_profile_collect(double *ms, long long *launches, int nclass) {
+    for (int c = 0; c < nclass; ++c) { ms[c] = 0.0; launches[c] = 0; }
+    int n = 0;
+    for (const ProfRec &r : g_recs) {
+        if (r.ev1 < 0 || r.cls >= nclass) continue;
+        if (cudaEventSynchronize(g_events[r.ev1]) != cudaSuccess) return -1;
+        float t = 0.f;
+        cudaEventElapsedTime(&t, g_events[r.ev0], g_events[r.ev1]);
+        ms[r.cls] += t;
+        launches[r.cls] += 1;
+        ++n;
+    }
+    g_recs.clear();
+    g_open.clear();
+    g_ev_used = 0;
+    return n;
+}
+
+int irr_profile_num_classes(void) { return NKCLASS; }
+
+const char *irr_profile_class_name(int c) { return (c >= 0 && c < NKCLASS) ? k_names[c] : ""; }
+
+long long irr_launch_count(int reset) {
+    long long c = launch_counter();
+    if (reset) launch_counter() = 0;
+    return c;
+}
+
+void irr_set_tuning(const char *key, int value) {
+    if (!key) return;
+    if (!strcmp(key, "nb")) g_tuning.nb = value < 1 ? 1 : (value > 64 ? 64 : value);
+    else if (!strcmp(key, "tier_s")) g_tuning.tier_s = value ? 1 : 0;
+    else if (!strcmp(key, "tier_m_max")) g_tuning.tier_m_max = value < 0 ? 0 : (value > TIER_M_MAX_DEFAULT ? TIER_M_MAX_DEFAULT : value);
+    else if (!strcmp(key, "panel_rows")) g_tuning.panel_rows = value < 0 ? 0 : value;
+    else if (!strcmp(key, "trsm_nb")) g_tuning.trsm_nb = value < 1 ? 1 : (value > 32 ? 32 : value);
+}
+
+int irr_get_tuning(const char *key) {
+    if (!key) return -1;
+    if (!strcmp(key, "nb")) return g_tuning.nb;
+    if (!strcmp(key, "tier_s")) return g_tuning.tier_s;
+    if (!strcmp(key, "tier_m_max")) return g_tuning.tier_m_max;
+    if (!strcmp(key, "panel_rows")) return g_tuning.panel_rows;
+    if (!strcmp(key, "trsm_nb")) return g_tuning.trsm_nb;
+    return -1;
+}
+
+void irr_reset_tuning(void) { g_tuning = g_default; }
+
+size_t irr_getrf_workspace_size(int batch, int max_m, int max_n) {
+    (void)max_m; (void)max_n;
+    return work_bytes_for(batch);
+}
+
+int irr_getrf(int batch, int max_m, int max_n, const int *m, const int *n, double *const *A, const int *ld,
+              int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream) {
+    if (batch < 0) return -1;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!m) return -4;
+    if (!n) return -5;
+    if (!A) return -6;
+    if (!ld) return -7;
+    if (!ipiv) return -8;
+    if (!info) return -9;
+    if (!work) return -10;
+    if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    Work w = carve(work, batch);
+    rc = resolve_max_dims(batch, max_m, max_n, m, n, w.counters, s);
+    if (rc) return rc;
+    GetrfArgs a{batch, max_m, max_n, m, n, A, ld, ipiv, info};
+    return getrf_core(a, w, 0, s);
+}
+
+size_t irr_getrf_partial_workspace_size(int batch, int max_n1, int max_n2) {
+    (void)max_n1; (void)max_n2;
+    return work_bytes_for(batch);
+}
+
+int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const int *n2, double *const *F11,
+                      const int *ld11, double *const *F12, const int *ld12, const double *const *F21,
+                      const int *ld21, double *const *F22, const int *ld22, int *const *ipiv, int *info, void *work,
+                      size_t work_bytes, irr_stream_t stream) {
+    if (batch < 0) return -1;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!n1) return -4;
+    if (!n2) return -5;
+    if (!F11) return -6;
+    if (!ld11) return -7;
+    if (!F12) return -8;
+    if (!ld12) return -9;
+    if (!F21) return -10;
+    if (!ld21) return -11;
+    if (!F22) return -12;
+    if (!ld22) return -13;
+    if (!ipiv) return -14;
+    if (!info) return -15;
+    if (!work) return -16;
+    if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    Work w = carve(work, batch);
+    rc = resolve_max_dims(batch, max_n1, max_n2, n1, n2, w.counters, s);
+    if (rc) return rc;
+    if (max_n1 > 0 && laswp_smem(max_n1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
+    launch_partial_validate(batch, max_n1, max_n2, n1, n2, ld11, ld12, ld21, ld22, F11, F12, F21, F22, ipiv, info, s);
+    // step 1: P L U <- LU(F11), pivoting restricted to F11
+    GetrfArgs a{batch, max_n1, max_n1, n1, n1, F11, ld11, ipiv, info};
+    rc = getrf_core(a, w, 1, s);
+    if (rc) return rc;
+    if (max_n1 <= 0 || max_n2 <= 0) return IRR_SUCCESS;
+    // step 2: F12 <- U^-1 L^-1 P^T F12: irrLASWP + 2 x irrTRSM (GETRS)
+    launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s);
+    TrsmArgs t{};
+    t.side = IRR_LEFT; t.uplo = IRR_LOWER; t.trans = IRR_NO_TRANS; t.diag = IRR_UNIT;
+    t.max_m = max_n1; t.max_n = max_n2; t.m = n1; t.n = n2; t.alpha = 1.0;
+    t.T = (const double *const *)F11; t.Ti = 0; t.Tj = 0; t.ldt = ld11;
+    t.B = F12; t.Bi = 0; t.Bj = 0; t.ldb = ld12; t.batch = batch;
+    run_trsm_masked(t, info, w.counters, w.tile_off, s);
+    t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
+    run_trsm_masked(t, info, w.counters, w.tile_off, s);
+    // step 3: F22 <- F22 - F21 F12, F21 untouched
+    GemmArgs g{};
+    g.ta = 0; g.tb = 0; g.max_m = max_n2; g.max_n = max_n2; g.max_k = max_n1;
+    g.m = n2; g.n = n2; g.k = n1; g.alpha = -1.0; g.beta = 1.0;
+    g.A = F21; g.Ai = 0; g.Aj = 0; g.lda = ld21;
+    g.B = (const double *const *)F12; g.Bi = 0; g.Bj = 0; g.ldb = ld12;
+    g.C = F22; g.Ci = 0; g.Cj = 0; g.ldc = ld22; g.batch = batch;
+    launch_gemm_masked(g, info, w.counters, w.tile_off, s);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+size_t irr_gemm_workspace_size(int batch) { return work_bytes_for(batch); }
+
+int irr_gemm(irr_trans_t ta, irr_trans_t tb, int max_m, int max_n, int max_k, const int *m, const int *n,
+             const int *k, double alpha, const double *const *A, int Ai, int Aj, const int *lda,
+             const double *const *B, int Bi, int Bj, const int *ldb, double beta, double *const *C, int Ci, int Cj,
+             const int *ldc, int batch, void *work, size_t work_bytes, irr_stream_t stream) {
+    if (ta != IRR_NO_TRANS && ta != IRR_TRANS) return -1;
+    if (tb != IRR_NO_TRANS && tb != IRR_TRANS) return -2;
+    if (max_m < 0) return -3;
+    if (max_n < 0) return -4;
+    if (max_k < 0) return -5;
+    if (Ai < 0) return -11;
+    if (Aj < 0) return -12;
+    if (Bi < 0) return -15;
+    if (Bj < 0) return -16;
+    if (Ci < 0) return -20;
+    if (Cj < 0) return -21;
+    if (batch < 0) return -23;
+    if (batch == 0 || max_m == 0 || max_n == 0) return IRR_SUCCESS;
+    if (!m) return -6;
+    if (!n) return -7;
+    if (!k) return -8;
+    if (!A) return -10;
+    if (!lda) return -13;
+    if (!B) return -14;
+    if (!ldb) return -17;
+    if (!C) return -19;
+    if (!ldc) return -22;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    int *tile_off = nullptr;
+    if (work) {
+        if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+        tile_off = carve(work, batch).tile_off;
+    }
+    GemmArgs g{(int)ta, (int)tb, max_m, max_n, max_k, m, n, k, alpha, beta, A, Ai, Aj, lda, B, Bi, Bj, ldb,
+               C, Ci, Cj, ldc, batch};
+    launch_gemm_masked(g, nullptr, nullptr, tile_off, s);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+size_t irr_trsm_workspace_size(int batch) { return work_bytes_for(batch); }
+
+int irr_trsm(irr_side_t side, irr_uplo_t uplo, irr_trans_t trans, irr_diag_t diag, int max_m, int max_n,
+             const int *m, const int *n, double alpha, const double *const *T, int Ti, int Tj, const int *ldt,
+             double *const *B, int Bi, int Bj, const int *ldb, int batch, void *work, size_t work_bytes,
+             irr_stream_t stream) {
+    if (side != IRR_LEFT && side != IRR_RIGHT) return -1;
+    if (uplo != IRR_LOWER && uplo != IRR_UPPER) return -2;
+    if (trans != IRR_NO_TRANS && trans != IRR_TRANS) return -3;
+    if (diag != IRR_NON_UNIT && diag != IRR_UNIT) return -4;
+    if (max_m < 0) return -5;
+    if (max_n < 0) return -6;
+    if (Ti < 0) return -11;
+    if (Tj < 0) return -12;
+    if (Bi < 0) return -15;
+    if (Bj < 0) return -16;
+    if (batch < 0) return -18;
+    if (batch == 0 || max_m == 0 || max_n == 0) return IRR_SUCCESS;
+    if (!m) return -7;
+    if (!n) return -8;
+    if (!T) return -10;
+    if (!ldt) return -13;
+    if (!B) return -14;
+    if (!ldb) return -17;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    int *tile_off = nullptr, *counters = nullptr;
+    if (work) {
+        if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+        Work w = carve(work, batch);
+        tile_off = w.tile_off;
+        counters = w.counters;
+    }
+    TrsmArgs t{(int)side, (int)uplo, (int)trans, (int)diag, max_m, max_n, m, n, alpha, T, Ti, Tj, ldt,
+               B, Bi, Bj, ldb, batch};
+    run_trsm_masked(t, nullptr, counters, tile_off, s);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
+              const int *kcount, int *const *ipiv, int batch, irr_stream_t stream) {
+    if (max_n < 0) return -1;
+    if (Ai < 0) return -4;
+    if (Aj < 0) return -5;
+    if (k1 < 0) return -7;
+    if (k2 < k1) return -8;
+    if (batch < 0) return -11;
+    if (batch == 0 || max_n == 0 || k2 == k1) return IRR_SUCCESS;
+    if (!n) return -2;
+    if (!A) return -3;
+    if (!lda) return -6;
+    if (!kcount) return -9;
+    if (!ipiv) return -10;
+    if (laswp_smem(k2 - k1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
+    int rc = check_device();
+    if (rc) return rc;
+    launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, (cudaStream_t)stream);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+}  // extern "C"

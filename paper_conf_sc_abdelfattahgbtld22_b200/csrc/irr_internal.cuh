@@ -1,0 +1,169 @@
+// irr_internal.cuh -- device/host internals shared by the libirr kernels.
+// (Product code only; the CPU oracle under oracle/ shares nothing with this.)
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <float.h>
+
+#include "irr.h"
+
+namespace irr {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+// ---------------------------------------------------------------- tuning
+struct Tuning {
+    int nb;          // tier-L panel width ("typically 16-32 columns")
+    int tier_s;      // 1: warp-per-matrix tier for m, n <= 32
+    int tier_m_max;  // max padded m*n (doubles) of the shared-memory tier
+    int panel_rows;  // max rows of a tier-L panel staged in shared memory
+    int trsm_nb;     // TRSM recursion leaf (<= 32)
+};
+Tuning &tuning();
+
+// host-side launch counter (per thread)
+long long &launch_counter();
+inline void count_launch(int k = 1) { launch_counter() += k; }
+
+// kernel classes for the optional per-class device timing (irr_profile_*)
+enum KClass {
+    K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, NKCLASS
+};
+void prof_record(int cls, cudaStream_t s, bool begin);
+bool prof_on();
+// RAII scope around one kernel launch: counts it and, when profiling is on,
+// brackets it with CUDA events on its stream.
+struct KScope {
+    int cls;
+    cudaStream_t s;
+    KScope(int c, cudaStream_t st) : cls(c), s(st) {
+        if (prof_on()) prof_record(cls, s, true);
+    }
+    ~KScope() {
+        if (prof_on()) prof_record(cls, s, false);
+        count_launch();
+    }
+};
+
+// ---------------------------------------------------------------- bins
+// Size classes of irr_getrf (a pure function of (m_i, n_i), SURVEY §7 hard
+// part 7): S = warp per matrix; M1..M3 = CTA per matrix with the whole matrix
+// in shared memory (three footprints so small ones pack several CTAs per SM);
+// L = blocked right-looking LU with one kernel chain per panel iteration.
+enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, NBINS = 5 };
+constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
+constexpr int M2_ELEMS = 12288;   // 96 KB  -> 2 CTAs / SM
+constexpr int TIER_M_MAX_DEFAULT = 24576;  // 192 KB -> 1 CTA / SM
+
+// shared-memory leading dimension of a tier-M matrix: odd, so row-wise
+// accesses of consecutive columns fall in different banks
+__host__ __device__ inline int mid_lds(int m) { return m | 1; }
+
+// counters block at the head of every workspace (ints)
+constexpr int CNT_INTS = 64;
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10 };
+
+inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
+
+// ---------------------------------------------------------------- device helpers
+__device__ __forceinline__ unsigned long long dkey(double absv) {
+    return (unsigned long long)__double_as_longlong(absv);
+}
+
+// Warp arg-max of (key, row) over lanes with cand == true: the largest key,
+// ties -> the smallest row (BLAS idamax).  Keys are the bit
+// patterns of non-negative doubles, so integer order == value order.
+// Returns row = -1 if no lane is a candidate.
+__device__ __forceinline__ void warp_argmax(bool cand, unsigned long long key, int row,
+                                            unsigned long long &kout, int &rout) {
+    unsigned hi = cand ? (unsigned)(key >> 32) : 0u;
+    unsigned lo = cand ? (unsigned)(key & 0xffffffffu) : 0u;
+    unsigned mhi = __reduce_max_sync(FULL, hi);
+    bool e1 = cand && hi == mhi;
+    unsigned mlo = __reduce_max_sync(FULL, e1 ? lo : 0u);
+    bool e2 = e1 && lo == mlo;
+    unsigned r = __reduce_min_sync(FULL, e2 ? (unsigned)row : 0xffffffffu);
+    kout = ((unsigned long long)mhi << 32) | mlo;
+    rout = (int)r;  // 0xffffffff -> -1
+}
+
+// Pivot scaling as LAPACK dgetf2: multiply by the reciprocal when
+// |pivot| >= sfmin, else divide (the tolerance absorbs the 1 ulp).
+struct PivotScale {
+    double pv, rcp;
+    bool use_rcp;
+    __device__ __forceinline__ explicit PivotScale(double p) : pv(p) {
+        use_rcp = fabs(p) >= DBL_MIN;
+        rcp = use_rcp ? __drcp_rn(p) : 0.0;
+    }
+    __device__ __forceinline__ double operator()(double v) const { return use_rcp ? v * rcp : v / pv; }
+};
+
+__device__ __forceinline__ int imin(int a, int b) { return a < b ? a : b; }
+__device__ __forceinline__ int imax(int a, int b) { return a > b ? a : b; }
+
+// ---------------------------------------------------------------- launchers (host)
+struct GetrfArgs {
+    int batch, max_m, max_n;
+    const int *m, *n;
+    double *const *A;
+    const int *ld;
+    int *const *ipiv;
+    int *info;
+};
+
+// classify.cu
+void launch_classify(const GetrfArgs &a, int *counters, int *bins, int keep_neg_info, cudaStream_t s);
+void launch_max_dims(int batch, const int *m, const int *n, int *counters, cudaStream_t s);
+
+// lu_small.cu
+void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s);
+// lu_mid.cu
+void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
+                   cudaStream_t s);
+// lu_large.cu
+void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s);
+
+// gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)
+struct GemmArgs {
+    int ta, tb, max_m, max_n, max_k;
+    const int *m, *n, *k;
+    double alpha, beta;
+    const double *const *A; int Ai, Aj; const int *lda;
+    const double *const *B; int Bi, Bj; const int *ldb;
+    double *const *C; int Ci, Cj; const int *ldc;
+    int batch;
+};
+void launch_gemm_dcwi(const GemmArgs &g, int *counters, int *tile_off, cudaStream_t s);
+
+// trsm_vb.cu
+struct TrsmArgs {
+    int side, uplo, trans, diag, max_m, max_n;
+    const int *m, *n;
+    double alpha;
+    const double *const *T; int Ti, Tj; const int *ldt;
+    double *const *B; int Bi, Bj; const int *ldb;
+    int batch;
+};
+void run_trsm(const TrsmArgs &t, int *counters, int *tile_off, cudaStream_t s);
+
+// laswp_vb.cu
+void launch_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
+                  const int *kcount, int *const *ipiv, int batch, cudaStream_t s);
+
+// partial.cu
+void launch_partial_validate(int batch, int max_n1, int max_n2, const int *n1, const int *n2,
+                             const int *ld11, const int *ld12, const int *ld21, const int *ld22,
+                             double *const *F11, double *const *F12, const double *const *F21,
+                             double *const *F22, int *const *ipiv, int *info, cudaStream_t s);
+
+int num_sms();
+}  // namespace irr
+
+#define IRR_CUDA_TRY(x)                                  \
+    do {                                                 \
+        cudaError_t e__ = (x);                           \
+        if (e__ != cudaSuccess) return IRR_ERR_CUDA;     \
+    } while (0)

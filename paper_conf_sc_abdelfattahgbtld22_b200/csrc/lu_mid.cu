@@ -1,0 +1,121 @@
+// lu_mid.cu -- tier M: one CTA per matrix, the whole matrix resident in shared
+// memory.
+//
+// The fused irrGETF2 panel is only worthwhile while the data fits in
+// shared memory ("the advantage ... is saving memory traffic"; the
+// 192 KB of the A100 vs 64 KB of the MI100 decided the switch).  On
+// B200 (227 KB per CTA) the whole matrix fits for m*n <= 24,576, so the full
+// blocked right-looking LU (Fig. 1) runs on chip: A is read once and
+// written once.  Per panel of NBM columns: fused panel (panel.cuh), in-place
+// TRSM of the U12 row block, register-tiled GEMM update of the trailing
+// matrix, all in shared memory.
+#include "panel.cuh"
+
+namespace irr {
+
+constexpr int M_NT = 256;
+constexpr int NBM = 16;
+
+__global__ void __launch_bounds__(M_NT) lu_mid_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                      const int *__restrict__ bins, int bin) {
+    extern __shared__ __align__(16) double s[];
+    __shared__ PanelScratch sc;
+    __shared__ int piv_s[NBM];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    constexpr int NW = M_NT / 32;
+    const int count = counters[CNT_BIN0 + bin];
+    const int *list = bins + (size_t)bin * a.batch;
+    for (int t = blockIdx.x; t < count; t += gridDim.x) {
+        const int i = list[t];
+        const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
+        double *__restrict__ gA = a.A[i];
+        const int lds = mid_lds(mi);
+        // ---- load (coalesced along columns)
+        for (int c = warp; c < ni; c += NW)
+            for (int r = lane; r < mi; r += 32) s[r + c * lds] = gA[r + (size_t)c * ld];
+        __syncthreads();
+        const int K = mi < ni ? mi : ni;
+        int info = 0;
+        int *gipiv = a.ipiv[i];
+        for (int j = 0; j < K; j += NBM) {
+            const int ib = K - j < NBM ? K - j : NBM;
+            // ---- fused panel, interchanges applied to the full rows
+            int z = panel_getf2<M_NT>(s, lds, j, mi, j, ib, 0, ni, piv_s, sc);
+            if (z && !info) info = j + z;
+            if (tid < ib) gipiv[j + tid] = piv_s[tid] + 1;
+            const int c1 = j + ib;
+            if (c1 >= ni) continue;
+            // ---- U12 <- L11^-1 A12 (unit lower, in place), one thread per column
+            for (int cc = c1 + tid; cc < ni; cc += M_NT) {
+                double x[NBM];
+#pragma unroll
+                for (int q = 0; q < NBM; ++q) x[q] = (q < ib) ? s[j + q + cc * lds] : 0.0;
+#pragma unroll
+                for (int q = 0; q < NBM; ++q) {
+#pragma unroll
+                    for (int r = q + 1; r < NBM; ++r)
+                        if (r < ib) x[r] = fma(-s[j + r + (j + q) * lds], x[q], x[r]);
+                }
+#pragma unroll
+                for (int q = 0; q < NBM; ++q)
+                    if (q < ib) s[j + q + cc * lds] = x[q];
+            }
+            __syncthreads();
+            // ---- A22 -= L21 * U12 : warp tiles of 64 rows x 4 columns,
+            //      lane owns rows (lane, lane + 32) of the tile
+            const int Mr = mi - c1, Nc = ni - c1;
+            if (Mr > 0) {
+                const int nrt = (Mr + 63) >> 6, nct = (Nc + 3) >> 2;
+                for (int item = warp; item < nrt * nct; item += NW) {
+                    const int tr = item % nrt, tc = item / nrt;
+                    const int r0 = c1 + tr * 64 + lane, cb = c1 + tc * 4;
+                    const bool v0 = r0 < mi, v1 = r0 + 32 < mi;
+                    double acc[2][4] = {{0, 0, 0, 0}, {0, 0, 0, 0}};
+                    for (int kk = 0; kk < ib; ++kk) {
+                        const double *Lc = s + (j + kk) * lds;
+                        double a0 = v0 ? Lc[r0] : 0.0, a1 = v1 ? Lc[r0 + 32] : 0.0;
+#pragma unroll
+                        for (int p = 0; p < 4; ++p) {
+                            double b = (cb + p < ni) ? s[j + kk + (cb + p) * lds] : 0.0;
+                            acc[0][p] = fma(a0, b, acc[0][p]);
+                            acc[1][p] = fma(a1, b, acc[1][p]);
+                        }
+                    }
+#pragma unroll
+                    for (int p = 0; p < 4; ++p) {
+                        if (cb + p < ni) {
+                            if (v0) s[r0 + (cb + p) * lds] -= acc[0][p];
+                            if (v1) s[r0 + 32 + (cb + p) * lds] -= acc[1][p];
+                        }
+                    }
+                }
+            }
+            __syncthreads();
+        }
+        // ---- store
+        for (int c = warp; c < ni; c += NW)
+            for (int r = lane; r < mi; r += 32) gA[r + (size_t)c * ld] = s[r + c * lds];
+        if (tid == 0) a.info[i] = info;
+        __syncthreads();
+    }
+}
+
+void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
+                   cudaStream_t s) {
+    size_t smem = (size_t)max_elems * sizeof(double);
+    static size_t attr_max = 0;  // the attribute is per function: keep the largest
+    if (smem > attr_max) {
+        cudaFuncSetAttribute(lu_mid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr_max = smem;
+    }
+    int per_sm = (int)(200 * 1024 / (smem + 4096));
+    if (per_sm < 1) per_sm = 1;
+    if (per_sm > 8) per_sm = 8;
+    int grid = num_sms() * per_sm;
+    if (grid > a.batch) grid = a.batch;
+    if (grid < 1) grid = 1;
+    KScope k(K_LU_MID, s);
+    lu_mid_kernel<<<grid, M_NT, smem, s>>>(a, counters, bins, bin);
+}
+
+}  // namespace irr

@@ -1,0 +1,39 @@
+// partial.cu -- argument validation of the partial front factorization
+// (§III-A); the steps themselves are composed in api.cu from the
+// getrf tiers, irrLASWP, irrTRSM and irrGEMM.
+#include "irr_internal.cuh"
+
+namespace irr {
+
+__global__ void partial_validate_kernel(int batch, int max_n1, int max_n2, const int *n1, const int *n2,
+                                        const int *ld11, const int *ld12, const int *ld21, const int *ld22,
+                                        double *const *F11, double *const *F12, const double *const *F21,
+                                        double *const *F22, int *const *ipiv, int *info) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= batch) return;
+    const int a = n1[i], b = n2[i];
+    int e = 0;
+    if (a < 0 || a > max_n1) e = -1;
+    else if (b < 0 || b > max_n2) e = -2;
+    else if (a > 0 && F11[i] == nullptr) e = -3;
+    else if (ld11[i] < (a > 1 ? a : 1)) e = -4;
+    else if (a > 0 && b > 0 && F12[i] == nullptr) e = -5;
+    else if (ld12[i] < (a > 1 ? a : 1)) e = -6;
+    else if (a > 0 && b > 0 && F21[i] == nullptr) e = -7;
+    else if (ld21[i] < (b > 1 ? b : 1)) e = -8;
+    else if (b > 0 && F22[i] == nullptr) e = -9;
+    else if (ld22[i] < (b > 1 ? b : 1)) e = -10;
+    else if (a > 0 && ipiv[i] == nullptr) e = -11;
+    info[i] = e;
+}
+
+void launch_partial_validate(int batch, int max_n1, int max_n2, const int *n1, const int *n2, const int *ld11,
+                             const int *ld12, const int *ld21, const int *ld22, double *const *F11,
+                             double *const *F12, const double *const *F21, double *const *F22, int *const *ipiv,
+                             int *info, cudaStream_t s) {
+    KScope k(K_MISC, s);
+    partial_validate_kernel<<<(batch + 255) / 256, 256, 0, s>>>(batch, max_n1, max_n2, n1, n2, ld11, ld12, ld21,
+                                                               ld22, F11, F12, F21, F22, ipiv, info);
+}
+
+}  // namespace irr

@@ -1,0 +1,53 @@
+"""Flop-balanced sharding of an irregular batch over the GPUs of one box
+(north_star: "fronts are partitioned flop-balanced across the GPUs ... with
+NCCL over NVLink used only to gather per-matrix info/pivot status").
+
+Host-side bookkeeping only: the matrices are independent, so the only data-
+path exchange is the final gather of the per-matrix status words.
+"""
+from __future__ import annotations
+
+import heapq
+
+import numpy as np
+
+
+def lpt_partition(work, parts: int) -> np.ndarray:
+    """Longest-processing-time-first greedy: items sorted by decreasing work,
+    each given to the currently least-loaded part (ties -> lowest part id).
+    Returns owner[i] in [0, parts).  Deterministic."""
+    work = np.asarray(work, dtype=np.float64)
+    owner = np.zeros(len(work), dtype=np.int64)
+    if parts <= 1 or len(work) == 0:
+        return owner
+    order = np.lexsort((np.arange(len(work)), -work))   # by work desc, then index asc
+    heap = [(0.0, p) for p in range(parts)]
+    heapq.heapify(heap)
+    for i in order:
+        load, p = heapq.heappop(heap)
+        owner[i] = p
+        heapq.heappush(heap, (load + work[i], p))
+    return owner
+
+
+def shard_indices(work, parts: int, rank: int) -> np.ndarray:
+    """Global indices owned by `rank`, in ascending order."""
+    return np.nonzero(lpt_partition(work, parts) == rank)[0]
+
+
+def imbalance(work, owner, parts: int) -> float:
+    """max part load / mean part load (1.0 = perfect)."""
+    loads = np.bincount(owner, weights=np.asarray(work, dtype=np.float64), minlength=parts)
+    mean = loads.mean()
+    return float(loads.max() / mean) if mean > 0 else 1.0
+
+
+def merge_status(gathered: np.ndarray, shards) -> np.ndarray:
+    """Scatter the gathered per-rank status rows back to global order.
+    gathered: [parts, pad] array (row r = rank r's status words, padded);
+    shards: list of index arrays (rank r's global indices)."""
+    total = sum(len(s) for s in shards)
+    out = np.zeros(total, dtype=gathered.dtype)
+    for r, idx in enumerate(shards):
+        out[idx] = gathered[r, : len(idx)]
+    return out

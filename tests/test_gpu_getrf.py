@@ -1,0 +1,188 @@
+"""GPU parity of irr_getrf (through the C ABI) against the CPU oracle.
+
+Covers every tier (S: warp per matrix, M: CTA with the matrix in shared
+memory, L: blocked right-looking with panel / swap+TRSM / GEMM kernels), the
+size edge cases of SURVEY §8(c) ("Sizes the unit tests must cover"), ld > m,
+bad arguments, exact families (bit-exact) and the configs of BASELINE.json.
+"""
+import numpy as np
+import pytest
+
+import irrgen
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from gpu_util import check_getrf, gpu_getrf  # noqa: E402
+from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _reset_tuning():
+    irr.irr_reset_tuning()
+    yield
+    irr.irr_reset_tuning()
+
+
+EDGE = [0, 1, 2, 3, 7, 8, 15, 16, 17, 31, 32, 33, 63, 64, 65, 127, 128, 129]
+
+
+def _uniform(shapes, seed=77):
+    return [irrgen.uniform_values(seed, g, m, n) for g, (m, n) in enumerate(shapes)]
+
+
+def _run_and_check(mats, exact=False, **kw):
+    LUs, ipivs, info, _ = gpu_getrf(mats, **kw)
+    stats = {}
+    for g, (A, LU, ip, inf) in enumerate(zip(mats, LUs, ipivs, info)):
+        st = check_getrf(A, LU, ip, int(inf), exact=exact, label=f"#{g} {A.shape}")
+        stats[st] = stats.get(st, 0) + 1
+    return stats
+
+
+def test_c1_parity():
+    """configs[0]: 100 square matrices n ~ U{1..32} (tier S)."""
+    cfg = irrgen.config("C1")
+    mats = [irrgen.uniform_values(cfg.seed, g, int(m), int(n)) for g, (m, n) in enumerate(zip(cfg.m, cfg.n))]
+    st = _run_and_check(mats)
+    assert st.get("match", 0) >= 98
+
+
+def test_edge_shapes_all_tiers():
+    shapes = [(m, n) for m in EDGE for n in EDGE]
+    st = _run_and_check(_uniform(shapes))
+    assert st.get("match", 0) + st.get("empty", 0) >= len(shapes) - 2
+
+
+def test_tier_m_boundary_and_extreme_shapes():
+    # m * n around the tier-M limit (padded m*n <= 24576) and very thin shapes
+    shapes = [(151, 162), (151, 163), (153, 160), (160, 153), (96, 256), (256, 96), (97, 256),
+              (1, 1024), (1024, 1), (33, 1), (1, 33), (300, 7), (7, 300), (1000, 30), (30, 1000)]
+    _run_and_check(_uniform(shapes, seed=5))
+
+
+@pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
+def test_tier_l_forced_small_nb(nb):
+    """Force everything through the tier-L chain: nb-1, nb, nb+1, 2nb+-1 sizes."""
+    irr.irr_set_tuning("tier_s", 0)
+    irr.irr_set_tuning("tier_m_max", 0)
+    irr.irr_set_tuning("nb", nb)
+    sizes = sorted({1, 2, nb - 1, nb, nb + 1, 2 * nb - 1, 2 * nb + 1, 3 * nb + 2} - {0})
+    shapes = [(a, b) for a in sizes for b in sizes] + [(70, 45), (45, 70)]
+    _run_and_check(_uniform(shapes, seed=nb))
+
+
+def test_e1_replica_dcwi():
+    """P:L167 Fig. 4: three matrices, the largest 15x15, nb = 5, three
+    iterations; the second iteration sees full, partial and no work."""
+    irr.irr_set_tuning("tier_s", 0)
+    irr.irr_set_tuning("tier_m_max", 0)
+    irr.irr_set_tuning("nb", 5)
+    mats = _uniform([(15, 15), (8, 8), (4, 4)], seed=15)
+    _run_and_check(mats)
+    A, L, U, ipiv, _ = irrgen.g1_exact(1, 1, 15, 15)
+    B, _, _, _, _ = irrgen.g1_exact(1, 2, 8, 8)
+    Cm, _, _, _, _ = irrgen.g1_exact(1, 3, 4, 4)
+    _run_and_check([A, B, Cm], exact=True)
+
+
+def test_panel_in_global_memory():
+    """Tall panels that do not fit shared memory take the in-place path."""
+    irr.irr_set_tuning("panel_rows", 40)
+    mats = _uniform([(300, 200), (200, 300), (257, 257), (100, 100)], seed=9)
+    _run_and_check(mats)
+
+
+@pytest.mark.parametrize("tier", ["default", "L"])
+def test_g1_exact_bitexact(tier):
+    """G1: bit-exact L, U, ipiv in any arithmetic order."""
+    if tier == "L":
+        irr.irr_set_tuning("tier_s", 0)
+        irr.irr_set_tuning("tier_m_max", 0)
+    shapes = [(1, 1), (5, 5), (32, 32), (32, 17), (17, 32), (33, 33), (64, 20), (20, 64), (130, 130),
+              (150, 160), (257, 100), (100, 257), (300, 300)]
+    mats = [irrgen.g1_exact(3, g, m, n)[0] for g, (m, n) in enumerate(shapes)]
+    _run_and_check(mats, exact=True)
+
+
+def test_g1_singular_info():
+    cases = [(6, 6, 0), (6, 6, 2), (32, 32, 31), (100, 100, 99), (64, 40, 17), (40, 64, 39), (300, 300, 150)]
+    mats = [irrgen.g1_singular(4, g, m, n, c)[0] for g, (m, n, c) in enumerate(cases)]
+    LUs, ipivs, info, _ = gpu_getrf(mats)
+    for (m, n, c), A, LU, ip, inf in zip(cases, mats, LUs, ipivs, info):
+        assert inf == c + 1
+        check_getrf(A, LU, ip, int(inf), exact=True, label=f"sing {m}x{n}@{c}")
+
+
+def test_g2_dominant_ipiv():
+    shapes = [(1, 1), (5, 5), (32, 32), (64, 64), (300, 40), (40, 300), (256, 255), (200, 200), (500, 500)]
+    for g, (m, n) in enumerate(shapes):
+        A, ipiv = irrgen.g2_dominant(9, g, m, n)
+        LUs, ipivs, info, _ = gpu_getrf([A])
+        assert np.array_equal(ipivs[0], ipiv), (m, n)
+        check_getrf(A, LUs[0], ipivs[0], int(info[0]), label=f"G2 {m}x{n}")
+
+
+def test_g5_closed_forms():
+    mats = [np.array([[3.5]]), np.array([[0.0]]), np.array([[0.5], [-3.0], [3.0], [1.0]]),
+            np.array([[2.0, -1.0, 7.0]]), np.eye(9), np.eye(5)[[3, 0, 4, 1, 2]], np.zeros((4, 6)),
+            np.zeros((40, 40)), np.eye(200)]
+    _run_and_check(mats, exact=True)
+
+
+@pytest.mark.parametrize("extra", [1, 7])
+def test_leading_dimension(extra):
+    shapes = [(5, 5), (31, 20), (64, 64), (100, 150), (300, 280)]
+    _run_and_check(_uniform(shapes, seed=extra), ld_extra=extra)
+
+
+def test_bad_arguments_are_skipped():
+    """info < 0 for bad local dims; neighbours are unaffected."""
+    mats = _uniform([(10, 10), (20, 20), (40, 30), (5, 5)], seed=3)
+    m = [10, 20, 40, 5]
+    n = [10, 20, 30, 5]
+    m_bad = list(m)
+    m_bad[1] = -3                       # bad m -> -1
+    LUs, ipivs, info, _ = gpu_getrf(mats, m=m_bad, n=n, max_m=40, max_n=30)
+    assert info[1] == -1
+    for g in (0, 2, 3):
+        check_getrf(mats[g], LUs[g], ipivs[g], int(info[g]))
+    # larger than the required dims -> -1 / -2
+    LUs, ipivs, info, _ = gpu_getrf(mats, max_m=30, max_n=30)
+    assert info[2] == -1 and info[0] == 0
+
+
+def test_required_dims_computed_on_device():
+    mats = _uniform([(10, 12), (50, 40), (3, 3)], seed=8)
+    LUs, ipivs, info, _ = gpu_getrf(mats, max_m=0, max_n=0)
+    for A, LU, ip, inf in zip(mats, LUs, ipivs, info):
+        check_getrf(A, LU, ip, int(inf))
+
+
+def test_results_independent_of_batch_composition():
+    """SURVEY §7 hard part 7 / G8: a matrix factors bitwise identically alone
+    and inside a mixed batch (tier choice is a function of (m, n) only)."""
+    shapes = [(20, 20), (100, 90), (300, 300), (7, 31)]
+    mats = _uniform(shapes, seed=21)
+    together, ip_t, _, _ = gpu_getrf(mats + _uniform([(256, 256)] * 3, seed=22))
+    for g, A in enumerate(mats):
+        alone, ip_a, _, _ = gpu_getrf([A])
+        assert np.array_equal(alone[0], together[g]) and np.array_equal(ip_a[0], ip_t[g])
+
+
+def test_c2_scaled_parity():
+    """configs[1] shape (mixed square / rectangular, dims U{1..256}) on a 1/10 sample, every matrix."""
+    cfg = irrgen.config("C2", scale=0.1)
+    mats = [irrgen.uniform_values(cfg.seed, g, int(m), int(n)) for g, (m, n) in enumerate(zip(cfg.m, cfg.n))]
+    st = _run_and_check(mats)
+    assert st.get("match", 0) >= len(mats) - 3
+
+
+def test_c3_sample_parity():
+    """configs[2] shape (square U{256..1024}), a sample of 12 matrices."""
+    cfg = irrgen.config("C3", scale=0.006)
+    mats = [irrgen.uniform_values(cfg.seed, g, int(m), int(n)) for g, (m, n) in enumerate(zip(cfg.m, cfg.n))]
+    _run_and_check(mats)
