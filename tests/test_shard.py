@@ -1,0 +1,79 @@
+"""Host logic of the multi-GPU path: LPT flop-balanced
+partition and the status gather, exercised with world_size 2 over gloo on CPU."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import irrgen
+from paper_conf_sc_abdelfattahgbtld22_b200 import flops as F
+from paper_conf_sc_abdelfattahgbtld22_b200.shard import imbalance, lpt_partition, merge_status, shard_indices
+
+
+def test_lpt_is_a_partition_and_balanced():
+    cfg = irrgen.config("C5", scale=0.1)           # 20,000 fronts, heavy tail
+    w = F.getrf_flops(cfg.m, cfg.n)
+    for parts in (1, 2, 4, 8):
+        owner = lpt_partition(w, parts)
+        assert owner.min() >= 0 and owner.max() < parts
+        shards = [shard_indices(w, parts, r) for r in range(parts)]
+        allidx = np.sort(np.concatenate(shards))
+        assert np.array_equal(allidx, np.arange(len(w)))
+        assert imbalance(w, owner, parts) < 1.01
+    # deterministic
+    assert np.array_equal(lpt_partition(w, 8), lpt_partition(w, 8))
+
+
+def test_lpt_small_cases():
+    assert list(lpt_partition([5, 4, 3, 3, 3], 2)) == [0, 1, 1, 0, 1]   # loads 8 / 10 -> LPT greedy
+    assert list(lpt_partition([], 3)) == []
+    assert list(lpt_partition([1.0], 4)) == [0]
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    cfg = irrgen.config("C2", scale=0.2 * world)
+    w = F.getrf_flops(cfg.m, cfg.n)
+    owner = lpt_partition(w, world)
+    mine = np.nonzero(owner == rank)[0]
+    pad = int(np.bincount(owner, minlength=world).max())
+    # per-matrix status word of this rank (here a deterministic stand-in: the global id)
+    status = torch.full((pad,), -7, dtype=torch.int64)
+    status[: len(mine)] = torch.from_numpy(mine)
+    gathered = torch.zeros(world * pad, dtype=torch.int64)
+    dist.all_gather_into_tensor(gathered, status)
+    t = torch.tensor([float(rank + 1)], dtype=torch.float64)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)       # max-over-ranks timing reduction
+    if rank == 0:
+        shards = [np.nonzero(owner == r)[0] for r in range(world)]
+        merged = merge_status(gathered.view(world, pad).numpy(), shards)
+        q.put((merged.tolist(), float(t.item()), len(w)))
+    dist.destroy_process_group()
+
+
+def test_gloo_two_ranks_gather_and_merge():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    merged, tmax, total = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert merged == list(range(total))           # every matrix's word lands at its global id
+    assert tmax == 2.0
