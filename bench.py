@@ -99,11 +99,15 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ per-tier algorithmic work
-def tier_of(m, n, tier_m_max=24576):
+def tier_of(m, n, tier_m_max=24576, l1=True):
+    """0 = S (warp), 1 = M (CTA, in smem), 2 = L1 (CTA per matrix), 3 = L2
+    (grid-wide chain), -1 = empty; mirrors classify.cu."""
     m = np.asarray(m)
     n = np.asarray(n)
     lds = m | 1
-    t = np.full(len(m), 2)
+    t = np.full(len(m), 3)
+    if l1:
+        t[m <= 256] = 2
     t[(lds * n) <= tier_m_max] = 1
     t[(m <= 32) & (n <= 32)] = 0
     t[(m == 0) | (n == 0)] = -1
@@ -117,10 +121,10 @@ def class_work(m, n, nb=32):
     n = np.asarray(n, dtype=np.int64)
     t = tier_of(m, n)
     out = {}
-    for cls, tier in (("lu_small", 0), ("lu_mid", 1)):
+    for cls, tier in (("lu_small", 0), ("lu_mid", 1), ("lu_l1", 2)):
         sel = t == tier
         out[cls] = (float(F.getrf_flops(m[sel], n[sel]).sum()), float(F.getrf_bytes(m[sel], n[sel]).sum()))
-    sel = t == 2
+    sel = t == 3
     mL, nL = m[sel], n[sel]
     g_f = g_b = p_f = p_b = s_f = s_b = 0.0
     kL = np.minimum(mL, nL)

@@ -20,7 +20,7 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s);
 size_t laswp_smem(int span);
 
-static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32};
+static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -60,7 +60,7 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 }
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
-                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc"};
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1"};
 
 struct DeviceInfo {
     int sms = 0;
@@ -153,7 +153,10 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
                 launch_lu_mid(a, w.counters, w.bins, BIN_M2, (int)(mmax < M2_ELEMS ? mmax : M2_ELEMS), s);
             if (big > M2_ELEMS && mmax > M2_ELEMS) launch_lu_mid(a, w.counters, w.bins, BIN_M3, (int)mmax, s);
         }
-        if (big > mmax) launch_lu_large(a, w.counters, w.bins, w.tile_off, s);
+        if (big > mmax) {
+            if (t.l1) launch_lu_l1(a, w.counters, w.bins, s);
+            if (!t.l1 || a.max_m > L1_MAX_ROWS) launch_lu_large(a, w.counters, w.bins, w.tile_off, s);
+        }
     }
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
@@ -215,6 +218,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "tier_m_max")) g_tuning.tier_m_max = value < 0 ? 0 : (value > TIER_M_MAX_DEFAULT ? TIER_M_MAX_DEFAULT : value);
     else if (!strcmp(key, "panel_rows")) g_tuning.panel_rows = value < 0 ? 0 : value;
     else if (!strcmp(key, "trsm_nb")) g_tuning.trsm_nb = value < 1 ? 1 : (value > 32 ? 32 : value);
+    else if (!strcmp(key, "l1")) g_tuning.l1 = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -224,6 +228,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "tier_m_max")) return g_tuning.tier_m_max;
     if (!strcmp(key, "panel_rows")) return g_tuning.panel_rows;
     if (!strcmp(key, "trsm_nb")) return g_tuning.trsm_nb;
+    if (!strcmp(key, "l1")) return g_tuning.l1;
     return -1;
 }
 

@@ -9,15 +9,19 @@
 // for the largest matrix with most CTAs idle.
 //
 // FP64 on sm_100a: tcgen05 has no f64 kind (SURVEY §7 hard part 4); the
-// tensor path would be mma.sync DMMA whose peak equals the DFMA pipe.  This
-// core uses DFMA with a 4x4 register tile per thread (64x64 CTA tile, K chunk
-// 16, double-buffered shared memory).
+// tensor path would be mma.sync DMMA whose nominal peak equals the DFMA pipe.
+// This core uses DFMA: 64x64 CTA tile, 128 threads, 8x4 register tile per
+// thread (12 shared-memory wavefronts per 32 DFMA, below the 1:2 ratio the
+// SM sustains), operands staged by cp.async in K chunks of 16 with double
+// buffering, the C tile staged asynchronously, and the next tile's first
+// chunk prefetched while the current tile computes.
 #pragma once
 #include "irr_internal.cuh"
 
 namespace irr {
 
-constexpr int GBM = 64, GBN = 64, GBK = 16, G_NT = 256;
+constexpr int GBM = 64, GBN = 64, GBK = 16, G_NT = 128;
+constexpr int GPAD = GBM + 1;
 
 struct GemmDesc {
     const double *A; long lda; int ta;
@@ -28,102 +32,124 @@ struct GemmDesc {
 };
 
 struct GemmSmem {
-    double As[2][GBK][GBM + 1];
-    double Bs[2][GBK][GBN + 1];
+    double As[2][GBK][GPAD];
+    double Bs[2][GBK][GPAD];
+    double Cs[GBN][GPAD];
 };
+constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
-__device__ __forceinline__ void gemm_load_chunk(const GemmDesc &d, int r0, int c0, int k0, double (*As)[GBM + 1],
-                                                double (*Bs)[GBN + 1], double ra[4], double rb[4]) {
+// Issue the cp.async copies of K chunk [k0, k0+16) of tile (r0, c0) into buffer
+// `buf` (out-of-range elements are zero-filled with plain stores).
+__device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int c0, int k0, GemmSmem &sm, int buf) {
     const int tid = threadIdx.x;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+    for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int r, kk;
         if (!d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
         const int gr = r0 + r, gk = k0 + kk;
-        double v = 0.0;
-        if (gr < d.m && gk < d.k) v = d.ta ? d.A[gk + (size_t)gr * d.lda] : d.A[gr + (size_t)gk * d.lda];
-        ra[q] = v;
+        double *dst = &sm.As[buf][kk][r];
+        if (gr < d.m && gk < d.k) cp_async8(dst, d.ta ? d.A + gk + (size_t)gr * d.lda : d.A + gr + (size_t)gk * d.lda);
+        else *dst = 0.0;
     }
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
+    for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int c, kk;
         if (!d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
         const int gc = c0 + c, gk = k0 + kk;
-        double v = 0.0;
-        if (gc < d.n && gk < d.k) v = d.tb ? d.B[gc + (size_t)gk * d.ldb] : d.B[gk + (size_t)gc * d.ldb];
-        rb[q] = v;
+        double *dst = &sm.Bs[buf][kk][c];
+        if (gc < d.n && gk < d.k) cp_async8(dst, d.tb ? d.B + gc + (size_t)gk * d.ldb : d.B + gk + (size_t)gc * d.ldb);
+        else *dst = 0.0;
     }
-    (void)As; (void)Bs;
 }
 
-__device__ __forceinline__ void gemm_store_chunk(const GemmDesc &d, double (*As)[GBM + 1], double (*Bs)[GBN + 1],
-                                                 const double ra[4], const double rb[4]) {
+__device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, GemmSmem &sm) {
+    if (d.beta == 0.0) return;
     const int tid = threadIdx.x;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int e = tid + G_NT * q;
-        int r, kk;
-        if (!d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
-        As[kk][r] = ra[q];
-    }
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int e = tid + G_NT * q;
-        int c, kk;
-        if (!d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
-        Bs[kk][c] = rb[q];
+    const int mr = imin(GBM, d.m - r0), nc = imin(GBN, d.n - c0);
+    for (int e = tid; e < GBM * GBN; e += G_NT) {
+        const int r = e & 63, c = e >> 6;
+        if (r < mr && c < nc) cp_async8(&sm.Cs[c][r], d.C + r0 + r + (size_t)(c0 + c) * d.ldc);
     }
 }
 
-// One 64x64 output tile at (r0, c0) of problem d:  C <- alpha op(A) op(B) + beta C
-// (beta == 0: C is not read).  All G_NT threads participate.
-__device__ __forceinline__ void gemm_tile(const GemmDesc &d, int r0, int c0, GemmSmem &sm) {
-    const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-    double acc[4][4];
+__device__ __forceinline__ void gemm_compute_chunk(const GemmSmem &sm, int buf, double acc[8][4]) {
+    const int tid = threadIdx.x, tx = tid & 7, ty = tid >> 3;
 #pragma unroll
-    for (int q = 0; q < 4; ++q)
+    for (int kk = 0; kk < GBK; ++kk) {
+        double a[8], b[4];
 #pragma unroll
-        for (int p = 0; p < 4; ++p) acc[q][p] = 0.0;
-    double ra[4], rb[4];
-    int buf = 0;
-    if (d.k > 0) {
-        gemm_load_chunk(d, r0, c0, 0, sm.As[0], sm.Bs[0], ra, rb);
-        gemm_store_chunk(d, sm.As[0], sm.Bs[0], ra, rb);
+        for (int q = 0; q < 8; ++q) a[q] = sm.As[buf][kk][tx + 8 * q];
+#pragma unroll
+        for (int p = 0; p < 4; ++p) b[p] = sm.Bs[buf][kk][ty + 16 * p];
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+#pragma unroll
+            for (int p = 0; p < 4; ++p) acc[q][p] = fma(a[q], b[p], acc[q][p]);
     }
-    __syncthreads();
-    for (int k0 = 0; k0 < d.k; k0 += GBK) {
-        const bool has_next = k0 + GBK < d.k;
-        if (has_next) gemm_load_chunk(d, r0, c0, k0 + GBK, sm.As[buf ^ 1], sm.Bs[buf ^ 1], ra, rb);
-#pragma unroll
-        for (int kk = 0; kk < GBK; ++kk) {
-            double a[4], b[4];
-#pragma unroll
-            for (int q = 0; q < 4; ++q) a[q] = sm.As[buf][kk][tx + 16 * q];
-#pragma unroll
-            for (int p = 0; p < 4; ++p) b[p] = sm.Bs[buf][kk][ty + 16 * p];
-#pragma unroll
-            for (int q = 0; q < 4; ++q)
-#pragma unroll
-                for (int p = 0; p < 4; ++p) acc[q][p] = fma(a[q], b[p], acc[q][p]);
-        }
-        if (has_next) gemm_store_chunk(d, sm.As[buf ^ 1], sm.Bs[buf ^ 1], ra, rb);
-        __syncthreads();
-        buf ^= 1;
-    }
+}
+
+__device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0, const GemmSmem &sm, double acc[8][4]) {
+    const int tid = threadIdx.x, tx = tid & 7, ty = tid >> 3;
 #pragma unroll
     for (int p = 0; p < 4; ++p) {
-        const int c = c0 + ty + 16 * p;
+        const int cl = ty + 16 * p, c = c0 + cl;
         if (c >= d.n) continue;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            const int r = r0 + tx + 16 * q;
+        for (int q = 0; q < 8; ++q) {
+            const int rl = tx + 8 * q, r = r0 + rl;
             if (r >= d.m) continue;
-            double *cp = d.C + r + (size_t)c * d.ldc;
-            *cp = (d.beta == 0.0) ? d.alpha * acc[q][p] : d.alpha * acc[q][p] + d.beta * *cp;
+            double v = d.alpha * acc[q][p];
+            if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
+            d.C[r + (size_t)c * d.ldc] = v;
         }
     }
+}
+
+// A stream of tiles processed by one CTA with the software pipeline described
+// above.  `next(d, r0, c0)` returns false when the CTA has no more tiles.
+template <class Next>
+__device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
+    GemmDesc d, dn;
+    int r0, c0, rn, cn;
+    if (!next(d, r0, c0)) return;
+    int buf = 0;
+    if (d.k > 0) gemm_issue_chunk(d, r0, c0, 0, sm, buf);
+    cp_async_commit();
+    bool have = true;
+    while (have) {
+        gemm_issue_c(d, r0, c0, sm);
+        cp_async_commit();
+        double acc[8][4];
+#pragma unroll
+        for (int q = 0; q < 8; ++q)
+#pragma unroll
+            for (int p = 0; p < 4; ++p) acc[q][p] = 0.0;
+        const int nchunks = (d.k + GBK - 1) / GBK;
+        bool has_next_tile = false;
+        for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
+            if (c + 1 < nchunks) {
+                gemm_issue_chunk(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
+            } else {
+                has_next_tile = next(dn, rn, cn);
+                if (has_next_tile && dn.k > 0) gemm_issue_chunk(dn, rn, cn, 0, sm, buf ^ 1);
+            }
+            cp_async_commit();
+            if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();
+            __syncthreads();
+            if (nchunks > 0) gemm_compute_chunk(sm, buf, acc);
+            __syncthreads();
+            buf ^= 1;
+        }
+        cp_async_wait<1>();
+        __syncthreads();
+        gemm_epilogue(d, r0, c0, sm, acc);
+        __syncthreads();
+        have = has_next_tile;
+        if (have) { d = dn; r0 = rn; c0 = cn; }
+    }
+    cp_async_wait<0>();
 }
 
 __device__ __forceinline__ int gemm_tiles_of(const GemmDesc &d) {
@@ -176,9 +202,10 @@ __global__ void __launch_bounds__(1024) gemm_scan_kernel(Prob P, int count, cons
 }
 
 template <class Prob>
-__global__ void __launch_bounds__(G_NT) gemm_sched_kernel(Prob P, int count, const int *count_ptr,
+__global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, const int *count_ptr,
                                                           const int *__restrict__ tile_off) {
-    __shared__ GemmSmem sm;
+    extern __shared__ __align__(16) unsigned char g_smem[];
+    GemmSmem &sm = *reinterpret_cast<GemmSmem *>(g_smem);
     if (count < 0) count = *count_ptr;
     if (count <= 0) return;
     const int total = tile_off[count];
@@ -186,47 +213,69 @@ __global__ void __launch_bounds__(G_NT) gemm_sched_kernel(Prob P, int count, con
     const int t_begin = (int)((long long)blockIdx.x * total / G);
     const int t_end = (int)((long long)(blockIdx.x + 1) * total / G);
     if (t_begin >= t_end) return;
-    // first slot b with tile_off[b] <= t_begin < tile_off[b+1]
+    // last slot b with tile_off[b] <= t_begin (the one whose range holds t_begin)
     int lo = 0, hi = count - 1;
     while (lo < hi) {
         int mid = (lo + hi + 1) >> 1;
         if (tile_off[mid] <= t_begin) lo = mid; else hi = mid - 1;
     }
-    int b = lo;
-    GemmDesc d;
-    P.get(b, d);
-    int b_end = tile_off[b + 1];
-    for (int t = t_begin; t < t_end; ++t) {
+    int b = lo, t = t_begin;
+    GemmDesc cur;
+    P.get(b, cur);
+    int b_beg = tile_off[b], b_end = tile_off[b + 1];
+    auto next = [&](GemmDesc &d, int &r0, int &c0) -> bool {
+        if (t >= t_end) return false;
         while (t >= b_end) {
             ++b;
-            P.get(b, d);
+            P.get(b, cur);
+            b_beg = tile_off[b];
             b_end = tile_off[b + 1];
         }
-        const int local = t - tile_off[b];
-        const int ntm = (d.m + GBM - 1) / GBM;
-        const int tm = local % ntm, tn = local / ntm;
-        gemm_tile(d, tm * GBM, tn * GBN, sm);
-        __syncthreads();
-    }
+        const int local = t - b_beg;
+        const int ntm = (cur.m + GBM - 1) / GBM;
+        r0 = (local % ntm) * GBM;
+        c0 = (local / ntm) * GBN;
+        d = cur;
+        ++t;
+        return true;
+    };
+    gemm_tile_stream(next, sm);
 }
 
 // DCWI-grid fallback (no workspace): virtual tiles over the required dims,
-// empty ones exit immediately ("If no workload is detected, the
+// empty ones are skipped ("If no workload is detected, the
 // corresponding GPU threads perform no work at all").
 template <class Prob>
-__global__ void __launch_bounds__(G_NT) gemm_grid_kernel(Prob P, int count, int tiles_m, int tiles_n) {
-    __shared__ GemmSmem sm;
+__global__ void __launch_bounds__(G_NT, 3) gemm_grid_kernel(Prob P, int count, int tiles_m, int tiles_n) {
+    extern __shared__ __align__(16) unsigned char g_smem[];
+    GemmSmem &sm = *reinterpret_cast<GemmSmem *>(g_smem);
     const long long per = (long long)tiles_m * tiles_n;
     const long long total = per * count;
-    for (long long w = blockIdx.x; w < total; w += gridDim.x) {
-        const int b = (int)(w / per);
-        const int local = (int)(w - (long long)b * per);
-        GemmDesc d;
-        if (!P.get(b, d)) continue;
-        const int tm = local % tiles_m, tn = local / tiles_m;
-        if (tm * GBM >= d.m || tn * GBN >= d.n) continue;
-        gemm_tile(d, tm * GBM, tn * GBN, sm);
-        __syncthreads();
+    long long w = blockIdx.x;
+    auto next = [&](GemmDesc &d, int &r0, int &c0) -> bool {
+        for (; w < total; w += gridDim.x) {
+            const int b = (int)(w / per);
+            const int local = (int)(w - (long long)b * per);
+            if (!P.get(b, d)) continue;
+            const int tm = local % tiles_m, tn = local / tiles_m;
+            if (tm * GBM >= d.m || tn * GBN >= d.n) continue;
+            r0 = tm * GBM;
+            c0 = tn * GBN;
+            w += gridDim.x;
+            return true;
+        }
+        return false;
+    };
+    gemm_tile_stream(next, sm);
+}
+
+// opt-in to > 48 KB dynamic shared memory once per kernel instantiation
+template <class K>
+inline void gemm_smem_optin(K kernel) {
+    static bool done = false;
+    if (!done) {
+        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)GEMM_SMEM);
+        done = true;
     }
 }
 

@@ -48,14 +48,16 @@ void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *
             gemm_scan_kernel<DcwiGemmProb><<<1, 1024, 0, s>>>(P, g.batch, nullptr, tile_off);
         }
         KScope k(K_GEMM_DCWI, s);
-        gemm_sched_kernel<DcwiGemmProb><<<sms * 2, G_NT, 0, s>>>(P, g.batch, nullptr, tile_off);
+        gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb>);
+        gemm_sched_kernel<DcwiGemmProb><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, g.batch, nullptr, tile_off);
     } else {
         const int tm = (g.max_m + GBM - 1) / GBM, tn = (g.max_n + GBN - 1) / GBN;
         long long total = (long long)tm * tn * g.batch;
         int grid = sms * 4;
         if (total < grid) grid = (int)total;
         KScope k(K_GEMM_DCWI, s);
-        gemm_grid_kernel<DcwiGemmProb><<<grid, G_NT, 0, s>>>(P, g.batch, tm, tn);
+        gemm_smem_optin(gemm_grid_kernel<DcwiGemmProb>);
+        gemm_grid_kernel<DcwiGemmProb><<<grid, G_NT, GEMM_SMEM, s>>>(P, g.batch, tm, tn);
     }
     (void)counters;
 }

@@ -19,6 +19,7 @@ struct Tuning {
     int tier_m_max;  // max padded m*n (doubles) of the shared-memory tier
     int panel_rows;  // max rows of a tier-L panel staged in shared memory
     int trsm_nb;     // TRSM recursion leaf (<= 32)
+    int l1;          // 1: CTA-per-matrix tier for tier-L matrices with m <= L1_MAX_ROWS
 };
 Tuning &tuning();
 
@@ -29,7 +30,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();
@@ -52,7 +53,10 @@ struct KScope {
 // part 7): S = warp per matrix; M1..M3 = CTA per matrix with the whole matrix
 // in shared memory (three footprints so small ones pack several CTAs per SM);
 // L = blocked right-looking LU with one kernel chain per panel iteration.
-enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, NBINS = 5 };
+// L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
+// kernels per panel iteration.
+enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, NBINS = 6 };
+constexpr int L1_MAX_ROWS = 256;
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
 constexpr int M2_ELEMS = 12288;   // 96 KB  -> 2 CTAs / SM
 constexpr int TIER_M_MAX_DEFAULT = 24576;  // 192 KB -> 1 CTA / SM
@@ -63,7 +67,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10 };
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11 };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
@@ -104,6 +108,47 @@ struct PivotScale {
 __device__ __forceinline__ int imin(int a, int b) { return a < b ? a : b; }
 __device__ __forceinline__ int imax(int a, int b) { return a > b ? a : b; }
 
+// ---------------------------------------------------------------- async staging
+// cp.async (LDGSTS): global -> shared without registers, so a whole matrix
+// or panel is in flight at once instead of one dependent load per iteration.
+__device__ __forceinline__ void cp_async8(void *smem, const void *gmem) {
+    unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+    unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+
+// Copy an m x n column-major block (leading dim ld) into shared memory with
+// leading dim lds, issued by `nthr` threads starting at thread `t0`
+// (cooperative).  Uses 16-byte copies when the block is one contiguous,
+// 16-byte aligned range in both spaces, else 8-byte copies per element.
+__device__ __forceinline__ void stage_block_async(double *s, int lds, const double *g, long ld, int m, int n,
+                                                  int t, int nthr) {
+    const int total = m * n;
+    if (ld == m && lds == m) {
+        const bool al = ((((uintptr_t)s) | ((uintptr_t)g)) & 15) == 0;
+        if (al) {
+            const int pairs = total >> 1;
+            for (int e = t; e < pairs; e += nthr) cp_async16(s + 2 * e, g + 2 * e);
+            if ((total & 1) && t == 0) cp_async8(s + total - 1, g + total - 1);
+        } else {
+            for (int e = t; e < total; e += nthr) cp_async8(s + e, g + e);
+        }
+    } else {
+        for (int e = t; e < total; e += nthr) {
+            const int c = e / m, r = e - c * m;
+            cp_async8(s + r + c * lds, g + r + (size_t)c * ld);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- launchers (host)
 struct GetrfArgs {
     int batch, max_m, max_n;
@@ -125,6 +170,7 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
                    cudaStream_t s);
 // lu_large.cu
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s);
+void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)
 struct GemmArgs {

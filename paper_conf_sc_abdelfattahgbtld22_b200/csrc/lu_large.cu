@@ -1,17 +1,24 @@
 // lu_large.cu -- tier L: blocked right-looking LU with partial pivoting on
 // the matrices too large for one shared-memory tile.
 //
-// One iteration per panel of nb columns (Fig. 1), written for the
-// largest matrix (DCWI: the host loops over ITERATIONS of the largest
-// matrix, never over matrices; each kernel infers full / partial / no work):
-//   a4.1 panel_kernel     fused irrGETF2 on the (m_i - j) x ib panel, staged in
-//                         shared memory when it fits, else in place
-//   a4.2+a4.3 swap_trsm   the panel's row interchanges, "rehearsed" on an
-//                         index list first and then applied once per
-//                         moved row to the left and right column blocks; the
-//                         right block is solved in the same pass:
-//                         U12 <- L11^-1 P A12 (irrLASWP + irrTRSM fused)
-//   a4.4 gemm            A22 -= L21 U12 through the device tile schedule
+// The algorithm is the paper's (Fig. 1): per panel of nb columns,
+//   a4.1 panel       fused irrGETF2 on the (m_i - j) x ib panel, staged in
+//                    shared memory, interchanges inside the panel
+//   a4.2+a4.3 swap   the panel's row interchanges "rehearsed" on an index list
+//                     and applied once per moved row to the left and
+//                    right column blocks; the right block is solved in the
+//                    same pass: U12 <- L11^-1 P A12 (irrLASWP + irrTRSM fused)
+//   a4.4 gemm        A22 -= L21 U12 with the pipelined FP64 GEMM core
+// in two execution shapes:
+//   L1  (m <= 256 rows): ONE CTA per matrix runs every iteration of every step
+//       back to back (persistent CTAs, dynamic matrix queue); the matrix stays
+//       L2-resident between iterations, so HBM sees it about once, and there
+//       is no inter-kernel synchronisation at all.  Three CTAs per SM overlap
+//       one matrix's latency-bound panel with other matrices' GEMMs.
+//   L2  (taller): the host loops over panel ITERATIONS of the largest matrix
+//       (DCWI: each kernel infers full / partial / no work per
+//       matrix) with grid-wide kernels per step, so a few huge fronts use the
+//       whole GPU.
 #include "gemm_core.cuh"
 #include "panel.cuh"
 
@@ -19,13 +26,234 @@ namespace irr {
 
 constexpr int P_NT = 512;
 constexpr int NBMAX = 64;     // largest supported panel width
-constexpr int SW_COLS = 32;   // columns per swap/TRSM work item
+constexpr int SW_COLS = 32;   // columns per swap/TRSM chunk
 constexpr int SW_NT = 128;
+constexpr int L1_NT = 128;    // threads of the CTA-per-matrix kernel (== G_NT == SW_NT)
+static_assert(L1_NT == G_NT && L1_NT == SW_NT, "L1 composes the GEMM and swap pieces at one CTA size");
 
-// ------------------------------------------------------------------ a4.1 panel
+// ------------------------------------------------------------------ swap plan
+// Composition of the ib interchanges of one panel (rows j .. j+ib-1) on an
+// index list: position j+t receives row top_src[t]; position bot_pos[b] (below
+// the panel block) receives row bot_src[b].
+struct SwapPlan {
+    int top_src[NBMAX];
+    int piv[NBMAX];
+    int bot_pos[NBMAX], bot_src[NBMAX];
+    int nbot;
+};
+
+// Warp 0 composes the interchanges held in sp.piv[0..ib) (0-based absolute
+// rows).  Caller synchronises the CTA afterwards.
+__device__ __forceinline__ void plan_swaps_core(int j, int ib, SwapPlan &sp) {
+    const int lane = threadIdx.x & 31;
+    const int c1 = j + ib;
+    for (int t = lane; t < ib; t += 32) sp.top_src[t] = j + t;
+    int nbot = 0;
+    __syncwarp();
+    for (int t = 0; t < ib; ++t) {
+        const int p = sp.piv[t];
+        if (p == j + t) continue;
+        if (p < c1) {
+            if (lane == 0) {
+                int x = sp.top_src[t];
+                sp.top_src[t] = sp.top_src[p - j];
+                sp.top_src[p - j] = x;
+            }
+        } else {
+            int found = -1;
+            for (int b0 = 0; b0 < nbot; b0 += 32) {
+                int b = b0 + lane;
+                unsigned mk = __ballot_sync(FULL, b < nbot && sp.bot_pos[b] == p);
+                if (mk) { found = b0 + __ffs(mk) - 1; break; }
+            }
+            if (found < 0) {
+                found = nbot++;
+                if (lane == 0) { sp.bot_pos[found] = p; sp.bot_src[found] = p; }
+            }
+            if (lane == 0) {
+                int x = sp.top_src[t];
+                sp.top_src[t] = sp.bot_src[found];
+                sp.bot_src[found] = x;
+            }
+        }
+        __syncwarp();
+    }
+    if (lane == 0) sp.nbot = nbot;
+}
+
+// plan from ipiv[j .. j+ib) in global memory (1-based): one coalesced load
+__device__ __forceinline__ void plan_swaps(const int *__restrict__ ip, int j, int ib, SwapPlan &sp) {
+    if ((threadIdx.x >> 5) != 0) return;
+    for (int t = threadIdx.x & 31; t < ib; t += 32) sp.piv[t] = ip[j + t] - 1;
+    __syncwarp();
+    plan_swaps_core(j, ib, sp);
+}
+
+// plan from pivots already in shared memory (0-based absolute rows)
+__device__ __forceinline__ void plan_swaps_from(const int *piv_abs, int j, int ib, SwapPlan &sp) {
+    if ((threadIdx.x >> 5) != 0) return;
+    for (int t = threadIdx.x & 31; t < ib; t += 32) sp.piv[t] = piv_abs[t];
+    __syncwarp();
+    plan_swaps_core(j, ib, sp);
+}
+
+// Apply the plan to columns [cbeg, cbeg+W) of one matrix; when `solve`, also
+// U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory: L(r,s) = L11[r*ldl+s],
+// or, with ldl == 0, the packed strict lower triangle L11[r(r-1)/2 + s].
+// top / bot: shared buffers of nb x (SW_COLS+1).  SW_NT threads.
+__device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int cbeg, int W,
+                                           bool solve, const SwapPlan &sp, const double *L11, int ldl,
+                                           double *top, double *bot) {
+    const int tid = threadIdx.x;
+    constexpr int LT = SW_COLS + 1;
+    const int nbot = sp.nbot;
+    for (int e = tid; e < ib * W; e += SW_NT) {
+        int t = e % ib, c = e / ib;
+        cp_async8(&top[t * LT + c], gA + sp.top_src[t] + (size_t)(cbeg + c) * ld);
+    }
+    for (int e = tid; e < nbot * W; e += SW_NT) {
+        int b = e % nbot, c = e / nbot;
+        cp_async8(&bot[b * LT + c], gA + sp.bot_src[b] + (size_t)(cbeg + c) * ld);
+    }
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncthreads();
+    if (solve && tid < W) {
+        for (int s = 0; s < ib; ++s) {
+            const double x = top[s * LT + tid];
+            for (int r = s + 1; r < ib; ++r) {
+                const double l = ldl ? L11[r * ldl + s] : L11[((r * (r - 1)) >> 1) + s];
+                top[r * LT + tid] = fma(-l, x, top[r * LT + tid]);
+            }
+        }
+    }
+    __syncthreads();
+    for (int e = tid; e < ib * W; e += SW_NT) {
+        int t = e % ib, c = e / ib;
+        gA[j + t + (size_t)(cbeg + c) * ld] = top[t * LT + c];
+    }
+    for (int e = tid; e < nbot * W; e += SW_NT) {
+        int b = e % nbot, c = e / nbot;
+        gA[sp.bot_pos[b] + (size_t)(cbeg + c) * ld] = bot[b * LT + c];
+    }
+    __syncthreads();
+}
+
+__device__ __forceinline__ void load_L11_async(double *L11, int ldl, const double *gA, long ld, int j, int ib) {
+    for (int e = threadIdx.x; e < ib * ib; e += blockDim.x) {
+        int r = e % ib, c = e / ib;
+        cp_async8(&L11[r * ldl + c], gA + j + r + (size_t)(j + c) * ld);
+    }
+}
+
+// trailing-update descriptor of one matrix at iteration j (false: no GEMM work)
+__device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni, int j, int nb, GemmDesc &d) {
+    const int K = mi < ni ? mi : ni;
+    d.m = 0; d.n = 0; d.k = 0;
+    if (j >= K) return false;
+    const int ib = K - j < nb ? K - j : nb;
+    const int c1 = j + ib;
+    if (c1 >= mi || c1 >= ni) return false;
+    d.A = A + c1 + (size_t)j * ld; d.lda = ld; d.ta = 0;
+    d.B = A + j + (size_t)c1 * ld; d.ldb = ld; d.tb = 0;
+    d.C = A + c1 + (size_t)c1 * ld; d.ldc = ld;
+    d.m = mi - c1; d.n = ni - c1; d.k = ib;
+    d.alpha = -1.0; d.beta = 1.0;
+    return true;
+}
+
+// ================================================================== L1
+// One CTA per matrix, all iterations inside (matrices with m <= L1 rows).
+__global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__restrict__ counters,
+                                                         const int *__restrict__ bins, int nb,
+                                                         int l1_region_doubles) {
+    extern __shared__ __align__(16) unsigned char l1_smem[];
+    __shared__ PanelScratch sc;
+    __shared__ SwapPlan sp;
+    __shared__ int piv_s[NBMAX];
+    __shared__ int next_s;
+    double *smd = reinterpret_cast<double *>(l1_smem);
+    GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(l1_smem);
+    const int tid = threadIdx.x;
+    const int count = counters[CNT_BIN0 + BIN_L1];
+    const int *list = bins + (size_t)BIN_L1 * a.batch;
+    while (true) {
+        if (tid == 0) next_s = atomicAdd(&counters[CNT_L1_NEXT], 1);
+        __syncthreads();
+        const int t = next_s;
+        __syncthreads();
+        if (t >= count) break;
+        const int i = list[t];
+        const int mi = a.m[i], ni = a.n[i];
+        const long ld = a.ld[i];
+        double *gA = a.A[i];
+        int *gip = a.ipiv[i];
+        const int K = mi < ni ? mi : ni;
+        int info = 0;
+        for (int j = 0; j < K; j += nb) {
+            const int ib = K - j < nb ? K - j : nb;
+            const int rows = mi - j, c1 = j + ib;
+            // ---- a4.1 panel, staged in shared memory
+            double *P = smd;
+            const int ldp = rows | 1;
+            double *gP = gA + j + (size_t)j * ld;
+            stage_block_async(P, ldp, gP, ld, rows, ib, tid, L1_NT);
+            cp_async_commit();
+            cp_async_wait<0>();
+            __syncthreads();
+            const int z = panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            if (z && !info) info = j + z;
+            for (int e = tid; e < rows * ib; e += L1_NT) {
+                const int c = e / rows, r = e - c * rows;
+                gP[r + (size_t)c * ld] = P[r + c * ldp];
+            }
+            // packed unit-lower L11 kept past the union region for the U12 solve
+            double *L11p = smd + l1_region_doubles;
+            for (int e = tid; e < ib * ib; e += L1_NT) {
+                const int s = e / ib, r = e - s * ib;
+                if (r > s) L11p[((r * (r - 1)) >> 1) + s] = P[r + s * ldp];
+            }
+            if (tid < ib) {
+                piv_s[tid] += j;                  // absolute row
+                gip[j + tid] = piv_s[tid] + 1;
+            }
+            __syncthreads();
+            // ---- a4.2 + a4.3 interchanges left / right, U12 solve
+            if (j > 0 || c1 < ni) {
+                double *top = smd;
+                double *bot = top + nb * (SW_COLS + 1);
+                plan_swaps_from(piv_s, j, ib, sp);
+                __syncthreads();
+                for (int cb = 0; cb < j; cb += SW_COLS)
+                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, j - cb), false, sp, L11p, 0, top, bot);
+                for (int cb = c1; cb < ni; cb += SW_COLS)
+                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, ni - cb), true, sp, L11p, 0, top, bot);
+            }
+            // ---- a4.4 trailing update through the pipelined GEMM core
+            GemmDesc d0;
+            if (trailing_desc(gA, ld, mi, ni, j, nb, d0)) {
+                const int ntm = (d0.m + GBM - 1) / GBM, ntiles = ntm * ((d0.n + GBN - 1) / GBN);
+                int tt = 0;
+                auto next = [&](GemmDesc &d, int &r0, int &cc0) -> bool {
+                    if (tt >= ntiles) return false;
+                    d = d0;
+                    r0 = (tt % ntm) * GBM;
+                    cc0 = (tt / ntm) * GBN;
+                    ++tt;
+                    return true;
+                };
+                gemm_tile_stream(next, gsm);
+            }
+            __syncthreads();
+        }
+        if (tid == 0) a.info[i] = info;
+    }
+}
+
+// ================================================================== L2
 __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                      const int *__restrict__ bins, int j, int nb, int smem_rows) {
-    extern __shared__ __align__(16) double sp[];
+    extern __shared__ __align__(16) double sp_panel[];
     __shared__ PanelScratch sc;
     __shared__ int piv_s[NBMAX];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -45,9 +273,10 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
         const bool staged = rows <= smem_rows;
         if (staged) {
             ldp = rows | 1;
-            P = sp;
-            for (int c = warp; c < ib; c += NW)
-                for (int r = lane; r < rows; r += 32) P[r + c * ldp] = gP[r + (size_t)c * ld];
+            P = sp_panel;
+            stage_block_async(P, ldp, gP, ld, rows, ib, tid, P_NT);
+            cp_async_commit();
+            cp_async_wait<0>();
             __syncthreads();
         } else {
             P = gP;
@@ -64,25 +293,18 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
     }
 }
 
-// ------------------------------------------------------------------ a4.2 + a4.3
-// Work item = (tier-L slot, column chunk of SW_COLS).  Chunks 0..nleft-1 cover
-// the columns left of the panel [0, j) (interchanges only), the rest cover
+// Work item = (tier-L slot, column chunk).  Chunks 0..nleft-1 cover the
+// columns left of the panel [0, j) (interchanges only), the rest cover
 // [j+ib, n) (interchanges + forward substitution with the unit L11).
 __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                           const int *__restrict__ bins, int j, int nb,
                                                           int chunks_per) {
     extern __shared__ __align__(16) double sw_smem[];
-    // L11: nb x (nb+1); top: rows j..j+ib-1 of the chunk; bot: moved rows below
-    double *L11s = sw_smem;
-    double *tops = L11s + nb * (nb + 1);
-    double *bots = tops + nb * (SW_COLS + 1);
-#define L11(r, c) L11s[(r) * (nb + 1) + (c)]
-#define top(t, c) tops[(t) * (SW_COLS + 1) + (c)]
-#define bot(b, c) bots[(b) * (SW_COLS + 1) + (c)]
-    __shared__ int top_src[NBMAX];                // source row of position j+t
-    __shared__ int bot_pos[NBMAX], bot_src[NBMAX];
-    __shared__ int nbot_s;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int ldl = nb + 1;
+    double *L11 = sw_smem;
+    double *top = L11 + nb * ldl;
+    double *bot = top + nb * (SW_COLS + 1);
+    __shared__ SwapPlan sp;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
     const long long total = (long long)count * chunks_per;
@@ -101,128 +323,65 @@ __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int
         const bool right = q >= nleft;
         const int cbeg = right ? c1 + (q - nleft) * SW_COLS : q * SW_COLS;
         const int cend = right ? imin(ni, cbeg + SW_COLS) : imin(j, cbeg + SW_COLS);
-        const int W = cend - cbeg;
         double *gA = a.A[i];
-        const int *ip = a.ipiv[i];
-        // ---- rehearsal: compose the ib interchanges on an index list (warp 0)
         if (i != last_i) {
             __syncthreads();
-            if (warp == 0) {
-                for (int t = lane; t < ib; t += 32) top_src[t] = j + t;
-                int nbot = 0;
-                __syncwarp();
-                for (int t = 0; t < ib; ++t) {
-                    const int p = ip[j + t] - 1;  // absolute row
-                    if (p == j + t) continue;
-                    if (p < c1) {
-                        if (lane == 0) {
-                            int x = top_src[t];
-                            top_src[t] = top_src[p - j];
-                            top_src[p - j] = x;
-                        }
-                    } else {
-                        // find p in the bottom list (warp-parallel search)
-                        int found = -1;
-                        for (int b0 = 0; b0 < nbot; b0 += 32) {
-                            int b = b0 + lane;
-                            unsigned mk = __ballot_sync(FULL, b < nbot && bot_pos[b] == p);
-                            if (mk) { found = b0 + __ffs(mk) - 1; break; }
-                        }
-                        if (found < 0) {
-                            found = nbot++;
-                            if (lane == 0) { bot_pos[found] = p; bot_src[found] = p; }
-                        }
-                        if (lane == 0) {
-                            int x = top_src[t];
-                            top_src[t] = bot_src[found];
-                            bot_src[found] = x;
-                        }
-                    }
-                    __syncwarp();
-                }
-                if (lane == 0) nbot_s = nbot;
-            }
-            if (right) {
-                for (int e = tid; e < ib * ib; e += SW_NT) {
-                    int r = e % ib, c = e / ib;
-                    L11(r, c) = gA[j + r + (size_t)(j + c) * ld];
-                }
-            }
+            if (right) load_L11_async(L11, ldl, gA, ld, j, ib);
+            cp_async_commit();
+            plan_swaps(a.ipiv[i], j, ib, sp);
             last_i = right ? i : -1;  // L11 only valid when loaded
             __syncthreads();
         }
-        const int nbot = nbot_s;
-        // ---- gather the moved rows of this chunk (reads before any write)
-        for (int e = tid; e < ib * W; e += SW_NT) {
-            int t = e % ib, c = e / ib;
-            top(t, c) = gA[top_src[t] + (size_t)(cbeg + c) * ld];
-        }
-        for (int e = tid; e < nbot * W; e += SW_NT) {
-            int b = e % nbot, c = e / nbot;
-            bot(b, c) = gA[bot_src[b] + (size_t)(cbeg + c) * ld];
-        }
-        __syncthreads();
-        // ---- forward substitution on the top block (right chunks), one thread per column
-        if (right && tid < W) {
-            for (int s = 0; s < ib; ++s) {
-                const double x = top(s, tid);
-                for (int r = s + 1; r < ib; ++r) top(r, tid) = fma(-L11(r, s), x, top(r, tid));
-            }
-        }
-        __syncthreads();
-        // ---- write back
-        for (int e = tid; e < ib * W; e += SW_NT) {
-            int t = e % ib, c = e / ib;
-            gA[j + t + (size_t)(cbeg + c) * ld] = top(t, c);
-        }
-        for (int e = tid; e < nbot * W; e += SW_NT) {
-            int b = e % nbot, c = e / nbot;
-            gA[bot_pos[b] + (size_t)(cbeg + c) * ld] = bot(b, c);
-        }
-        __syncthreads();
+        swap_chunk(gA, ld, j, ib, cbeg, cend - cbeg, right, sp, L11, ldl, top, bot);
     }
-#undef L11
-#undef top
-#undef bot
 }
 
-// ------------------------------------------------------------------ a4.4 problem
 struct TrailingProb {
     GetrfArgs a;
     const int *list;
     int j, nb;
     __device__ bool get(int slot, GemmDesc &d) const {
         const int i = list[slot];
-        const int mi = a.m[i], ni = a.n[i];
-        const int K = mi < ni ? mi : ni;
-        d.m = 0; d.n = 0; d.k = 0;
-        if (j >= K) return false;
-        const int ib = K - j < nb ? K - j : nb;
-        const int c1 = j + ib;
-        if (c1 >= mi || c1 >= ni) return false;
-        const long ld = a.ld[i];
-        double *A = a.A[i];
-        d.A = A + c1 + (size_t)j * ld; d.lda = ld; d.ta = 0;
-        d.B = A + j + (size_t)c1 * ld; d.ldb = ld; d.tb = 0;
-        d.C = A + c1 + (size_t)c1 * ld; d.ldc = ld;
-        d.m = mi - c1; d.n = ni - c1; d.k = ib;
-        d.alpha = -1.0; d.beta = 1.0;
-        return true;
+        return trailing_desc(a.A[i], a.ld[i], a.m[i], a.n[i], j, nb, d);
     }
 };
 
+static int clamp_nb(int nb) { return nb < 1 ? 1 : (nb > NBMAX ? NBMAX : nb); }
+
+// L1 shared memory: a union region (panel | swap buffers | GEMM stages) plus
+// the packed L11 behind it.
+static size_t l1_region_bytes(int nb) {
+    size_t panel = (size_t)(L1_MAX_ROWS | 1) * nb * sizeof(double);
+    size_t swap = (size_t)(2 * nb * (SW_COLS + 1)) * sizeof(double);
+    size_t m = panel > swap ? panel : swap;
+    m = m > GEMM_SMEM ? m : GEMM_SMEM;
+    return (m + 15) & ~size_t(15);
+}
+
+void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream_t s) {
+    const int nb = clamp_nb(tuning().nb);
+    const size_t region = l1_region_bytes(nb);
+    const size_t smem = region + (size_t)(nb * (nb - 1) / 2 + 2) * sizeof(double);
+    static size_t attr = 0;
+    if (smem > attr) {
+        cudaFuncSetAttribute(lu_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr = smem;
+    }
+    int grid = num_sms() * 3;
+    if (grid > a.batch) grid = a.batch;
+    KScope k(K_LU_L1, s);
+    lu_l1_kernel<<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)));
+}
+
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s) {
     const Tuning &tu = tuning();
-    int nb = tu.nb;
-    if (nb < 1) nb = 1;
-    if (nb > NBMAX) nb = NBMAX;
+    const int nb = clamp_nb(tu.nb);
     const int Kmax = a.max_m < a.max_n ? a.max_m : a.max_n;
     // shared-memory panel rows: (rows|1) * nb doubles within the opt-in limit
     int smem_rows = tu.panel_rows;
     const int cap_rows = (int)((200 * 1024) / (sizeof(double) * nb)) - 1;
     if (smem_rows > cap_rows) smem_rows = cap_rows;
-    int rows_need = a.max_m;
-    if (smem_rows > rows_need) smem_rows = rows_need;
+    if (smem_rows > a.max_m) smem_rows = a.max_m;
     size_t psmem = (size_t)((smem_rows | 1) + 1) * nb * sizeof(double);
     static size_t attr_max = 0;
     if (psmem > attr_max) {
@@ -259,7 +418,9 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         }
         {
             KScope k(K_GEMM_TRAIL, s);
-            gemm_sched_kernel<TrailingProb><<<sms * 2, G_NT, 0, s>>>(P, -1, counters + CNT_BIN0 + BIN_L, tile_off);
+            gemm_smem_optin(gemm_sched_kernel<TrailingProb>);
+            gemm_sched_kernel<TrailingProb><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, -1, counters + CNT_BIN0 + BIN_L,
+                                                                           tile_off);
         }
     }
 }

@@ -13,10 +13,12 @@
 
 namespace irr {
 
-constexpr int M_NT = 256;
 constexpr int NBM = 16;
 
-__global__ void __launch_bounds__(M_NT) lu_mid_kernel(GetrfArgs a, const int *__restrict__ counters,
+// M_NT threads, MINB CTAs per SM (registers capped so the footprint-limited
+// occupancy is reachable: M1 48 KB -> 4 CTAs, M2 96 KB -> 2, M3 192 KB -> 1)
+template <int M_NT, int MINB>
+__global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                       const int *__restrict__ bins, int bin) {
     extern __shared__ __align__(16) double s[];
     __shared__ PanelScratch sc;
@@ -30,9 +32,10 @@ __global__ void __launch_bounds__(M_NT) lu_mid_kernel(GetrfArgs a, const int *__
         const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
         double *__restrict__ gA = a.A[i];
         const int lds = mid_lds(mi);
-        // ---- load (coalesced along columns)
-        for (int c = warp; c < ni; c += NW)
-            for (int r = lane; r < mi; r += 32) s[r + c * lds] = gA[r + (size_t)c * ld];
+        // ---- load: the whole matrix in flight at once (cp.async)
+        stage_block_async(s, lds, gA, ld, mi, ni, tid, M_NT);
+        cp_async_commit();
+        cp_async_wait<0>();
         __syncthreads();
         const int K = mi < ni ? mi : ni;
         int info = 0;
@@ -103,19 +106,26 @@ __global__ void __launch_bounds__(M_NT) lu_mid_kernel(GetrfArgs a, const int *__
 void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
                    cudaStream_t s) {
     size_t smem = (size_t)max_elems * sizeof(double);
-    static size_t attr_max = 0;  // the attribute is per function: keep the largest
-    if (smem > attr_max) {
-        cudaFuncSetAttribute(lu_mid_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr_max = smem;
-    }
-    int per_sm = (int)(200 * 1024 / (smem + 4096));
+    int per_sm = (int)(220 * 1024 / (smem + 2048));
     if (per_sm < 1) per_sm = 1;
-    if (per_sm > 8) per_sm = 8;
+    if (per_sm > 4) per_sm = 4;
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     if (grid < 1) grid = 1;
     KScope k(K_LU_MID, s);
-    lu_mid_kernel<<<grid, M_NT, smem, s>>>(a, counters, bins, bin);
+    if (per_sm >= 4) {
+        static size_t attr = 0;
+        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<128, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin);
+    } else if (per_sm >= 2) {
+        static size_t attr = 0;
+        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin);
+    } else {
+        static size_t attr = 0;
+        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin);
+    }
 }
 
 }  // namespace irr

@@ -64,12 +64,15 @@ def test_tier_m_boundary_and_extreme_shapes():
     _run_and_check(_uniform(shapes, seed=5))
 
 
+@pytest.mark.parametrize("l1", [1, 0])
 @pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
-def test_tier_l_forced_small_nb(nb):
-    """Force everything through the tier-L chain: nb-1, nb, nb+1, 2nb+-1 sizes."""
+def test_tier_l_forced_small_nb(nb, l1):
+    """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256,
+    l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
     irr.irr_set_tuning("tier_s", 0)
     irr.irr_set_tuning("tier_m_max", 0)
     irr.irr_set_tuning("nb", nb)
+    irr.irr_set_tuning("l1", l1)
     sizes = sorted({1, 2, nb - 1, nb, nb + 1, 2 * nb - 1, 2 * nb + 1, 3 * nb + 2} - {0})
     shapes = [(a, b) for a in sizes for b in sizes] + [(70, 45), (45, 70)]
     _run_and_check(_uniform(shapes, seed=nb))
@@ -96,12 +99,14 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "L"])
+@pytest.mark.parametrize("tier", ["default", "L", "L2"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
-    if tier == "L":
+    if tier in ("L", "L2"):
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
+    if tier == "L2":
+        irr.irr_set_tuning("l1", 0)
     shapes = [(1, 1), (5, 5), (32, 32), (32, 17), (17, 32), (33, 33), (64, 20), (20, 64), (130, 130),
               (150, 160), (257, 100), (100, 257), (300, 300)]
     mats = [irrgen.g1_exact(3, g, m, n)[0] for g, (m, n) in enumerate(shapes)]
