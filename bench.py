@@ -237,6 +237,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--ref-seconds", type=float, default=5.0)
     ap.add_argument("--profile-out", default=None, help="write per-kernel-class timings here (json)")
+    ap.add_argument("--tune", action="append", default=[], help="key=value passed to irr_set_tuning (experiments)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -253,6 +254,9 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    for kv in args.tune:
+        k, v = kv.split("=")
+        irr.irr_set_tuning(k, int(v))
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 

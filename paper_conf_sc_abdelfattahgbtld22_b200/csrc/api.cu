@@ -20,7 +20,7 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s);
 size_t laswp_smem(int span);
 
-static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32, 1};
+static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32, 1, 0, 3};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -219,6 +219,8 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "panel_rows")) g_tuning.panel_rows = value < 0 ? 0 : value;
     else if (!strcmp(key, "trsm_nb")) g_tuning.trsm_nb = value < 1 ? 1 : (value > 32 ? 32 : value);
     else if (!strcmp(key, "l1")) g_tuning.l1 = value ? 1 : 0;
+    else if (!strcmp(key, "phase_timing")) g_tuning.phase_timing = value ? 1 : 0;
+    else if (!strcmp(key, "l1_ctas_per_sm")) g_tuning.l1_ctas_per_sm = value < 1 ? 1 : (value > 3 ? 3 : value);
 }
 
 int irr_get_tuning(const char *key) {
@@ -229,6 +231,8 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "panel_rows")) return g_tuning.panel_rows;
     if (!strcmp(key, "trsm_nb")) return g_tuning.trsm_nb;
     if (!strcmp(key, "l1")) return g_tuning.l1;
+    if (!strcmp(key, "phase_timing")) return g_tuning.phase_timing;
+    if (!strcmp(key, "l1_ctas_per_sm")) return g_tuning.l1_ctas_per_sm;
     return -1;
 }
 

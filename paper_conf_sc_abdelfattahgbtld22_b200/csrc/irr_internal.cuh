@@ -20,6 +20,8 @@ struct Tuning {
     int panel_rows;  // max rows of a tier-L panel staged in shared memory
     int trsm_nb;     // TRSM recursion leaf (<= 32)
     int l1;          // 1: CTA-per-matrix tier for tier-L matrices with m <= L1_MAX_ROWS
+    int phase_timing;  // 1: accumulate per-phase SM cycles into the workspace counters
+    int l1_ctas_per_sm;  // resident CTAs per SM of the L1 kernel (1..3)
 };
 Tuning &tuning();
 
@@ -67,7 +69,8 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11 };
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11,
+                   CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
@@ -142,9 +145,12 @@ __device__ __forceinline__ void stage_block_async(double *s, int lds, const doub
             for (int e = t; e < total; e += nthr) cp_async8(s + e, g + e);
         }
     } else {
-        for (int e = t; e < total; e += nthr) {
-            const int c = e / m, r = e - c * m;
-            cp_async8(s + r + c * lds, g + r + (size_t)c * ld);
+        // warps over columns, lanes over rows: no per-element integer division
+        const int lane = t & 31, w0 = t >> 5, nw = nthr >> 5;
+        for (int c = w0; c < n; c += nw) {
+            const double *gc = g + (size_t)c * ld;
+            double *sc = s + c * lds;
+            for (int r = lane; r < m; r += 32) cp_async8(sc + r, gc + r);
         }
     }
 }

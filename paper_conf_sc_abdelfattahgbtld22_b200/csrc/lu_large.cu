@@ -26,7 +26,7 @@ namespace irr {
 
 constexpr int P_NT = 512;
 constexpr int NBMAX = 64;     // largest supported panel width
-constexpr int SW_COLS = 32;   // columns per swap/TRSM chunk
+constexpr int SW_COLS = 128;  // columns per swap/TRSM chunk (one thread per column)
 constexpr int SW_NT = 128;
 constexpr int L1_NT = 128;    // threads of the CTA-per-matrix kernel (== G_NT == SW_NT)
 static_assert(L1_NT == G_NT && L1_NT == SW_NT, "L1 composes the GEMM and swap pieces at one CTA size");
@@ -97,53 +97,78 @@ __device__ __forceinline__ void plan_swaps_from(const int *piv_abs, int j, int i
     plan_swaps_core(j, ib, sp);
 }
 
+// x <- L11^-1 x for one column x (stride ldx in shared memory), unit lower L11
+// column-major with leading dimension ldl, or, when ldl == 0, its strict lower
+// triangle packed by columns (column s = rows s+1..ib-1 at s(2ib-s-1)/2).
+// Shift-register form (as in tier S): v[0] is always the next solution
+// entry, so the loop body is the same for every step (O(NBX) code, no local
+// memory) and each step is NBX-1 independent FMAs.
+template <int NBX>
+__device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const double *L11, int ldl) {
+    double v[NBX];
+#pragma unroll
+    for (int r = 0; r < NBX; ++r) v[r] = (r < ib) ? x[r * ldx] : 0.0;
+    for (int s = 0; s < ib; ++s) {
+        const double xs = v[0];
+        x[s * ldx] = xs;
+        // column s of L11 below the diagonal is contiguous in both layouts
+        const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
+        const int cnt = ib - s - 1;
+#pragma unroll
+        for (int q = 0; q + 1 < NBX; ++q) {
+            const double l = (q < cnt) ? Ls[q] : 0.0;
+            v[q] = fma(-l, xs, v[q + 1]);
+        }
+        v[NBX - 1] = 0.0;
+    }
+}
+
 // Apply the plan to columns [cbeg, cbeg+W) of one matrix; when `solve`, also
-// U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory: L(r,s) = L11[r*ldl+s],
-// or, with ldl == 0, the packed strict lower triangle L11[r(r-1)/2 + s].
-// top / bot: shared buffers of nb x (SW_COLS+1).  SW_NT threads.
+// U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory in the layouts of
+// trsm_col_regs.  top / bot: shared buffers of nb x (SW_COLS+1).  SW_NT threads.
 __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int cbeg, int W,
                                            bool solve, const SwapPlan &sp, const double *L11, int ldl,
                                            double *top, double *bot) {
-    const int tid = threadIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     constexpr int LT = SW_COLS + 1;
+    constexpr int NWS = SW_NT / 32;
     const int nbot = sp.nbot;
-    for (int e = tid; e < ib * W; e += SW_NT) {
-        int t = e % ib, c = e / ib;
-        cp_async8(&top[t * LT + c], gA + sp.top_src[t] + (size_t)(cbeg + c) * ld);
-    }
-    for (int e = tid; e < nbot * W; e += SW_NT) {
-        int b = e % nbot, c = e / nbot;
-        cp_async8(&bot[b * LT + c], gA + sp.bot_src[b] + (size_t)(cbeg + c) * ld);
+    // warps over columns, lanes over the (<= 64) moved rows: no integer division
+    for (int c = warp; c < W; c += NWS) {
+        const double *gc = gA + (size_t)(cbeg + c) * ld;
+        for (int t = lane; t < ib; t += 32) cp_async8(&top[t * LT + c], gc + sp.top_src[t]);
+        for (int b = lane; b < nbot; b += 32) cp_async8(&bot[b * LT + c], gc + sp.bot_src[b]);
     }
     cp_async_commit();
     cp_async_wait<0>();
     __syncthreads();
     if (solve && tid < W) {
-        for (int s = 0; s < ib; ++s) {
-            const double x = top[s * LT + tid];
-            for (int r = s + 1; r < ib; ++r) {
-                const double l = ldl ? L11[r * ldl + s] : L11[((r * (r - 1)) >> 1) + s];
-                top[r * LT + tid] = fma(-l, x, top[r * LT + tid]);
+        // one thread per column, the column in registers (the smem
+        // read-modify-write form was a serial LDS->DFMA->STS chain)
+        if (ib <= 32) {
+            trsm_col_regs<32>(top + tid, LT, ib, L11, ldl);
+        } else {  // nb > 32 (tuning only): plain shared-memory substitution
+            for (int s = 0; s < ib; ++s) {
+                const double x = top[s * LT + tid];
+                const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
+                for (int r = s + 1; r < ib; ++r) top[r * LT + tid] = fma(-Ls[r - s - 1], x, top[r * LT + tid]);
             }
         }
     }
     __syncthreads();
-    for (int e = tid; e < ib * W; e += SW_NT) {
-        int t = e % ib, c = e / ib;
-        gA[j + t + (size_t)(cbeg + c) * ld] = top[t * LT + c];
-    }
-    for (int e = tid; e < nbot * W; e += SW_NT) {
-        int b = e % nbot, c = e / nbot;
-        gA[sp.bot_pos[b] + (size_t)(cbeg + c) * ld] = bot[b * LT + c];
+    for (int c = warp; c < W; c += NWS) {
+        double *gc = gA + (size_t)(cbeg + c) * ld;
+        for (int t = lane; t < ib; t += 32) gc[j + t] = top[t * LT + c];
+        for (int b = lane; b < nbot; b += 32) gc[sp.bot_pos[b]] = bot[b * LT + c];
     }
     __syncthreads();
 }
 
+// L11 (ib x ib diagonal block at (j, j)) -> shared memory, column-major (ldl)
 __device__ __forceinline__ void load_L11_async(double *L11, int ldl, const double *gA, long ld, int j, int ib) {
-    for (int e = threadIdx.x; e < ib * ib; e += blockDim.x) {
-        int r = e % ib, c = e / ib;
-        cp_async8(&L11[r * ldl + c], gA + j + r + (size_t)(j + c) * ld);
-    }
+    const int lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    for (int c = threadIdx.x >> 5; c < ib; c += nw)
+        for (int r = lane; r < ib; r += 32) cp_async8(&L11[r + c * ldl], gA + j + r + (size_t)(j + c) * ld);
 }
 
 // trailing-update descriptor of one matrix at iteration j (false: no GEMM work)
@@ -166,9 +191,10 @@ __device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni
 // One CTA per matrix, all iterations inside (matrices with m <= L1 rows).
 __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__restrict__ counters,
                                                          const int *__restrict__ bins, int nb,
-                                                         int l1_region_doubles) {
+                                                         int l1_region_doubles, int phase_timing) {
     extern __shared__ __align__(16) unsigned char l1_smem[];
     __shared__ PanelScratch sc;
+    __shared__ __align__(16) PanelRegScratch<L1_NT / 32, 32> prs;
     __shared__ SwapPlan sp;
     __shared__ int piv_s[NBMAX];
     __shared__ int next_s;
@@ -190,6 +216,8 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
         int *gip = a.ipiv[i];
         const int K = mi < ni ? mi : ni;
         int info = 0;
+        unsigned long long *ph = reinterpret_cast<unsigned long long *>(counters + CNT_PHASE0);
+        long long t0 = phase_timing ? clock64() : 0;
         for (int j = 0; j < K; j += nb) {
             const int ib = K - j < nb ? K - j : nb;
             const int rows = mi - j, c1 = j + ib;
@@ -201,23 +229,30 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
             cp_async_commit();
             cp_async_wait<0>();
             __syncthreads();
-            const int z = panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 3, (unsigned long long)(t1 - t0)); t0 = t1; }
+            const int z = (ib <= 32) ? panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs)
+                                     : panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 4, (unsigned long long)(t1 - t0)); t0 = t1; }
             if (z && !info) info = j + z;
-            for (int e = tid; e < rows * ib; e += L1_NT) {
-                const int c = e / rows, r = e - c * rows;
-                gP[r + (size_t)c * ld] = P[r + c * ldp];
-            }
-            // packed unit-lower L11 kept past the union region for the U12 solve
+            // write the factored panel back; keep the strict lower triangle of
+            // L11, packed by columns, past the union region for the U12 solve
             double *L11p = smd + l1_region_doubles;
-            for (int e = tid; e < ib * ib; e += L1_NT) {
-                const int s = e / ib, r = e - s * ib;
-                if (r > s) L11p[((r * (r - 1)) >> 1) + s] = P[r + s * ldp];
+            {
+                const int lane = tid & 31, warp = tid >> 5;
+                for (int c = warp; c < ib; c += L1_NT / 32) {
+                    double *gc = gP + (size_t)c * ld;
+                    const double *pc = P + c * ldp;
+                    for (int r = lane; r < rows; r += 32) gc[r] = pc[r];
+                    double *lc = L11p + (c * (2 * ib - c - 1)) / 2 - (c + 1);
+                    for (int r = c + 1 + lane; r < ib; r += 32) lc[r] = pc[r];
+                }
             }
             if (tid < ib) {
                 piv_s[tid] += j;                  // absolute row
                 gip[j + tid] = piv_s[tid] + 1;
             }
             __syncthreads();
+            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 0, (unsigned long long)(t1 - t0)); t0 = t1; }
             // ---- a4.2 + a4.3 interchanges left / right, U12 solve
             if (j > 0 || c1 < ni) {
                 double *top = smd;
@@ -229,6 +264,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                 for (int cb = c1; cb < ni; cb += SW_COLS)
                     swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, ni - cb), true, sp, L11p, 0, top, bot);
             }
+            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 1, (unsigned long long)(t1 - t0)); t0 = t1; }
             // ---- a4.4 trailing update through the pipelined GEMM core
             GemmDesc d0;
             if (trailing_desc(gA, ld, mi, ni, j, nb, d0)) {
@@ -245,6 +281,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                 gemm_tile_stream(next, gsm);
             }
             __syncthreads();
+            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 2, (unsigned long long)(t1 - t0)); t0 = t1; }
         }
         if (tid == 0) a.info[i] = info;
     }
@@ -255,6 +292,7 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
                                                      const int *__restrict__ bins, int j, int nb, int smem_rows) {
     extern __shared__ __align__(16) double sp_panel[];
     __shared__ PanelScratch sc;
+    __shared__ __align__(16) PanelRegScratch<P_NT / 32, 32> prs;
     __shared__ int piv_s[NBMAX];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     constexpr int NW = P_NT / 32;
@@ -282,7 +320,9 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
             P = gP;
             ldp = ld;
         }
-        int z = panel_getf2<P_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+        int z = (staged && ib <= 32 && rows <= 2 * P_NT)
+                    ? panel_regs<P_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs)
+                    : panel_getf2<P_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
         if (staged) {
             for (int c = warp; c < ib; c += NW)
                 for (int r = lane; r < rows; r += 32) gP[r + (size_t)c * ld] = P[r + c * ldp];
@@ -367,10 +407,13 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
         cudaFuncSetAttribute(lu_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
-    int grid = num_sms() * 3;
+    int per_sm = tuning().l1_ctas_per_sm;
+    if (per_sm < 1 || per_sm > 3) per_sm = 3;
+    int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     KScope k(K_LU_L1, s);
-    lu_l1_kernel<<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)));
+    lu_l1_kernel<<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
+                                           tuning().phase_timing);
 }
 
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s) {

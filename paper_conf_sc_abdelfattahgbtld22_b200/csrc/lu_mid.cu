@@ -19,9 +19,18 @@ constexpr int NBM = 16;
 // occupancy is reachable: M1 48 KB -> 4 CTAs, M2 96 KB -> 2, M3 192 KB -> 1)
 template <int M_NT, int MINB>
 __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const int *__restrict__ counters,
-                                                      const int *__restrict__ bins, int bin) {
+                                                      const int *__restrict__ bins, int bin,
+                                                      unsigned long long *ph) {
     extern __shared__ __align__(16) double s[];
+    long long t0 = 0;
+#define MID_PHASE(k)                                                                    \
+    if (ph && threadIdx.x == 0) {                                                       \
+        long long t1 = clock64();                                                       \
+        atomicAdd(ph + (k), (unsigned long long)(t1 - t0));                             \
+        t0 = t1;                                                                        \
+    }
     __shared__ PanelScratch sc;
+    __shared__ __align__(16) PanelRegScratch<M_NT / 32, NBM> prs;
     __shared__ int piv_s[NBM];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     constexpr int NW = M_NT / 32;
@@ -32,20 +41,44 @@ __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const i
         const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
         double *__restrict__ gA = a.A[i];
         const int lds = mid_lds(mi);
+        if (ph && tid == 0) t0 = clock64();
         // ---- load: the whole matrix in flight at once (cp.async)
         stage_block_async(s, lds, gA, ld, mi, ni, tid, M_NT);
         cp_async_commit();
         cp_async_wait<0>();
         __syncthreads();
+        MID_PHASE(3)
         const int K = mi < ni ? mi : ni;
         int info = 0;
         int *gipiv = a.ipiv[i];
         for (int j = 0; j < K; j += NBM) {
             const int ib = K - j < NBM ? K - j : NBM;
             // ---- fused panel, interchanges applied to the full rows
-            int z = panel_getf2<M_NT>(s, lds, j, mi, j, ib, 0, ni, piv_s, sc);
+            int z;
+            if (mi - j <= 2 * M_NT) {
+                // register-resident panel (1 barrier per column), then the
+                // panel's interchanges on the other columns, one thread per column
+                z = panel_regs<M_NT, 2, NBM>(s + j + j * lds, lds, mi - j, ib, piv_s, prs);
+                for (int cc = tid; cc < ni; cc += M_NT) {
+                    if (cc >= j && cc < j + ib) continue;
+                    double *col = s + cc * lds;
+                    for (int c = 0; c < ib; ++c) {
+                        const int p = j + piv_s[c];
+                        if (p != j + c) {
+                            const double x = col[j + c];
+                            col[j + c] = col[p];
+                            col[p] = x;
+                        }
+                    }
+                }
+                __syncthreads();
+                if (tid < ib) piv_s[tid] += j;
+            } else {
+                z = panel_getf2<M_NT>(s, lds, j, mi, j, ib, 0, ni, piv_s, sc);
+            }
             if (z && !info) info = j + z;
             if (tid < ib) gipiv[j + tid] = piv_s[tid] + 1;
+            MID_PHASE(4)
             const int c1 = j + ib;
             if (c1 >= ni) continue;
             // ---- U12 <- L11^-1 A12 (unit lower, in place), one thread per column
@@ -64,6 +97,7 @@ __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const i
                     if (q < ib) s[j + q + cc * lds] = x[q];
             }
             __syncthreads();
+            MID_PHASE(5)
             // ---- A22 -= L21 * U12 : warp tiles of 64 rows x 4 columns,
             //      lane owns rows (lane, lane + 32) of the tile
             const int Mr = mi - c1, Nc = ni - c1;
@@ -94,13 +128,16 @@ __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const i
                 }
             }
             __syncthreads();
+            MID_PHASE(6)
         }
         // ---- store
         for (int c = warp; c < ni; c += NW)
             for (int r = lane; r < mi; r += 32) gA[r + (size_t)c * ld] = s[r + c * lds];
         if (tid == 0) a.info[i] = info;
         __syncthreads();
+        MID_PHASE(7)
     }
+#undef MID_PHASE
 }
 
 void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
@@ -113,18 +150,21 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
     if (grid > a.batch) grid = a.batch;
     if (grid < 1) grid = 1;
     KScope k(K_LU_MID, s);
+    unsigned long long *ph =
+        tuning().phase_timing ? reinterpret_cast<unsigned long long *>(const_cast<int *>(counters) + CNT_PHASE0)
+                              : nullptr;
     if (per_sm >= 4) {
         static size_t attr = 0;
         if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<128, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
-        lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin);
+        lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin, ph);
     } else if (per_sm >= 2) {
         static size_t attr = 0;
         if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
-        lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin);
+        lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
     } else {
         static size_t attr = 0;
         if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
-        lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin);
+        lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
     }
 }
 
