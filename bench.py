@@ -114,12 +114,13 @@ def tier_of(m, n, tier_m_max=24576, l1=True):
     return t
 
 
-def class_work(m, n, nb=32):
+def class_work(m, n, nb=32, tier_m_max=24576, l1=True):
     """Algorithmic (flops, bytes) per kernel class for one getrf step
-    (DESIGN.md 'Roofline accounting')."""
+    (DESIGN.md 'Roofline accounting'); tiers mirror classify.cu with the
+    library's live tuning."""
     m = np.asarray(m, dtype=np.int64)
     n = np.asarray(n, dtype=np.int64)
-    t = tier_of(m, n)
+    t = tier_of(m, n, tier_m_max, l1)
     out = {}
     for cls, tier in (("lu_small", 0), ("lu_mid", 1), ("lu_l1", 2)):
         sel = t == tier
@@ -148,10 +149,10 @@ def class_work(m, n, nb=32):
     return out
 
 
-def class_work_partial(n1, n2, nb=32):
+def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=True):
     n1 = np.asarray(n1, dtype=np.int64)
     n2 = np.asarray(n2, dtype=np.int64)
-    out = class_work(n1, n1, nb)
+    out = class_work(n1, n1, nb, tier_m_max, l1)
     out["gemm_dcwi"] = (float((2.0 * n1 * n2 * n2).sum()), float((8.0 * (2 * n2 * n2 + n2 * n1 + n1 * n2)).sum()))
     out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((32.0 * n1 * n2).sum()))
     return out
@@ -274,7 +275,8 @@ def main():
         B = MatrixBatch(m_loc, n_loc, device=dev)
         ld_loc = B.ld_h
         call = lambda: B.getrf()  # noqa: E731
-        cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"))
+        cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
+                        bool(irr.irr_get_tuning("l1")))
         bytes_local = float(F.getrf_bytes(m_loc, n_loc).sum())
         host = B.host_buffer(pinned=True)
         hn = host.numpy()
@@ -285,7 +287,8 @@ def main():
     else:
         B = FrontBatch(m_loc, n_loc, device=dev)
         call = lambda: B.getrf_partial()  # noqa: E731
-        cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"))
+        cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
+                                bool(irr.irr_get_tuning("l1")))
         bytes_local = float(F.partial_bytes(m_loc, n_loc).sum())
         host = torch.empty(B.total, dtype=torch.float64, pin_memory=True)
         hn = host.numpy()

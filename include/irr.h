@@ -165,10 +165,15 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
               const int *kcount, int *const *ipiv, int batch, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
- * Tuning (tests only; defaults are fixed).  Keys: "nb" (tier-L panel width,
- * 8..64), "tier_s" (1 = enable warp-per-matrix tier), "tier_m_max" (max m*n
- * of the shared-memory tier, 0 disables it), "panel_rows" (max panel rows held
- * in shared memory), "trsm_nb" (TRSM recursion leaf).  Unknown keys are ignored.
+ * Tuning (tests and experiments; defaults are fixed by measurement and are
+ * process-global, not thread-safe).  Keys: "nb" (tier-L panel width, 1..64),
+ * "tier_s" (1 = enable the warp-per-matrix tier), "tier_m_max" (max padded
+ * m*n of the shared-memory tier, 0 disables it), "l1" (1 = CTA-per-matrix
+ * tier for m <= 256), "l1_ctas_per_sm" (1..3), "panel_rows" (max rows of a
+ * grid-wide panel staged in shared memory), "trsm_nb" (TRSM recursion leaf),
+ * "concurrent" (1 = S/M tiers on a forked stream), "dmma" (1 = grid-wide GEMMs
+ * on the FP64 tensor core), "l1_dmma" (same inside L1), "phase_timing"
+ * (1 = per-phase cycle counters in the workspace).  Unknown keys are ignored;
  * irr_get_tuning returns the current value (-1 for an unknown key).
  * ---------------------------------------------------------------------- */
 void irr_set_tuning(const char *key, int value);

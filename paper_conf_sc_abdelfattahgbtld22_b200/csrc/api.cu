@@ -11,16 +11,23 @@
 #include <vector>
 
 #include "irr_internal.cuh"
+#include "sched.cuh"
 
 namespace irr {
 
-void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s);
-void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *tile_off, cudaStream_t s);
+void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s,
+                        SlotList sl);
+void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *tile_off, cudaStream_t s,
+                     int *sort_ws);
 void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
-                         const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s);
+                         const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s,
+                         int *units_off, SlotList sl);
 size_t laswp_smem(int span);
 
-static Tuning g_default = {32, 1, TIER_M_MAX_DEFAULT, 768, 32, 1, 0, 3};
+// defaults chosen by measurement on B200: tier M only up to
+// 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
+// grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -91,6 +98,33 @@ int num_sms() {
     return d ? d->sms : 148;
 }
 
+// Per-device side stream + fork/join events, created once (never on the hot
+// path after the first call).  Non-blocking w.r.t. the legacy stream.
+struct DeviceStreams {
+    cudaStream_t side = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+};
+static DeviceStreams g_streams[64];
+
+static DeviceStreams *dev_streams() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    DeviceStreams &d = g_streams[dev];
+    if (!d.side) {
+        if (cudaStreamCreateWithFlags(&d.side, cudaStreamNonBlocking) != cudaSuccess) { d.side = nullptr; return nullptr; }
+        cudaEventCreateWithFlags(&d.fork, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&d.join, cudaEventDisableTiming);
+    }
+    return &d;
+}
+static cudaStream_t side_stream() {
+    DeviceStreams *d = dev_streams();
+    return d ? d->side : nullptr;
+}
+static cudaEvent_t fork_event() { return dev_streams()->fork; }
+static cudaEvent_t join_event() { return dev_streams()->join; }
+
 static int check_device() {
     const DeviceInfo *d = device_info();
     if (!d) return IRR_ERR_CUDA;
@@ -103,11 +137,13 @@ struct Work {
     int *counters;
     int *bins;
     int *tile_off;
+    int *sort;  // size sort (sched.cuh): sorted slots + bucket prefix
 };
 
 static size_t work_bytes_for(int batch) {
     size_t b = (size_t)(batch > 0 ? batch : 1);
-    return align256(CNT_INTS * sizeof(int)) + align256(NBINS * b * sizeof(int)) + align256((b + 1) * sizeof(int));
+    return align256(CNT_INTS * sizeof(int)) + align256(NBINS * b * sizeof(int)) + align256((b + 1) * sizeof(int)) +
+           align256(size_sort_ints((int)b) * sizeof(int));
 }
 
 static Work carve(void *work, int batch) {
@@ -119,6 +155,8 @@ static Work carve(void *work, int batch) {
     w.bins = (int *)p;
     p += align256(NBINS * b * sizeof(int));
     w.tile_off = (int *)p;
+    p += align256((b + 1) * sizeof(int));
+    w.sort = (int *)p;
     return w;
 }
 
@@ -144,19 +182,36 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
     // which tiers can be populated, from the required dims alone
     const long long big = (long long)mid_lds(a.max_m) * a.max_n;
     const bool only_s = t.tier_s && a.max_m <= 32 && a.max_n <= 32;
-    if (t.tier_s) launch_lu_small(a, w.counters, w.bins, s);
-    if (!only_s) {
-        const long long mmax = t.tier_m_max;
-        if (mmax > 0) {
-            launch_lu_mid(a, w.counters, w.bins, BIN_M1, (int)(mmax < M1_ELEMS ? mmax : M1_ELEMS), s);
-            if (big > M1_ELEMS && mmax > M1_ELEMS)
-                launch_lu_mid(a, w.counters, w.bins, BIN_M2, (int)(mmax < M2_ELEMS ? mmax : M2_ELEMS), s);
-            if (big > M2_ELEMS && mmax > M2_ELEMS) launch_lu_mid(a, w.counters, w.bins, BIN_M3, (int)mmax, s);
+    const long long mmax = t.tier_m_max;
+    const bool has_large = !only_s && big > mmax;
+    // The tiers touch disjoint matrices: with a large tier present, S and M run
+    // on a forked stream concurrently with it (fills each other's tails).
+    cudaStream_t side = s;
+    if (has_large && t.concurrent) {
+        side = side_stream();
+        if (side) {
+            IRR_CUDA_TRY(cudaEventRecord(fork_event(), s));
+            IRR_CUDA_TRY(cudaStreamWaitEvent(side, fork_event(), 0));
+        } else {
+            side = s;
         }
-        if (big > mmax) {
+    }
+    if (t.tier_s) launch_lu_small(a, w.counters, w.bins, side);
+    if (!only_s) {
+        if (mmax > 0) {
+            launch_lu_mid(a, w.counters, w.bins, BIN_M1, (int)(mmax < M1_ELEMS ? mmax : M1_ELEMS), side);
+            if (big > M1_ELEMS && mmax > M1_ELEMS)
+                launch_lu_mid(a, w.counters, w.bins, BIN_M2, (int)(mmax < M2_ELEMS ? mmax : M2_ELEMS), side);
+            if (big > M2_ELEMS && mmax > M2_ELEMS) launch_lu_mid(a, w.counters, w.bins, BIN_M3, (int)mmax, side);
+        }
+        if (has_large) {
             if (t.l1) launch_lu_l1(a, w.counters, w.bins, s);
             if (!t.l1 || a.max_m > L1_MAX_ROWS) launch_lu_large(a, w.counters, w.bins, w.tile_off, s);
         }
+    }
+    if (side != s) {
+        IRR_CUDA_TRY(cudaEventRecord(join_event(), side));
+        IRR_CUDA_TRY(cudaStreamWaitEvent(s, join_event(), 0));
     }
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
@@ -221,6 +276,9 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1")) g_tuning.l1 = value ? 1 : 0;
     else if (!strcmp(key, "phase_timing")) g_tuning.phase_timing = value ? 1 : 0;
     else if (!strcmp(key, "l1_ctas_per_sm")) g_tuning.l1_ctas_per_sm = value < 1 ? 1 : (value > 3 ? 3 : value);
+    else if (!strcmp(key, "concurrent")) g_tuning.concurrent = value ? 1 : 0;
+    else if (!strcmp(key, "dmma")) g_tuning.dmma = value ? 1 : 0;
+    else if (!strcmp(key, "l1_dmma")) g_tuning.l1_dmma = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -233,6 +291,9 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "l1")) return g_tuning.l1;
     if (!strcmp(key, "phase_timing")) return g_tuning.phase_timing;
     if (!strcmp(key, "l1_ctas_per_sm")) return g_tuning.l1_ctas_per_sm;
+    if (!strcmp(key, "concurrent")) return g_tuning.concurrent;
+    if (!strcmp(key, "dmma")) return g_tuning.dmma;
+    if (!strcmp(key, "l1_dmma")) return g_tuning.l1_dmma;
     return -1;
 }
 
@@ -303,16 +364,20 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     rc = getrf_core(a, w, 1, s);
     if (rc) return rc;
     if (max_n1 <= 0 || max_n2 <= 0) return IRR_SUCCESS;
+    // fronts sorted by n1 (descending buckets): every building-block call
+    // below visits only the fronts that still have work at its offset
+    launch_size_sort(n1, batch, w.sort, s);
     // step 2: F12 <- U^-1 L^-1 P^T F12: irrLASWP + 2 x irrTRSM (GETRS)
-    launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s);
+    launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s, w.tile_off,
+                        sorted_slots(w.sort, batch, 0));
     TrsmArgs t{};
     t.side = IRR_LEFT; t.uplo = IRR_LOWER; t.trans = IRR_NO_TRANS; t.diag = IRR_UNIT;
     t.max_m = max_n1; t.max_n = max_n2; t.m = n1; t.n = n2; t.alpha = 1.0;
     t.T = (const double *const *)F11; t.Ti = 0; t.Tj = 0; t.ldt = ld11;
     t.B = F12; t.Bi = 0; t.Bj = 0; t.ldb = ld12; t.batch = batch;
-    run_trsm_masked(t, info, w.counters, w.tile_off, s);
+    run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
     t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
-    run_trsm_masked(t, info, w.counters, w.tile_off, s);
+    run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
     // step 3: F22 <- F22 - F21 F12, F21 untouched
     GemmArgs g{};
     g.ta = 0; g.tb = 0; g.max_m = max_n2; g.max_n = max_n2; g.max_k = max_n1;
@@ -320,7 +385,7 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     g.A = F21; g.Ai = 0; g.Aj = 0; g.lda = ld21;
     g.B = (const double *const *)F12; g.Bi = 0; g.Bj = 0; g.ldb = ld12;
     g.C = F22; g.Ci = 0; g.Cj = 0; g.ldc = ld22; g.batch = batch;
-    launch_gemm_masked(g, info, w.counters, w.tile_off, s);
+    launch_gemm_masked(g, info, w.counters, w.tile_off, s, sorted_slots(w.sort, batch, 0));
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 
@@ -362,7 +427,7 @@ int irr_gemm(irr_trans_t ta, irr_trans_t tb, int max_m, int max_n, int max_k, co
     }
     GemmArgs g{(int)ta, (int)tb, max_m, max_n, max_k, m, n, k, alpha, beta, A, Ai, Aj, lda, B, Bi, Bj, ldb,
                C, Ci, Cj, ldc, batch};
-    launch_gemm_masked(g, nullptr, nullptr, tile_off, s);
+    launch_gemm_masked(g, nullptr, nullptr, tile_off, s, all_slots());
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 
@@ -393,16 +458,18 @@ int irr_trsm(irr_side_t side, irr_uplo_t uplo, irr_trans_t trans, irr_diag_t dia
     int rc = check_device();
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;
-    int *tile_off = nullptr, *counters = nullptr;
+    int *tile_off = nullptr, *counters = nullptr, *sort = nullptr;
     if (work) {
         if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
         Work w = carve(work, batch);
         tile_off = w.tile_off;
         counters = w.counters;
+        sort = w.sort;
+        launch_size_sort(side == IRR_LEFT ? m : n, batch, sort, s);
     }
     TrsmArgs t{(int)side, (int)uplo, (int)trans, (int)diag, max_m, max_n, m, n, alpha, T, Ti, Tj, ldt,
                B, Bi, Bj, ldb, batch};
-    run_trsm_masked(t, nullptr, counters, tile_off, s);
+    run_trsm_masked(t, nullptr, counters, tile_off, s, sort);
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 
@@ -423,7 +490,8 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
     if (laswp_smem(k2 - k1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     int rc = check_device();
     if (rc) return rc;
-    launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, (cudaStream_t)stream);
+    launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, (cudaStream_t)stream,
+                        nullptr, all_slots());
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 

@@ -74,7 +74,9 @@ __device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, 
     }
 }
 
-__device__ __forceinline__ void gemm_compute_chunk(const GemmSmem &sm, int buf, double acc[8][4]) {
+// ---- DFMA path: thread (tx, ty) owns rows tx + 8q (q < 8), cols ty + 16p (p < 4);
+//      acc[q * 4 + p].  12 shared-memory wavefronts per 32 DFMA per warp.
+__device__ __forceinline__ void gemm_compute_chunk_dfma(const GemmSmem &sm, int buf, double (&acc)[32]) {
     const int tid = threadIdx.x, tx = tid & 7, ty = tid >> 3;
 #pragma unroll
     for (int kk = 0; kk < GBK; ++kk) {
@@ -86,30 +88,85 @@ __device__ __forceinline__ void gemm_compute_chunk(const GemmSmem &sm, int buf, 
 #pragma unroll
         for (int q = 0; q < 8; ++q)
 #pragma unroll
-            for (int p = 0; p < 4; ++p) acc[q][p] = fma(a[q], b[p], acc[q][p]);
+            for (int p = 0; p < 4; ++p) acc[q * 4 + p] = fma(a[q], b[p], acc[q * 4 + p]);
     }
 }
 
-__device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0, const GemmSmem &sm, double acc[8][4]) {
-    const int tid = threadIdx.x, tx = tid & 7, ty = tid >> 3;
+// ---- DMMA path (FP64 tensor core, mma.sync m8n8k4 -> SASS DMMA.8x8x4):
+//      warp w computes the 32x32 sub-tile (rows 32 (w&1), cols 32 (w>>1)) as
+//      4 x 4 mma tiles; lane (g = lane>>2, t = lane&3) holds A(g, t), B(t, g)
+//      and C(g, 2t + i).  acc[(mi * 4 + ni) * 2 + i].  One DMMA = 256 FMA, so
+//      the operand traffic is two 8-byte loads per lane per 16 DMMA.
+__device__ __forceinline__ void dmma_8x8x4(double &c0, double &c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+__device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int buf, double (&acc)[32]) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+    const int rb = (warp & 1) * 32 + g, cb = (warp >> 1) * 32 + g;
 #pragma unroll
-    for (int p = 0; p < 4; ++p) {
-        const int cl = ty + 16 * p, c = c0 + cl;
-        if (c >= d.n) continue;
+    for (int ks = 0; ks < GBK; ks += 4) {
+        double a[4], b[4];
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-            const int rl = tx + 8 * q, r = r0 + rl;
+        for (int mi = 0; mi < 4; ++mi) a[mi] = sm.As[buf][ks + t][rb + 8 * mi];
+#pragma unroll
+        for (int ni = 0; ni < 4; ++ni) b[ni] = sm.Bs[buf][ks + t][cb + 8 * ni];
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 4; ++ni)
+                dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], a[mi], b[ni]);
+    }
+}
+
+template <bool DMMA>
+__device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0, const GemmSmem &sm,
+                                              const double (&acc)[32]) {
+    const int tid = threadIdx.x;
+    if (!DMMA) {
+        const int tx = tid & 7, ty = tid >> 3;
+#pragma unroll
+        for (int p = 0; p < 4; ++p) {
+            const int cl = ty + 16 * p, c = c0 + cl;
+            if (c >= d.n) continue;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const int rl = tx + 8 * q, r = r0 + rl;
+                if (r >= d.m) continue;
+                double v = d.alpha * acc[q * 4 + p];
+                if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
+                d.C[r + (size_t)c * d.ldc] = v;
+            }
+        }
+    } else {
+        const int lane = tid & 31, warp = tid >> 5;
+        const int g = lane >> 2, t = lane & 3;
+#pragma unroll
+        for (int mi = 0; mi < 4; ++mi) {
+            const int rl = (warp & 1) * 32 + 8 * mi + g, r = r0 + rl;
             if (r >= d.m) continue;
-            double v = d.alpha * acc[q][p];
-            if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
-            d.C[r + (size_t)c * d.ldc] = v;
+#pragma unroll
+            for (int ni = 0; ni < 4; ++ni) {
+#pragma unroll
+                for (int i = 0; i < 2; ++i) {
+                    const int cl = (warp >> 1) * 32 + 8 * ni + 2 * t + i, c = c0 + cl;
+                    if (c >= d.n) continue;
+                    double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
+                    if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
+                    d.C[r + (size_t)c * d.ldc] = v;
+                }
+            }
         }
     }
 }
 
 // A stream of tiles processed by one CTA with the software pipeline described
 // above.  `next(d, r0, c0)` returns false when the CTA has no more tiles.
-template <class Next>
+// DMMA selects the FP64 tensor-core path, else DFMA.
+template <bool DMMA, class Next>
 __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     GemmDesc d, dn;
     int r0, c0, rn, cn;
@@ -121,11 +178,9 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     while (have) {
         gemm_issue_c(d, r0, c0, sm);
         cp_async_commit();
-        double acc[8][4];
+        double acc[32];
 #pragma unroll
-        for (int q = 0; q < 8; ++q)
-#pragma unroll
-            for (int p = 0; p < 4; ++p) acc[q][p] = 0.0;
+        for (int q = 0; q < 32; ++q) acc[q] = 0.0;
         const int nchunks = (d.k + GBK - 1) / GBK;
         bool has_next_tile = false;
         for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
@@ -138,13 +193,16 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
             cp_async_commit();
             if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();
             __syncthreads();
-            if (nchunks > 0) gemm_compute_chunk(sm, buf, acc);
+            if (nchunks > 0) {
+                if (DMMA) gemm_compute_chunk_dmma(sm, buf, acc);
+                else gemm_compute_chunk_dfma(sm, buf, acc);
+            }
             __syncthreads();
             buf ^= 1;
         }
         cp_async_wait<1>();
         __syncthreads();
-        gemm_epilogue(d, r0, c0, sm, acc);
+        gemm_epilogue<DMMA>(d, r0, c0, sm, acc);
         __syncthreads();
         have = has_next_tile;
         if (have) { d = dn; r0 = rn; c0 = cn; }
@@ -201,7 +259,7 @@ __global__ void __launch_bounds__(1024) gemm_scan_kernel(Prob P, int count, cons
     if (tid == 0) tile_off[count] = carry_s;
 }
 
-template <class Prob>
+template <class Prob, bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, const int *count_ptr,
                                                           const int *__restrict__ tile_off) {
     extern __shared__ __align__(16) unsigned char g_smem[];
@@ -239,13 +297,13 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, 
         ++t;
         return true;
     };
-    gemm_tile_stream(next, sm);
+    gemm_tile_stream<DMMA>(next, sm);
 }
 
 // DCWI-grid fallback (no workspace): virtual tiles over the required dims,
 // empty ones are skipped ("If no workload is detected, the
 // corresponding GPU threads perform no work at all").
-template <class Prob>
+template <class Prob, bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) gemm_grid_kernel(Prob P, int count, int tiles_m, int tiles_n) {
     extern __shared__ __align__(16) unsigned char g_smem[];
     GemmSmem &sm = *reinterpret_cast<GemmSmem *>(g_smem);
@@ -266,7 +324,7 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_grid_kernel(Prob P, int count, i
         }
         return false;
     };
-    gemm_tile_stream(next, sm);
+    gemm_tile_stream<DMMA>(next, sm);
 }
 
 // opt-in to > 48 KB dynamic shared memory once per kernel instantiation

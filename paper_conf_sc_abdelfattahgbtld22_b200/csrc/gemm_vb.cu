@@ -3,13 +3,16 @@
 // submatrices selected by scalar offsets, with per-matrix effective sizes
 // inferred on the device.
 #include "gemm_core.cuh"
+#include "sched.cuh"
 
 namespace irr {
 
 struct DcwiGemmProb {
     GemmArgs g;
     const int *mask;  // optional: skip matrices with mask[i] < 0 (bad arguments)
-    __device__ bool get(int i, GemmDesc &d) const {
+    SlotList sl;      // slot -> matrix (identity, or a size-sorted prefix)
+    __device__ bool get(int slot, GemmDesc &d) const {
+        const int i = sl.matrix(slot);
         d.m = 0; d.n = 0; d.k = 0;
         if (mask && mask[i] < 0) return false;
         const int mi = g.m[i], ni = g.n[i], ki = g.k[i];
@@ -38,32 +41,46 @@ struct DcwiGemmProb {
     }
 };
 
-void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s) {
+void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s,
+                        SlotList sl) {
     if (g.batch <= 0 || g.max_m <= 0 || g.max_n <= 0) return;
-    DcwiGemmProb P{g, mask};
     const int sms = num_sms();
     if (tile_off) {
+        DcwiGemmProb P{g, mask, sl};
+        const int cnt = sl.prefix ? -1 : g.batch;
+        const int *cnt_ptr = sl.prefix ? sl.prefix + sl.bucket0 : nullptr;
         {
             KScope k(K_GEMM_SCAN, s);
-            gemm_scan_kernel<DcwiGemmProb><<<1, 1024, 0, s>>>(P, g.batch, nullptr, tile_off);
+            gemm_scan_kernel<DcwiGemmProb><<<1, 1024, 0, s>>>(P, cnt, cnt_ptr, tile_off);
         }
         KScope k(K_GEMM_DCWI, s);
-        gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb>);
-        gemm_sched_kernel<DcwiGemmProb><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, g.batch, nullptr, tile_off);
+        if (tuning().dmma) {
+            gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb, true>);
+            gemm_sched_kernel<DcwiGemmProb, true><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+        } else {
+            gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb, false>);
+            gemm_sched_kernel<DcwiGemmProb, false><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+        }
     } else {
+        DcwiGemmProb P{g, mask, all_slots()};
         const int tm = (g.max_m + GBM - 1) / GBM, tn = (g.max_n + GBN - 1) / GBN;
         long long total = (long long)tm * tn * g.batch;
         int grid = sms * 4;
         if (total < grid) grid = (int)total;
         KScope k(K_GEMM_DCWI, s);
-        gemm_smem_optin(gemm_grid_kernel<DcwiGemmProb>);
-        gemm_grid_kernel<DcwiGemmProb><<<grid, G_NT, GEMM_SMEM, s>>>(P, g.batch, tm, tn);
+        if (tuning().dmma) {
+            gemm_smem_optin(gemm_grid_kernel<DcwiGemmProb, true>);
+            gemm_grid_kernel<DcwiGemmProb, true><<<grid, G_NT, GEMM_SMEM, s>>>(P, g.batch, tm, tn);
+        } else {
+            gemm_smem_optin(gemm_grid_kernel<DcwiGemmProb, false>);
+            gemm_grid_kernel<DcwiGemmProb, false><<<grid, G_NT, GEMM_SMEM, s>>>(P, g.batch, tm, tn);
+        }
     }
     (void)counters;
 }
 
 void launch_gemm_dcwi(const GemmArgs &g, int *counters, int *tile_off, cudaStream_t s) {
-    launch_gemm_masked(g, nullptr, counters, tile_off, s);
+    launch_gemm_masked(g, nullptr, counters, tile_off, s, all_slots());
 }
 
 }  // namespace irr

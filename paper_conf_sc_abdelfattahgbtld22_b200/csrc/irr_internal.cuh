@@ -22,6 +22,9 @@ struct Tuning {
     int l1;          // 1: CTA-per-matrix tier for tier-L matrices with m <= L1_MAX_ROWS
     int phase_timing;  // 1: accumulate per-phase SM cycles into the workspace counters
     int l1_ctas_per_sm;  // resident CTAs per SM of the L1 kernel (1..3)
+    int concurrent;      // 1: tiers S/M on a forked stream, concurrent with L1/L2
+    int dmma;            // 1: grid-wide GEMMs on the FP64 tensor core (mma.sync DMMA), 0: DFMA
+    int l1_dmma;         // same switch for the GEMM phase inside the L1 kernel
 };
 Tuning &tuning();
 

@@ -8,6 +8,7 @@
 // per column (gather into shared memory, scatter back).  The widths are per
 // matrix (DCWI: columns [Aj, Aj + min(max_n, n_i - Aj))).
 #include "irr_internal.cuh"
+#include "sched.cuh"
 
 namespace irr {
 
@@ -28,7 +29,21 @@ struct LaswpArgs {
     int chunks;
 };
 
-__global__ void __launch_bounds__(LS_NT) laswp_kernel(LaswpArgs g) {
+struct LaswpUnits {
+    LaswpArgs g;
+    __device__ int units(int i) const {
+        if (g.mask && g.mask[i] < 0) return 0;
+        const int ncol = imin(g.max_n, g.n[i] - g.Aj);
+        const int kend = imin(g.k2, g.kcount[i]);
+        if (ncol <= 0 || kend <= g.k1) return 0;
+        return (ncol + LS_COLS - 1) / LS_COLS;
+    }
+};
+
+// WALK = false: DCWI grid over batch x chunks of the required width;
+// WALK = true : only the (matrix, chunk) units that exist (device schedule).
+template <bool WALK>
+__global__ void __launch_bounds__(LS_NT) laswp_kernel(LaswpArgs g, SlotList sl, const int *units_off) {
     extern __shared__ __align__(16) unsigned char ls_smem[];
     const int span = g.k2 - g.k1;
     int *top_src = (int *)ls_smem;             // [span]
@@ -39,16 +54,14 @@ __global__ void __launch_bounds__(LS_NT) laswp_kernel(LaswpArgs g) {
     double *vals = (double *)(((uintptr_t)(mv_src + 2 * span) + 15) & ~(uintptr_t)15);  // [2 span]
     __shared__ int nbot_s, nmov_s;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const long long total = (long long)g.batch * g.chunks;
     int last_i = -1;
-    for (long long w = blockIdx.x; w < total; w += gridDim.x) {
-        const int i = (int)(w / g.chunks), q = (int)(w - (long long)i * g.chunks);
-        if (g.mask && g.mask[i] < 0) continue;
+    auto body = [&](int i, int q) {
+        if (g.mask && g.mask[i] < 0) return;
         const int ncol = imin(g.max_n, g.n[i] - g.Aj);
         const int kend = imin(g.k2, g.kcount[i]);
-        if (ncol <= 0 || kend <= g.k1) continue;
+        if (ncol <= 0 || kend <= g.k1) return;
         const int c0 = q * LS_COLS;
-        if (c0 >= ncol) continue;
+        if (c0 >= ncol) return;
         const int W = imin(LS_COLS, ncol - c0);
         const long lda = g.lda[i];
         double *A = g.A[i] + g.Ai + (size_t)g.Aj * lda;
@@ -127,6 +140,15 @@ __global__ void __launch_bounds__(LS_NT) laswp_kernel(LaswpArgs g) {
             for (int e = tid; e < nmov; e += LS_NT) col[mv_dst[e]] = vals[e];
             __syncthreads();
         }
+    };
+    if (WALK) {
+        walk_units(sl, g.batch, units_off, body);
+    } else {
+        const long long total = (long long)g.batch * g.chunks;
+        for (long long w = blockIdx.x; w < total; w += gridDim.x) {
+            const int i = (int)(w / g.chunks), q = (int)(w - (long long)i * g.chunks);
+            body(i, q);
+        }
     }
 }
 
@@ -134,26 +156,43 @@ size_t laswp_smem(int span) {
     return (size_t)span * 7 * sizeof(int) + 16 + (size_t)span * 2 * sizeof(double);
 }
 
+// units_off: optional int[batch+1] workspace -> device-scheduled walk over
+// the slots of `sl`; nullptr -> DCWI grid (the exported irr_laswp has no workspace).
 void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
-                         const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s) {
+                         const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s,
+                         int *units_off, SlotList sl) {
     if (batch <= 0 || max_n <= 0 || k2 <= k1) return;
     LaswpArgs g{max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, mask, (max_n + LS_COLS - 1) / LS_COLS};
     size_t smem = laswp_smem(k2 - k1);
+    if (units_off) {
+        static size_t attr = 0;
+        if (smem > 48 * 1024 && smem > attr) {
+            cudaFuncSetAttribute(laswp_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            attr = smem;
+        }
+        {
+            KScope k(K_GEMM_SCAN, s);
+            scan_units_kernel<LaswpUnits><<<1, 1024, 0, s>>>(LaswpUnits{g}, sl, batch, units_off);
+        }
+        KScope k(K_LASWP, s);
+        laswp_kernel<true><<<num_sms() * 4, LS_NT, smem, s>>>(g, sl, units_off);
+        return;
+    }
     static size_t attr = 0;
     if (smem > 48 * 1024 && smem > attr) {
-        cudaFuncSetAttribute(laswp_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(laswp_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
     long long total = (long long)batch * g.chunks;
     int grid = num_sms() * 4;
     if (total < grid) grid = (int)total;
     KScope k(K_LASWP, s);
-    laswp_kernel<<<grid, LS_NT, smem, s>>>(g);
+    laswp_kernel<false><<<grid, LS_NT, smem, s>>>(g, all_slots(), nullptr);
 }
 
 void launch_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const int *lda, int k1, int k2,
                   const int *kcount, int *const *ipiv, int batch, cudaStream_t s) {
-    launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, s);
+    launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, s, nullptr, all_slots());
 }
 
 }  // namespace irr

@@ -189,6 +189,7 @@ __device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni
 
 // ================================================================== L1
 // One CTA per matrix, all iterations inside (matrices with m <= L1 rows).
+template <bool DMMA>
 __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__restrict__ counters,
                                                          const int *__restrict__ bins, int nb,
                                                          int l1_region_doubles, int phase_timing) {
@@ -278,7 +279,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                     ++tt;
                     return true;
                 };
-                gemm_tile_stream(next, gsm);
+                gemm_tile_stream<DMMA>(next, gsm);
             }
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 2, (unsigned long long)(t1 - t0)); t0 = t1; }
@@ -404,7 +405,8 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
     const size_t smem = region + (size_t)(nb * (nb - 1) / 2 + 2) * sizeof(double);
     static size_t attr = 0;
     if (smem > attr) {
-        cudaFuncSetAttribute(lu_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
     int per_sm = tuning().l1_ctas_per_sm;
@@ -412,8 +414,12 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     KScope k(K_LU_L1, s);
-    lu_l1_kernel<<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
-                                           tuning().phase_timing);
+    if (tuning().l1_dmma)  // measured: DFMA is faster inside L1 (DMMA variant spills)
+        lu_l1_kernel<true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
+                                                     tuning().phase_timing);
+    else
+        lu_l1_kernel<false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
+                                                      tuning().phase_timing);
 }
 
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s) {
@@ -461,9 +467,15 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         }
         {
             KScope k(K_GEMM_TRAIL, s);
-            gemm_smem_optin(gemm_sched_kernel<TrailingProb>);
-            gemm_sched_kernel<TrailingProb><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, -1, counters + CNT_BIN0 + BIN_L,
-                                                                           tile_off);
+            if (tu.dmma) {
+                gemm_smem_optin(gemm_sched_kernel<TrailingProb, true>);
+                gemm_sched_kernel<TrailingProb, true><<<sms * 3, G_NT, GEMM_SMEM, s>>>(
+                    P, -1, counters + CNT_BIN0 + BIN_L, tile_off);
+            } else {
+                gemm_smem_optin(gemm_sched_kernel<TrailingProb, false>);
+                gemm_sched_kernel<TrailingProb, false><<<sms * 3, G_NT, GEMM_SMEM, s>>>(
+                    P, -1, counters + CNT_BIN0 + BIN_L, tile_off);
+            }
         }
     }
 }

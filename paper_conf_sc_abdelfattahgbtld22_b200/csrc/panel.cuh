@@ -48,9 +48,9 @@ __shared__ unsigned long long s_ptime[8];
 
 template <int NW, int NBP>
 struct PanelRegScratch {
+    double row[2][NW][NBP];  // first: 16-byte aligned for the pair stores; row[.][w][0] = signed candidate
     unsigned long long key[2][NW];
     int pos[2][NW];
-    double row[2][NW][NBP];  // row[.][w][0] is the signed candidate value
 };
 
 // One column step of panel_regs on the W active (shifted) columns.

@@ -9,10 +9,12 @@
 // out-of-place workspace copy: leaves use plain substitution with
 // true division, in place.
 #include "gemm_core.cuh"
+#include "sched.cuh"
 
 namespace irr {
 
-void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s);
+void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *tile_off, cudaStream_t s,
+                        SlotList sl);
 
 constexpr int TL = 32;        // leaf size (triangular dimension)
 constexpr int TR_RHS = 128;   // right-hand sides per CTA
@@ -29,36 +31,51 @@ struct LeafArgs {
     int rhs_chunks;
 };
 
-__global__ void __launch_bounds__(TR_NT) trsm_leaf_kernel(LeafArgs L) {
-    __shared__ double S[TL][TL + 1];
-    __shared__ double buf[TL][TR_RHS + 1];
+// DCWI of one leaf for matrix i: effective triangle size and RHS count
+__device__ __forceinline__ void leaf_dims(const LeafArgs &L, int i, int &kt, int &nrhs) {
+    const TrsmArgs &t = L.t;
+    kt = 0;
+    nrhs = 0;
+    if (L.mask && L.mask[i] < 0) return;
+    const bool left = t.side == IRR_LEFT;
+    const int mi = t.m[i], ni = t.n[i];
+    const int tri = left ? mi : ni;  // local size of T
+    kt = imin(L.kt, imin(tri - (t.Ti + L.off), tri - (t.Tj + L.off)));
+    if (left) {
+        kt = imin(kt, mi - (t.Bi + L.off));
+        nrhs = imin(t.max_n, ni - t.Bj);
+    } else {
+        kt = imin(kt, ni - (t.Bj + L.off));
+        nrhs = imin(t.max_m, mi - t.Bi);
+    }
+}
+
+struct LeafUnits {
+    LeafArgs L;
+    __device__ int units(int i) const {
+        int kt, nrhs;
+        leaf_dims(L, i, kt, nrhs);
+        return (kt > 0 && nrhs > 0) ? (nrhs + TR_RHS - 1) / TR_RHS : 0;
+    }
+};
+
+// one (matrix, RHS chunk) leaf solve by the whole CTA
+__device__ __forceinline__ void leaf_item(const LeafArgs &L, int i, int q, double (*S)[TL + 1],
+                                          double (*buf)[TR_RHS + 1]) {
     const TrsmArgs &t = L.t;
     const int tid = threadIdx.x;
     const bool left = t.side == IRR_LEFT;
-    const long long total = (long long)t.batch * L.rhs_chunks;
-    for (long long w = blockIdx.x; w < total; w += gridDim.x) {
-        const int i = (int)(w / L.rhs_chunks), q = (int)(w - (long long)i * L.rhs_chunks);
-        if (L.mask && L.mask[i] < 0) continue;
-        const int mi = t.m[i], ni = t.n[i];
-        const int tri = left ? mi : ni;  // local size of T
-        const int toff_r = t.Ti + L.off, toff_c = t.Tj + L.off;
-        int kt = imin(L.kt, imin(tri - toff_r, tri - toff_c));
-        int nrhs;
-        if (left) {
-            kt = imin(kt, mi - (t.Bi + L.off));
-            nrhs = imin(t.max_n, ni - t.Bj);
-        } else {
-            kt = imin(kt, ni - (t.Bj + L.off));
-            nrhs = imin(t.max_m, mi - t.Bi);
-        }
-        if (kt <= 0) continue;
+    int kt, nrhs;
+    leaf_dims(L, i, kt, nrhs);
+    const int toff_r = t.Ti + L.off, toff_c = t.Tj + L.off;
+    {
+        if (kt <= 0) return;
         const int r0 = q * TR_RHS;
-        if (r0 >= nrhs) continue;
+        if (r0 >= nrhs) return;
         const int W = imin(TR_RHS, nrhs - r0);
         const long ldt = t.ldt[i], ldb = t.ldb[i];
         const double *T = t.T[i];
         double *B = t.B[i];
-        __syncthreads();
         // ---- S = the solved triangle (dense, zeros outside, unit diag)
         for (int e = tid; e < kt * kt; e += TR_NT) {
             const int r = e % kt, c = e / kt;
@@ -124,7 +141,26 @@ __global__ void __launch_bounds__(TR_NT) trsm_leaf_kernel(LeafArgs L) {
                 B[t.Bi + r0 + c + (size_t)(t.Bj + L.off + r) * ldb] = buf[r][c];
             }
         }
+        __syncthreads();
     }
+}
+
+// DCWI grid over (batch x RHS chunks of the required dims) (no workspace)
+__global__ void __launch_bounds__(TR_NT) trsm_leaf_kernel(LeafArgs L) {
+    __shared__ double S[TL][TL + 1];
+    __shared__ double buf[TL][TR_RHS + 1];
+    const long long total = (long long)L.t.batch * L.rhs_chunks;
+    for (long long w = blockIdx.x; w < total; w += gridDim.x) {
+        const int i = (int)(w / L.rhs_chunks), q = (int)(w - (long long)i * L.rhs_chunks);
+        leaf_item(L, i, q, S, buf);
+    }
+}
+
+// device-scheduled: only (matrix, chunk) units that exist, on the active slots
+__global__ void __launch_bounds__(TR_NT) trsm_leaf_walk_kernel(LeafArgs L, SlotList sl, const int *off) {
+    __shared__ double S[TL][TL + 1];
+    __shared__ double buf[TL][TR_RHS + 1];
+    walk_units(sl, L.t.batch, off, [&](int i, int q) { leaf_item(L, i, q, S, buf); });
 }
 
 namespace {
@@ -133,6 +169,7 @@ struct TrsmRec {
     TrsmArgs t;
     const int *mask;
     int *counters, *tile_off;
+    int *sort_ws;  // size-sorted slots by the triangular dimension (nullptr: none)
     cudaStream_t s;
     int leaf;
     int m_lower;  // op(T) is lower triangular
@@ -147,6 +184,16 @@ struct TrsmRec {
         L.tr = left ? (t.trans == IRR_TRANS) : (t.trans != IRR_TRANS);
         const int nrhs_max = left ? t.max_n : t.max_m;
         L.rhs_chunks = (nrhs_max + TR_RHS - 1) / TR_RHS;
+        if (tile_off) {
+            const SlotList sl = slots(off);
+            {
+                KScope k(K_GEMM_SCAN, s);
+                scan_units_kernel<LeafUnits><<<1, 1024, 0, s>>>(LeafUnits{L}, sl, t.batch, tile_off);
+            }
+            KScope k(K_TRSM_LEAF, s);
+            trsm_leaf_walk_kernel<<<num_sms() * 8, TR_NT, 0, s>>>(L, sl, tile_off);
+            return;
+        }
         long long total = (long long)t.batch * L.rhs_chunks;
         int grid = num_sms() * 8;
         if (total < grid) grid = (int)total;
@@ -154,6 +201,9 @@ struct TrsmRec {
         KScope k(K_TRSM_LEAF, s);
         trsm_leaf_kernel<<<grid, TR_NT, 0, s>>>(L);
     }
+
+    // matrices whose triangular dimension exceeds `thr` (all when unsorted)
+    SlotList slots(int thr) const { return sort_ws ? sorted_slots(sort_ws, t.batch, thr) : all_slots(); }
 
     // op(T) block with rows [R, R+nr) and columns [C, C+nc) as a GEMM operand
     void opT_operand(int R, int C, int &trans, int &oi, int &oj) const {
@@ -189,7 +239,7 @@ struct TrsmRec {
             g.B = t.T; g.Bi = oi; g.Bj = oj; g.ldb = t.ldt;
             g.C = t.B; g.Ci = t.Bi; g.Cj = t.Bj + off_c; g.ldc = t.ldb;
         }
-        launch_gemm_masked(g, mask, counters, tile_off, s);
+        launch_gemm_masked(g, mask, counters, tile_off, s, slots(off_x < off_c ? off_x : off_c));
     }
 
     void solve(int off, int K, double alpha) {
@@ -216,10 +266,15 @@ struct TrsmRec {
 
 }  // namespace
 
-void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *tile_off, cudaStream_t s) {
+// sort_ws: nullptr, or a size sort of the batch by the triangular dimension
+// (launch_size_sort on t.m for LEFT, t.n for RIGHT) that TRSM levels use to
+// visit only the matrices still active at their offset.
+void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *tile_off, cudaStream_t s,
+                     int *sort_ws) {
     if (t.batch <= 0 || t.max_m <= 0 || t.max_n <= 0) return;
     TrsmRec R;
     R.t = t; R.mask = mask; R.counters = counters; R.tile_off = tile_off; R.s = s;
+    R.sort_ws = tile_off ? sort_ws : nullptr;
     int leaf = tuning().trsm_nb;
     if (leaf < 1 || leaf > TL) leaf = TL;
     R.leaf = leaf;
@@ -229,7 +284,7 @@ void run_trsm_masked(const TrsmArgs &t, const int *mask, int *counters, int *til
 }
 
 void run_trsm(const TrsmArgs &t, int *counters, int *tile_off, cudaStream_t s) {
-    run_trsm_masked(t, nullptr, counters, tile_off, s);
+    run_trsm_masked(t, nullptr, counters, tile_off, s, nullptr);
 }
 
 }  // namespace irr

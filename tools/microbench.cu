@@ -88,7 +88,7 @@ __global__ void k_dfma_tput(double *out, long long *cyc, double a, double b) {
     if (threadIdx.x == 0 && blockIdx.x == 0) cyc[0] = t1 - t0;
 }
 
-int main() {
+int main1() {
     double *dd; unsigned *du; int *di; long long *dc; long long hc;
     cudaMalloc(&dd, 1 << 20); cudaMalloc(&du, 1 << 20); cudaMalloc(&di, 1 << 20); cudaMalloc(&dc, 64);
     k_dfma<<<1, 32>>>(dd, dc, 1.0000001, 1e-9); cudaMemcpy(&hc, dc, 8, cudaMemcpyDeviceToHost);
@@ -111,3 +111,34 @@ int main() {
     }
     return 0;
 }
+
+// ---- FP64 tensor core (mma.sync m8n8k4 f64 -> SASS DMMA) throughput
+__global__ void k_dmma(double *out, long long *cyc) {
+    double a = threadIdx.x * 1e-3, b = 1.0 + threadIdx.x * 1e-4;
+    double c[8][2];
+    for (int j = 0; j < 8; ++j) { c[j][0] = 0; c[j][1] = 0; }
+    long long t0 = clock64();
+    for (int i = 0; i < N; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j)
+            asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                         : "+d"(c[j][0]), "+d"(c[j][1]) : "d"(a), "d"(b));
+    }
+    long long t1 = clock64();
+    double s = 0;
+    for (int j = 0; j < 8; ++j) s += c[j][0] + c[j][1];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+    if (threadIdx.x == 0 && blockIdx.x == 0) cyc[0] = t1 - t0;
+}
+
+int main2() {
+    double *dd; long long *dc; long long hc;
+    cudaMalloc(&dd, 1 << 22); cudaMalloc(&dc, 64);
+    for (int w : {1, 4, 8, 16}) {
+        k_dmma<<<1, 32 * w>>>(dd, dc); cudaMemcpy(&hc, dc, 8, cudaMemcpyDeviceToHost);
+        double per = (double)hc / (N * 8.0 * w);
+        printf("DMMA m8n8k4, %2d warps: %.2f cycles per warp-mma per SM -> %.0f FMA/clk/SM\n", w, per, 256.0 / per);
+    }
+    return 0;
+}
+int main() { main1(); return main2(); }
