@@ -32,15 +32,7 @@ constexpr int L1_NT = 128;    // threads of the CTA-per-matrix kernel (== G_NT =
 static_assert(L1_NT == G_NT && L1_NT == SW_NT, "L1 composes the GEMM and swap pieces at one CTA size");
 
 // ------------------------------------------------------------------ swap plan
-// Composition of the ib interchanges of one panel (rows j .. j+ib-1) on an
-// index list: position j+t receives row top_src[t]; position bot_pos[b] (below
-// the panel block) receives row bot_src[b].
-struct SwapPlan {
-    int top_src[NBMAX];
-    int piv[NBMAX];
-    int bot_pos[NBMAX], bot_src[NBMAX];
-    int nbot;
-};
+// (SwapPlan is defined in panel.cuh: panel_regs can emit it directly.)
 
 // Warp 0 composes the interchanges held in sp.piv[0..ib) (0-based absolute
 // rows).  Caller synchronises the CTA afterwards.
@@ -128,8 +120,15 @@ __device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const 
 // trsm_col_regs.  top / bot: shared buffers of nb x (SW_COLS+1).  SW_NT threads.
 __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int cbeg, int W,
                                            bool solve, const SwapPlan &sp, const double *L11, int ldl,
-                                           double *top, double *bot) {
+                                           double *top, double *bot, unsigned long long *ph = nullptr) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    long long tq = (ph && tid == 0) ? clock64() : 0;
+#define SWAP_PHASE(k)                                                         \
+    if (ph && tid == 0) {                                                     \
+        long long t1 = clock64();                                             \
+        atomicAdd(ph + (k), (unsigned long long)(t1 - tq));                   \
+        tq = t1;                                                              \
+    }
     constexpr int LT = SW_COLS + 1;
     constexpr int NWS = SW_NT / 32;
     const int nbot = sp.nbot;
@@ -142,6 +141,7 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
     cp_async_commit();
     cp_async_wait<0>();
     __syncthreads();
+    SWAP_PHASE(5)
     if (solve && tid < W) {
         // one thread per column, the column in registers (the smem
         // read-modify-write form was a serial LDS->DFMA->STS chain)
@@ -156,12 +156,15 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
         }
     }
     __syncthreads();
+    SWAP_PHASE(6)
     for (int c = warp; c < W; c += NWS) {
         double *gc = gA + (size_t)(cbeg + c) * ld;
         for (int t = lane; t < ib; t += 32) gc[j + t] = top[t * LT + c];
         for (int b = lane; b < nbot; b += 32) gc[sp.bot_pos[b]] = bot[b * LT + c];
     }
     __syncthreads();
+    SWAP_PHASE(7)
+#undef SWAP_PHASE
 }
 
 // L11 (ib x ib diagonal block at (j, j)) -> shared memory, column-major (ldl)
@@ -231,7 +234,8 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
             cp_async_wait<0>();
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 3, (unsigned long long)(t1 - t0)); t0 = t1; }
-            const int z = (ib <= 32) ? panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs)
+            const bool regs_panel = ib <= 32;
+            const int z = regs_panel ? panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs, &sp, j)
                                      : panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 4, (unsigned long long)(t1 - t0)); t0 = t1; }
             if (z && !info) info = j + z;
@@ -258,14 +262,18 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
             if (j > 0 || c1 < ni) {
                 double *top = smd;
                 double *bot = top + nb * (SW_COLS + 1);
-                plan_swaps_from(piv_s, j, ib, sp);
-                __syncthreads();
+                if (!regs_panel) {  // panel_regs already emitted the plan
+                    plan_swaps_from(piv_s, j, ib, sp);
+                    __syncthreads();
+                }
+                unsigned long long *phs = phase_timing ? ph : nullptr;
+                if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 1, (unsigned long long)(t1 - t0)); t0 = t1; }
                 for (int cb = 0; cb < j; cb += SW_COLS)
-                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, j - cb), false, sp, L11p, 0, top, bot);
+                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, j - cb), false, sp, L11p, 0, top, bot, phs);
                 for (int cb = c1; cb < ni; cb += SW_COLS)
-                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, ni - cb), true, sp, L11p, 0, top, bot);
+                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, ni - cb), true, sp, L11p, 0, top, bot, phs);
             }
-            if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 1, (unsigned long long)(t1 - t0)); t0 = t1; }
+            if (phase_timing && tid == 0) t0 = clock64();  // chunk phases were accounted in slots 5..7
             // ---- a4.4 trailing update through the pipelined GEMM core
             GemmDesc d0;
             if (trailing_desc(gA, ld, mi, ni, j, nb, d0)) {

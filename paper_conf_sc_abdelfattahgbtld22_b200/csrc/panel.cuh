@@ -10,6 +10,16 @@
 
 namespace irr {
 
+// Composition of the ib interchanges of one panel (rows j .. j+ib-1) on an
+// index list: position j+t receives row top_src[t]; position bot_pos[b] (below
+// the panel block) receives row bot_src[b].
+struct SwapPlan {
+    int top_src[64];
+    int piv[64];
+    int bot_pos[64], bot_src[64];
+    int nbot;
+};
+
 struct PanelScratch {
     unsigned long long key[32];
     int row[32];
@@ -177,8 +187,10 @@ __device__ __forceinline__ void preg_step(double (&a)[RPT][NBP], int (&pos)[RPT]
 // the first exact zero pivot, or 0.  All NT threads must call it.  The active
 // width W shrinks NBP -> NBP/2 -> ... -> 4 with the remaining columns.
 template <int NT, int RPT, int NBP>
-__device__ int panel_regs(double *P, int ldp, int rows, int ib, int *piv, PanelRegScratch<NT / 32, NBP> &sc) {
+__device__ int panel_regs(double *P, int ldp, int rows, int ib, int *piv, PanelRegScratch<NT / 32, NBP> &sc,
+                          SwapPlan *plan = nullptr, int row0 = 0) {
     const int tid = threadIdx.x;
+    if (plan && tid == 0) plan->nbot = 0;
     double a[RPT][NBP];
     int pos[RPT];
 #pragma unroll
@@ -198,6 +210,26 @@ __device__ int panel_regs(double *P, int ldp, int rows, int ib, int *piv, PanelR
         for (; c < ib && ib - c > 8; ++c) preg_step<NT, RPT, NBP, (NBP >= 16 ? 16 : NBP)>(a, pos, c, P, ldp, rows, ib, piv, sc, zero_at);
     for (; c < ib && ib - c > 4; ++c) preg_step<NT, RPT, NBP, 8>(a, pos, c, P, ldp, rows, ib, piv, sc, zero_at);
     for (; c < ib; ++c) preg_step<NT, RPT, NBP, 4>(a, pos, c, P, ldp, rows, ib, piv, sc, zero_at);
+    if (plan) {
+        // the interchange plan straight from the final positions (parallel;
+        // replaces composing the ib interchanges serially): a row ending in
+        // the top block names its source; a row pushed below it came from the
+        // top block and becomes a (pos, src) pair.  Absolute rows = row0 + .
+#pragma unroll
+        for (int q = 0; q < RPT; ++q) {
+            const int r = tid + NT * q;
+            if (r < rows) {
+                const int p = pos[q];
+                if (p < ib) {
+                    plan->top_src[p] = row0 + r;
+                } else if (p != r) {
+                    const int b = atomicAdd(&plan->nbot, 1);
+                    plan->bot_pos[b] = row0 + p;
+                    plan->bot_src[b] = row0 + r;
+                }
+            }
+        }
+    }
     __syncthreads();
     return zero_at;
 }

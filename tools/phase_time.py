@@ -17,7 +17,8 @@ import irrgen  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200.batch import MatrixBatch  # noqa: E402
 
-NAMES = ["L1 panel", "L1 swap+trsm", "L1 gemm", "M load", "M panel", "M trsm", "M gemm", "M store"]
+NAMES = ["L1 panel wb / (M: -)", "L1 swap plan", "L1 gemm", "L1 stage | M load", "L1 panel | M panel",
+         "L1 gather | M trsm", "L1 trsm | M gemm", "L1 scatter | M store"]
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
