@@ -253,13 +253,21 @@ def main():
     from paper_conf_sc_abdelfattahgbtld22_b200 import irr
     from paper_conf_sc_abdelfattahgbtld22_b200.batch import FrontBatch, MatrixBatch
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # one process per GPU; IRR_BENCH_DIST_BACKEND=gloo is a test-only override
+    # that lets several ranks share one GPU (exercises the N > 1 code path)
+    backend = os.environ.get("IRR_BENCH_DIST_BACKEND", "nccl")
+    dev_idx = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(dev_idx)
+    dev = torch.device("cuda", dev_idx)
     for kv in args.tune:
         k, v = kv.split("=")
         irr.irr_set_tuning(k, int(v))
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+    coll_dev = dev if backend == "nccl" else torch.device("cpu")
 
     # ---- workload: global batch = world x config, LPT-sharded by flops
     cfg = irrgen.config(args.config, scale=float(world))
@@ -302,8 +310,8 @@ def main():
 
     # status gather (the only collective): per-matrix info words, padded
     pad = int(max(np.bincount(owner, minlength=world))) if world > 1 else len(mine)
-    status = torch.zeros(max(1, pad), dtype=torch.int32, device=dev)
-    gathered = torch.zeros(world * max(1, pad), dtype=torch.int32, device=dev) if world > 1 else None
+    status = torch.zeros(max(1, pad), dtype=torch.int32, device=coll_dev)
+    gathered = torch.zeros(world * max(1, pad), dtype=torch.int32, device=coll_dev) if world > 1 else None
 
     def step():
         call()
@@ -324,7 +332,7 @@ def main():
     # ---- timed region
     irr.irr_profile_enable(100000)
     irr.irr_launch_count(reset=True)
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(dev_idx)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -346,7 +354,7 @@ def main():
     launches = irr.irr_launch_count()
     prof = irr.irr_profile_collect()
     irr.irr_profile_enable(0)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=coll_dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_max_ms = float(t.item())
@@ -379,7 +387,7 @@ def main():
             torch.cuda.synchronize()
             if s >= args.warmup:
                 e_ms.append(a.elapsed_time(b))
-        te = torch.tensor([float(np.sum(e_ms))], dtype=torch.float64, device=dev)
+        te = torch.tensor([float(np.sum(e_ms))], dtype=torch.float64, device=coll_dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
         e_step = float(te.item()) / args.steps
