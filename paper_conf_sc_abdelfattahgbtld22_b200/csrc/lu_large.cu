@@ -115,12 +115,17 @@ __device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const 
     }
 }
 
-// Apply the plan to columns [cbeg, cbeg+W) of one matrix; when `solve`, also
-// U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory in the layouts of
-// trsm_col_regs.  top / bot: shared buffers of nb x (SW_COLS+1).  SW_NT threads.
-__device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int cbeg, int W,
-                                           bool solve, const SwapPlan &sp, const double *L11, int ldl,
-                                           double *top, double *bot, unsigned long long *ph = nullptr) {
+// Apply the plan to W columns of one matrix given as a VIRTUAL range
+// [vbeg, vbeg+W): virtual column v is real column v (v < jsplit) or v + shift
+// (v >= jsplit), so one chunk can span the left block [0, j) and the right
+// block [j+ib, n) (fewer gather/solve/scatter rounds).  Real columns >=
+// solve_from also get U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory in
+// the layouts of trsm_col_regs.  top / bot: shared buffers of nb x
+// (SW_COLS+1).  SW_NT threads.
+__device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int vbeg, int W,
+                                           int jsplit, int shift, int solve_from, const SwapPlan &sp,
+                                           const double *L11, int ldl, double *top, double *bot,
+                                           unsigned long long *ph = nullptr) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     long long tq = (ph && tid == 0) ? clock64() : 0;
 #define SWAP_PHASE(k)                                                         \
@@ -134,7 +139,8 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
     const int nbot = sp.nbot;
     // warps over columns, lanes over the (<= 64) moved rows: no integer division
     for (int c = warp; c < W; c += NWS) {
-        const double *gc = gA + (size_t)(cbeg + c) * ld;
+        const int v = vbeg + c, col = v < jsplit ? v : v + shift;
+        const double *gc = gA + (size_t)col * ld;
         for (int t = lane; t < ib; t += 32) cp_async8(&top[t * LT + c], gc + sp.top_src[t]);
         for (int b = lane; b < nbot; b += 32) cp_async8(&bot[b * LT + c], gc + sp.bot_src[b]);
     }
@@ -142,23 +148,27 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
     cp_async_wait<0>();
     __syncthreads();
     SWAP_PHASE(5)
-    if (solve && tid < W) {
-        // one thread per column, the column in registers (the smem
-        // read-modify-write form was a serial LDS->DFMA->STS chain)
-        if (ib <= 32) {
-            trsm_col_regs<32>(top + tid, LT, ib, L11, ldl);
-        } else {  // nb > 32 (tuning only): plain shared-memory substitution
-            for (int s = 0; s < ib; ++s) {
-                const double x = top[s * LT + tid];
-                const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
-                for (int r = s + 1; r < ib; ++r) top[r * LT + tid] = fma(-Ls[r - s - 1], x, top[r * LT + tid]);
+    if (tid < W) {
+        const int v = vbeg + tid, col = v < jsplit ? v : v + shift;
+        if (col >= solve_from) {
+            // one thread per column, the column in registers (the smem
+            // read-modify-write form was a serial LDS->DFMA->STS chain)
+            if (ib <= 32) {
+                trsm_col_regs<32>(top + tid, LT, ib, L11, ldl);
+            } else {  // nb > 32 (tuning only): plain shared-memory substitution
+                for (int s = 0; s < ib; ++s) {
+                    const double x = top[s * LT + tid];
+                    const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
+                    for (int r = s + 1; r < ib; ++r) top[r * LT + tid] = fma(-Ls[r - s - 1], x, top[r * LT + tid]);
+                }
             }
         }
     }
     __syncthreads();
     SWAP_PHASE(6)
     for (int c = warp; c < W; c += NWS) {
-        double *gc = gA + (size_t)(cbeg + c) * ld;
+        const int v = vbeg + c, col = v < jsplit ? v : v + shift;
+        double *gc = gA + (size_t)col * ld;
         for (int t = lane; t < ib; t += 32) gc[j + t] = top[t * LT + c];
         for (int b = lane; b < nbot; b += 32) gc[sp.bot_pos[b]] = bot[b * LT + c];
     }
@@ -268,10 +278,10 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                 }
                 unsigned long long *phs = phase_timing ? ph : nullptr;
                 if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 1, (unsigned long long)(t1 - t0)); t0 = t1; }
-                for (int cb = 0; cb < j; cb += SW_COLS)
-                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, j - cb), false, sp, L11p, 0, top, bot, phs);
-                for (int cb = c1; cb < ni; cb += SW_COLS)
-                    swap_chunk(gA, ld, j, ib, cb, imin(SW_COLS, ni - cb), true, sp, L11p, 0, top, bot, phs);
+                // left block [0, j) and right block [c1, n) as one virtual range
+                const int vtot = j + (ni - c1);
+                for (int vb = 0; vb < vtot; vb += SW_COLS)
+                    swap_chunk(gA, ld, j, ib, vb, imin(SW_COLS, vtot - vb), j, ib, c1, sp, L11p, 0, top, bot, phs);
             }
             if (phase_timing && tid == 0) t0 = clock64();  // chunk phases were accounted in slots 5..7
             // ---- a4.4 trailing update through the pipelined GEMM core
@@ -381,7 +391,7 @@ __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int
             last_i = right ? i : -1;  // L11 only valid when loaded
             __syncthreads();
         }
-        swap_chunk(gA, ld, j, ib, cbeg, cend - cbeg, right, sp, L11, ldl, top, bot);
+        swap_chunk(gA, ld, j, ib, cbeg, cend - cbeg, 0x7fffffff, 0, right ? c1 : 0x7fffffff, sp, L11, ldl, top, bot);
     }
 }
 
