@@ -352,9 +352,11 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
     }
 }
 
-// Work item = (tier-L slot, column chunk).  Chunks 0..nleft-1 cover the
-// columns left of the panel [0, j) (interchanges only), the rest cover
-// [j+ib, n) (interchanges + forward substitution with the unit L11).
+// Work item = (tier-L slot, column chunk) over the virtual column range
+// [0, n - ib): virtual v < j is column v (interchanges only), v >= j is column
+// v + ib (interchanges + forward substitution with the unit L11).  Each CTA
+// takes a CONTIGUOUS run of items, so consecutive items share a matrix and
+// the interchange plan and L11 are built once per (CTA, matrix).
 __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                           const int *__restrict__ bins, int j, int nb,
                                                           int chunks_per) {
@@ -367,8 +369,9 @@ __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
     const long long total = (long long)count * chunks_per;
+    const long long w0 = total * blockIdx.x / gridDim.x, w1 = total * (blockIdx.x + 1) / gridDim.x;
     int last_i = -1;
-    for (long long w = blockIdx.x; w < total; w += gridDim.x) {
+    for (long long w = w0; w < w1; ++w) {
         const int slot = (int)(w / chunks_per), q = (int)(w - (long long)slot * chunks_per);
         const int i = list[slot];
         const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
@@ -376,22 +379,18 @@ __global__ void __launch_bounds__(SW_NT) swap_trsm_kernel(GetrfArgs a, const int
         if (j >= K) continue;
         const int ib = K - j < nb ? K - j : nb;
         const int c1 = j + ib;
-        const int nleft = (j + SW_COLS - 1) / SW_COLS;
-        const int nright = (ni - c1 + SW_COLS - 1) / SW_COLS;
-        if (q >= nleft + nright) continue;
-        const bool right = q >= nleft;
-        const int cbeg = right ? c1 + (q - nleft) * SW_COLS : q * SW_COLS;
-        const int cend = right ? imin(ni, cbeg + SW_COLS) : imin(j, cbeg + SW_COLS);
+        const int vtot = ni - ib, vb = q * SW_COLS;
+        if (vb >= vtot) continue;
         double *gA = a.A[i];
         if (i != last_i) {
             __syncthreads();
-            if (right) load_L11_async(L11, ldl, gA, ld, j, ib);
+            load_L11_async(L11, ldl, gA, ld, j, ib);
             cp_async_commit();
             plan_swaps(a.ipiv[i], j, ib, sp);
-            last_i = right ? i : -1;  // L11 only valid when loaded
+            last_i = i;
             __syncthreads();
         }
-        swap_chunk(gA, ld, j, ib, cbeg, cend - cbeg, 0x7fffffff, 0, right ? c1 : 0x7fffffff, sp, L11, ldl, top, bot);
+        swap_chunk(gA, ld, j, ib, vb, imin(SW_COLS, vtot - vb), j, ib, c1, sp, L11, ldl, top, bot);
     }
 }
 
@@ -458,7 +457,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     const int sms = num_sms();
     int grid_p = sms * 2;
     if (grid_p > a.batch) grid_p = a.batch;
-    const int chunks_per = (a.max_n + SW_COLS - 1) / SW_COLS + 1;
+    const int chunks_per = (a.max_n + SW_COLS - 1) / SW_COLS;
     long long sw_items = (long long)a.batch * chunks_per;
     int grid_s = sms * 8;
     if (grid_s > sw_items) grid_s = (int)sw_items;
