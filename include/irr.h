@@ -172,8 +172,10 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
  * tier for m <= 256), "l1_ctas_per_sm" (1..3), "panel_rows" (max rows of a
  * grid-wide panel staged in shared memory), "trsm_nb" (TRSM recursion leaf),
  * "concurrent" (1 = S/M tiers on a forked stream), "dmma" (1 = grid-wide GEMMs
- * on the FP64 tensor core), "l1_dmma" (same inside L1), "phase_timing"
- * (1 = per-phase cycle counters in the workspace).  Unknown keys are ignored;
+ * on the FP64 tensor core), "l1_dmma" (same inside L1), "panel_win" (1 =
+ * grid-wide panels of <= 2048 rows by the windowed register panel, 0 = the
+ * shared-memory / global-memory panels), "phase_timing" (1 = per-phase cycle
+ * counters in the workspace).  Unknown keys are ignored;
  * irr_get_tuning returns the current value (-1 for an unknown key).
  * ---------------------------------------------------------------------- */
 void irr_set_tuning(const char *key, int value);

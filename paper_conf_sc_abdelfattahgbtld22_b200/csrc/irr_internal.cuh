@@ -25,6 +25,7 @@ struct Tuning {
     int concurrent;      // 1: tiers S/M on a forked stream, concurrent with L1/L2
     int dmma;            // 1: grid-wide GEMMs on the FP64 tensor core (mma.sync DMMA), 0: DFMA
     int l1_dmma;         // same switch for the GEMM phase inside the L1 kernel
+    int panel_win;       // 1: grid-wide panels by the windowed register panel (rows <= 2048)
 };
 Tuning &tuning();
 

@@ -21,6 +21,7 @@
 //       whole GPU.
 #include "gemm_core.cuh"
 #include "panel.cuh"
+#include "panel_win.cuh"
 
 namespace irr {
 
@@ -352,6 +353,37 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
     }
 }
 
+// Windowed register panel straight on global memory (panel_win.cuh): rows
+// <= 2048 in registers (RPT = 2, 4, 8 with window 16, 8, 4), 2 CTAs / SM.
+constexpr int PW_NT = 256;
+__global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                             const int *__restrict__ bins, int j, int nb) {
+    extern __shared__ __align__(16) double pw_smem[];
+    PanelWinSmem<PW_NT / 32> &sm = *reinterpret_cast<PanelWinSmem<PW_NT / 32> *>(pw_smem);
+    __shared__ PanelScratch sc;
+    __shared__ int piv_s[NBMAX];
+    const int tid = threadIdx.x;
+    const int count = counters[CNT_BIN0 + BIN_L];
+    const int *list = bins + (size_t)BIN_L * a.batch;
+    for (int t = blockIdx.x; t < count; t += gridDim.x) {
+        const int i = list[t];
+        const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
+        const int K = mi < ni ? mi : ni;
+        if (j >= K) continue;  // DCWI: no work
+        const int ib = K - j < nb ? K - j : nb;
+        const int rows = mi - j;
+        double *gP = a.A[i] + j + (size_t)j * ld;
+        int z;
+        if (rows <= 2 * PW_NT) z = panel_win<PW_NT, 2, 16>(gP, ld, rows, ib, piv_s, sm);
+        else if (rows <= 4 * PW_NT) z = panel_win<PW_NT, 4, 8>(gP, ld, rows, ib, piv_s, sm);
+        else if (rows <= 8 * PW_NT) z = panel_win<PW_NT, 8, 4>(gP, ld, rows, ib, piv_s, sm);
+        else z = panel_getf2<PW_NT>(gP, ld, 0, rows, 0, ib, 0, ib, piv_s, sc);
+        if (tid < ib) a.ipiv[i][j + tid] = j + piv_s[tid] + 1;
+        if (tid == 0 && z && a.info[i] == 0) a.info[i] = j + z;
+        __syncthreads();
+    }
+}
+
 // Work item = (tier-L slot, column chunk) over the virtual column range
 // [0, n - ib): virtual v < j is column v (interchanges only), v >= j is column
 // v + ib (interchanges + forward substitution with the unit L11).  Each CTA
@@ -457,6 +489,14 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     const int sms = num_sms();
     int grid_p = sms * 2;
     if (grid_p > a.batch) grid_p = a.batch;
+    const size_t pw_smem = sizeof(PanelWinSmem<PW_NT / 32>);
+    static bool pw_attr = false;
+    if (!pw_attr) {
+        cudaFuncSetAttribute(panel_win_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pw_smem);
+        pw_attr = true;
+    }
+    int grid_w = sms * 2;
+    if (grid_w > a.batch) grid_w = a.batch;
     const int chunks_per = (a.max_n + SW_COLS - 1) / SW_COLS;
     long long sw_items = (long long)a.batch * chunks_per;
     int grid_s = sms * 8;
@@ -469,7 +509,10 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     }
     const int *listL = bins + (size_t)BIN_L * a.batch;
     for (int j = 0; j < Kmax; j += nb) {
-        {
+        if (tu.panel_win) {
+            KScope k(K_PANEL, s);
+            panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb);
+        } else {
             KScope k(K_PANEL, s);
             panel_kernel<<<grid_p, P_NT, psmem, s>>>(a, counters, bins, j, nb, smem_rows);
         }

@@ -191,3 +191,39 @@ def test_c3_sample_parity():
     cfg = irrgen.config("C3", scale=0.006)
     mats = [irrgen.uniform_values(cfg.seed, g, int(m), int(n)) for g, (m, n) in enumerate(zip(cfg.m, cfg.n))]
     _run_and_check(mats)
+
+
+@pytest.mark.parametrize("nb", [16, 32, 48, 64])
+def test_windowed_panel_grid_tier(nb):
+    """Grid-wide tier with the windowed register panel: every register
+    variant (rows <= 512 / 1024 / 2048) and the > 2048 global fallback,
+    tall, wide and square, window boundaries inside and at the panel edge."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("nb", nb)
+    shapes = [(700, 90), (1024, 64), (1025, 40), (1500, 33), (2048, 70), (2100, 40), (513, 513),
+              (90, 700), (600, 600), (300, 17), (257, 257)]
+    _run_and_check(_uniform(shapes, seed=31 + nb))
+
+
+def test_windowed_panel_exact_and_singular():
+    """G1 (bit-exact) and singular families through the windowed panel."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("tier_s", 0)
+    irr.irr_set_tuning("tier_m_max", 0)
+    shapes = [(1100, 80), (2000, 64), (600, 600), (40, 1300)]
+    mats = [irrgen.g1_exact(5, g, m, n)[0] for g, (m, n) in enumerate(shapes)]
+    _run_and_check(mats, exact=True)
+    cases = [(700, 700, 350), (1200, 90, 33), (520, 520, 0)]
+    mats = [irrgen.g1_singular(6, g, m, n, c)[0] for g, (m, n, c) in enumerate(cases)]
+    LUs, ipivs, info, _ = gpu_getrf(mats)
+    for (m, n, c), A, LU, ip, inf in zip(cases, mats, LUs, ipivs, info):
+        assert inf == c + 1
+        check_getrf(A, LU, ip, int(inf), exact=True, label=f"sing {m}x{n}@{c}")
+
+
+@pytest.mark.parametrize("win", [1, 0])
+def test_grid_panel_variants_agree(win):
+    """panel_win=1 (registers, global) and 0 (shared-memory / global getf2)."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("panel_win", win)
+    _run_and_check(_uniform([(800, 800), (300, 1000), (1000, 300)], seed=5))
