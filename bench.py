@@ -146,6 +146,7 @@ def class_work(m, n, nb=32, tier_m_max=24576, l1=True):
     out["gemm_trailing"] = (g_f, g_b)
     out["panel"] = (p_f, p_b)
     out["swap_trsm"] = (s_f, s_b)
+    out["strip"] = (g_f + s_f, g_b + s_b)  # fused interchange + TRSM + GEMM kernel
     return out
 
 

@@ -174,7 +174,9 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
  * "concurrent" (1 = S/M tiers on a forked stream), "dmma" (1 = grid-wide GEMMs
  * on the FP64 tensor core), "l1_dmma" (same inside L1), "panel_win" (1 =
  * grid-wide panels of <= 2048 rows by the windowed register panel, 0 = the
- * shared-memory / global-memory panels), "phase_timing" (1 = per-phase cycle
+ * shared-memory / global-memory panels), "strip" (1 = grid-wide tier fuses
+ * interchange + TRSM + trailing GEMM per 64-column strip; needs panel_win),
+ * "phase_timing" (1 = per-phase cycle
  * counters in the workspace).  Unknown keys are ignored;
  * irr_get_tuning returns the current value (-1 for an unknown key).
  * ---------------------------------------------------------------------- */

@@ -27,7 +27,7 @@ size_t laswp_smem(int span);
 // defaults chosen by measurement on B200: tier M only up to
 // 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1};
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -67,7 +67,7 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 }
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
-                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1"};
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip"};
 
 struct DeviceInfo {
     int sms = 0;
@@ -138,12 +138,20 @@ struct Work {
     int *bins;
     int *tile_off;
     int *sort;  // size sort (sched.cuh): sorted slots + bucket prefix
+    void *plans;  // getrf / partial only: one interchange plan per tier-L slot
 };
 
 static size_t work_bytes_for(int batch) {
     size_t b = (size_t)(batch > 0 ? batch : 1);
     return align256(CNT_INTS * sizeof(int)) + align256(NBINS * b * sizeof(int)) + align256((b + 1) * sizeof(int)) +
            align256(size_sort_ints((int)b) * sizeof(int));
+}
+
+// getrf / partial: the common part plus the per-slot interchange plans of the
+// grid-wide tier (written by its panel kernel, read by its strip kernel)
+static size_t work_bytes_getrf(int batch) {
+    size_t b = (size_t)(batch > 0 ? batch : 1);
+    return work_bytes_for(batch) + align256(b * SWAP_PLAN_BYTES);
 }
 
 static Work carve(void *work, int batch) {
@@ -157,6 +165,8 @@ static Work carve(void *work, int batch) {
     w.tile_off = (int *)p;
     p += align256((b + 1) * sizeof(int));
     w.sort = (int *)p;
+    p += align256(size_sort_ints((int)b) * sizeof(int));
+    w.plans = p;  // valid only in a work_bytes_getrf() workspace
     return w;
 }
 
@@ -206,7 +216,7 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
         }
         if (has_large) {
             if (t.l1) launch_lu_l1(a, w.counters, w.bins, s);
-            if (!t.l1 || a.max_m > L1_MAX_ROWS) launch_lu_large(a, w.counters, w.bins, w.tile_off, s);
+            if (!t.l1 || a.max_m > L1_MAX_ROWS) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, s);
         }
     }
     if (side != s) {
@@ -280,6 +290,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "dmma")) g_tuning.dmma = value ? 1 : 0;
     else if (!strcmp(key, "l1_dmma")) g_tuning.l1_dmma = value ? 1 : 0;
     else if (!strcmp(key, "panel_win")) g_tuning.panel_win = value ? 1 : 0;
+    else if (!strcmp(key, "strip")) g_tuning.strip = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -296,6 +307,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "dmma")) return g_tuning.dmma;
     if (!strcmp(key, "l1_dmma")) return g_tuning.l1_dmma;
     if (!strcmp(key, "panel_win")) return g_tuning.panel_win;
+    if (!strcmp(key, "strip")) return g_tuning.strip;
     return -1;
 }
 
@@ -303,7 +315,7 @@ void irr_reset_tuning(void) { g_tuning = g_default; }
 
 size_t irr_getrf_workspace_size(int batch, int max_m, int max_n) {
     (void)max_m; (void)max_n;
-    return work_bytes_for(batch);
+    return work_bytes_getrf(batch);
 }
 
 int irr_getrf(int batch, int max_m, int max_n, const int *m, const int *n, double *const *A, const int *ld,
@@ -317,7 +329,7 @@ int irr_getrf(int batch, int max_m, int max_n, const int *m, const int *n, doubl
     if (!ipiv) return -8;
     if (!info) return -9;
     if (!work) return -10;
-    if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+    if (work_bytes < work_bytes_getrf(batch)) return IRR_ERR_WORKSPACE;
     int rc = check_device();
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;
@@ -330,7 +342,7 @@ int irr_getrf(int batch, int max_m, int max_n, const int *m, const int *n, doubl
 
 size_t irr_getrf_partial_workspace_size(int batch, int max_n1, int max_n2) {
     (void)max_n1; (void)max_n2;
-    return work_bytes_for(batch);
+    return work_bytes_getrf(batch);
 }
 
 int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const int *n2, double *const *F11,
@@ -352,7 +364,7 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     if (!ipiv) return -14;
     if (!info) return -15;
     if (!work) return -16;
-    if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+    if (work_bytes < work_bytes_getrf(batch)) return IRR_ERR_WORKSPACE;
     int rc = check_device();
     if (rc) return rc;
     cudaStream_t s = (cudaStream_t)stream;

@@ -26,6 +26,7 @@ struct Tuning {
     int dmma;            // 1: grid-wide GEMMs on the FP64 tensor core (mma.sync DMMA), 0: DFMA
     int l1_dmma;         // same switch for the GEMM phase inside the L1 kernel
     int panel_win;       // 1: grid-wide panels by the windowed register panel (rows <= 2048)
+    int strip;           // 1: fused interchange + TRSM + GEMM per 64-column strip (needs panel_win)
 };
 Tuning &tuning();
 
@@ -36,7 +37,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();
@@ -73,7 +74,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
@@ -179,7 +180,8 @@ void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, c
 void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
                    cudaStream_t s);
 // lu_large.cu
-void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s);
+constexpr size_t SWAP_PLAN_BYTES = 1040;  // sizeof(SwapPlan), checked in lu_large.cu
+void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, cudaStream_t s);
 void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)

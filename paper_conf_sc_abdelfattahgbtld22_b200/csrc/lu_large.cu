@@ -123,6 +123,7 @@ __device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const 
 // solve_from also get U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory in
 // the layouts of trsm_col_regs.  top / bot: shared buffers of nb x
 // (SW_COLS+1).  SW_NT threads.
+template <int COLS = SW_COLS>
 __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int vbeg, int W,
                                            int jsplit, int shift, int solve_from, const SwapPlan &sp,
                                            const double *L11, int ldl, double *top, double *bot,
@@ -135,7 +136,7 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
         atomicAdd(ph + (k), (unsigned long long)(t1 - tq));                   \
         tq = t1;                                                              \
     }
-    constexpr int LT = SW_COLS + 1;
+    constexpr int LT = COLS + 1;
     constexpr int NWS = SW_NT / 32;
     const int nbot = sp.nbot;
     // warps over columns, lanes over the (<= 64) moved rows: no integer division
@@ -357,7 +358,8 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
 // <= 2048 in registers (RPT = 2, 4, 8 with window 16, 8, 4), 2 CTAs / SM.
 constexpr int PW_NT = 256;
 __global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const int *__restrict__ counters,
-                                                             const int *__restrict__ bins, int j, int nb) {
+                                                             const int *__restrict__ bins, int j, int nb,
+                                                             SwapPlan *__restrict__ plans, int *queue) {
     extern __shared__ __align__(16) double pw_smem[];
     PanelWinSmem<PW_NT / 32> &sm = *reinterpret_cast<PanelWinSmem<PW_NT / 32> *>(pw_smem);
     __shared__ PanelScratch sc;
@@ -365,6 +367,7 @@ __global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const 
     const int tid = threadIdx.x;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
+    if (blockIdx.x == 0 && tid == 0) *queue = 0;  // the strip kernel's work queue (stream-ordered)
     for (int t = blockIdx.x; t < count; t += gridDim.x) {
         const int i = list[t];
         const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
@@ -378,10 +381,105 @@ __global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const 
         else if (rows <= 4 * PW_NT) z = panel_win<PW_NT, 4, 8>(gP, ld, rows, ib, piv_s, sm);
         else if (rows <= 8 * PW_NT) z = panel_win<PW_NT, 8, 4>(gP, ld, rows, ib, piv_s, sm);
         else z = panel_getf2<PW_NT>(gP, ld, 0, rows, 0, ib, 0, ib, piv_s, sc);
+        if (rows <= 8 * PW_NT) {
+            // the interchange plan for the strip kernel (absolute rows)
+            SwapPlan &g = plans[t];
+            if (tid < ib) g.top_src[tid] = j + sm.plan.top_src[tid];
+            if (tid < sm.plan.nbot) {
+                g.bot_pos[tid] = j + sm.plan.bot_pos[tid];
+                g.bot_src[tid] = j + sm.plan.bot_src[tid];
+            }
+            if (tid == 0) g.nbot = sm.plan.nbot;
+        }
         if (tid < ib) a.ipiv[i][j + tid] = j + piv_s[tid] + 1;
         if (tid == 0 && z && a.info[i] == 0) a.info[i] = j + z;
         __syncthreads();
     }
+}
+
+// Fused step a4.2 + a4.3 + a4.4 of the grid-wide tier, one work item per
+// (tier-L slot, 64-column strip of the virtual range [0, n - ib)): gather the
+// moved rows of the strip (plan from the panel kernel), solve the U12 part with
+// the unit L11, scatter, then stream the trailing GEMM down the strip,
+// C(c1:m, strip) -= L21 U12(:, strip).  The interchanged rows are re-read by
+// the GEMM straight from L2, and every strip is owned by exactly one CTA, so
+// no other CTA can observe a half-swapped column.  Items come from a dynamic
+// queue (reset by the panel kernel).
+constexpr int ST_COLS = GBN;
+static_assert(sizeof(SwapPlan) <= SWAP_PLAN_BYTES, "plan slot");
+template <bool DMMA>
+__global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                        const int *__restrict__ bins,
+                                                        const SwapPlan *__restrict__ plans, int *queue, int j,
+                                                        int nb, int chunks_per) {
+    extern __shared__ __align__(16) double st_smem[];
+    GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
+    const int ldl = nb + 1;
+    double *L11 = st_smem;
+    double *top = L11 + nb * ldl;
+    double *bot = top + nb * (ST_COLS + 1);
+    __shared__ SwapPlan sp;
+    __shared__ int item_s;
+    const int tid = threadIdx.x;
+    const int count = counters[CNT_BIN0 + BIN_L];
+    const int *list = bins + (size_t)BIN_L * a.batch;
+    const long long total = (long long)count * chunks_per;
+    int last_slot = -1;
+    for (;;) {
+        if (tid == 0) item_s = atomicAdd(queue, 1);
+        __syncthreads();
+        const long long w = item_s;
+        if (w >= total) break;
+        const int slot = (int)(w / chunks_per), q = (int)(w - (long long)slot * chunks_per);
+        const int i = list[slot];
+        const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
+        const int K = mi < ni ? mi : ni;
+        if (j >= K) continue;
+        const int ib = K - j < nb ? K - j : nb;
+        const int c1 = j + ib;
+        const int vtot = ni - ib, vb = q * ST_COLS;
+        if (vb >= vtot) continue;
+        double *gA = a.A[i];
+        if (slot != last_slot) {
+            const int *src = reinterpret_cast<const int *>(plans + slot);
+            int *dst = reinterpret_cast<int *>(&sp);
+            for (int e = tid; e < (int)(sizeof(SwapPlan) / sizeof(int)); e += G_NT) dst[e] = src[e];
+            last_slot = slot;
+        }
+        load_L11_async(L11, ldl, gA, ld, j, ib);
+        cp_async_commit();
+        __syncthreads();
+        const int W = imin(ST_COLS, vtot - vb);
+        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, j, ib, c1, sp, L11, ldl, top, bot);
+        // trailing GEMM on the strip's right-of-panel columns
+        const int cbeg = (vb > j ? vb : j) + ib, cend = vb + W + ib;
+        if (cbeg < cend && c1 < mi) {
+            GemmDesc d0;
+            d0.A = gA + c1 + (size_t)j * ld; d0.lda = ld; d0.ta = 0;
+            d0.B = gA + j + (size_t)cbeg * ld; d0.ldb = ld; d0.tb = 0;
+            d0.C = gA + c1 + (size_t)cbeg * ld; d0.ldc = ld;
+            d0.m = mi - c1; d0.n = cend - cbeg; d0.k = ib;
+            d0.alpha = -1.0; d0.beta = 1.0;
+            const int ntm = (d0.m + GBM - 1) / GBM;
+            int tt = 0;
+            auto next = [&](GemmDesc &d, int &r0, int &cc0) -> bool {
+                if (tt >= ntm) return false;
+                d = d0;
+                r0 = tt * GBM;
+                cc0 = 0;
+                ++tt;
+                return true;
+            };
+            gemm_tile_stream<DMMA>(next, gsm);
+            __syncthreads();
+        }
+    }
+}
+
+static size_t strip_smem_bytes(int nb) {
+    size_t sw = (size_t)(nb * (nb + 1) + 2 * nb * (ST_COLS + 1)) * sizeof(double);
+    size_t m = sw > GEMM_SMEM ? sw : GEMM_SMEM;
+    return (m + 15) & ~size_t(15);
 }
 
 // Work item = (tier-L slot, column chunk) over the virtual column range
@@ -471,7 +569,9 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
                                                       tuning().phase_timing);
 }
 
-void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, cudaStream_t s) {
+void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans_v,
+                     cudaStream_t s) {
+    SwapPlan *plans = reinterpret_cast<SwapPlan *>(plans_v);
     const Tuning &tu = tuning();
     const int nb = clamp_nb(tu.nb);
     const int Kmax = a.max_m < a.max_n ? a.max_m : a.max_n;
@@ -508,13 +608,32 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         sw_attr = sw_smem;
     }
     const int *listL = bins + (size_t)BIN_L * a.batch;
+    const bool fused = tu.panel_win && tu.strip && a.max_m <= 8 * PW_NT;
+    const int st_chunks = (a.max_n + ST_COLS - 1) / ST_COLS;
+    const size_t st_smem = strip_smem_bytes(nb);
+    if (fused) {
+        static size_t st_attr[2] = {0, 0};
+        if (st_smem > st_attr[tu.dmma ? 1 : 0]) {
+            if (tu.dmma) cudaFuncSetAttribute(strip_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)st_smem);
+            else cudaFuncSetAttribute(strip_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)st_smem);
+            st_attr[tu.dmma ? 1 : 0] = st_smem;
+        }
+    }
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {
             KScope k(K_PANEL, s);
-            panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb);
+            panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb, plans, counters + CNT_STRIPQ);
         } else {
             KScope k(K_PANEL, s);
             panel_kernel<<<grid_p, P_NT, psmem, s>>>(a, counters, bins, j, nb, smem_rows);
+        }
+        if (fused) {
+            KScope k(K_STRIP, s);
+            if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
+                                                                             counters + CNT_STRIPQ, j, nb, st_chunks);
+            else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
+                                                                      counters + CNT_STRIPQ, j, nb, st_chunks);
+            continue;
         }
         {
             KScope k(K_SWAP_TRSM, s);
