@@ -215,7 +215,13 @@ __device__ __forceinline__ int gemm_tiles_of(const GemmDesc &d) {
     return ((d.m + GBM - 1) / GBM) * ((d.n + GBN - 1) / GBN);
 }
 
+// Schedule weight of one tile: its K chunks in units of 128 plus one for the C
+// tile (tiles of a batch differ in K by 100x in a multifrontal batch; equal
+// tile counts per CTA left the CTAs holding the big fronts 1.75x over).
+__device__ __forceinline__ int gemm_tile_weight(const GemmDesc &d) { return 1 + (d.k > 0 ? (d.k + 127) / 128 : 0); }
+
 // count: number of problem slots, from *count_ptr when count < 0.
+// tile_off[b] = weighted work before slot b (gemm_tile_weight units).
 template <class Prob>
 __global__ void __launch_bounds__(1024) gemm_scan_kernel(Prob P, int count, const int *count_ptr, int *tile_off) {
     __shared__ int warp_sums[32];
@@ -229,7 +235,7 @@ __global__ void __launch_bounds__(1024) gemm_scan_kernel(Prob P, int count, cons
         int v = 0;
         if (b < count) {
             GemmDesc d;
-            if (P.get(b, d)) v = gemm_tiles_of(d);
+            if (P.get(b, d)) v = gemm_tiles_of(d) * gemm_tile_weight(d);
         }
         int x = v;
 #pragma unroll
@@ -268,33 +274,37 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, 
     if (count <= 0) return;
     const int total = tile_off[count];
     const long long G = gridDim.x;
-    const int t_begin = (int)((long long)blockIdx.x * total / G);
-    const int t_end = (int)((long long)(blockIdx.x + 1) * total / G);
-    if (t_begin >= t_end) return;
-    // last slot b with tile_off[b] <= t_begin (the one whose range holds t_begin)
-    int lo = 0, hi = count - 1;
+    // this CTA owns the tiles whose weighted start lies in [u_begin, u_end)
+    const int u_begin = (int)((long long)blockIdx.x * total / G);
+    const int u_end = (int)((long long)(blockIdx.x + 1) * total / G);
+    if (u_begin >= u_end) return;
+    int lo = 0, hi = count - 1;  // last slot b with tile_off[b] <= u_begin
     while (lo < hi) {
         int mid = (lo + hi + 1) >> 1;
-        if (tile_off[mid] <= t_begin) lo = mid; else hi = mid - 1;
+        if (tile_off[mid] <= u_begin) lo = mid; else hi = mid - 1;
     }
-    int b = lo, t = t_begin;
+    int b = lo;
     GemmDesc cur;
     P.get(b, cur);
-    int b_beg = tile_off[b], b_end = tile_off[b + 1];
+    int w = gemm_tile_weight(cur), off_b = tile_off[b];
+    int nt_b = (tile_off[b + 1] - off_b) / w;
+    int local = u_begin > off_b ? (u_begin - off_b + w - 1) / w : 0;
     auto next = [&](GemmDesc &d, int &r0, int &c0) -> bool {
-        if (t >= t_end) return false;
-        while (t >= b_end) {
-            ++b;
+        while (local >= nt_b) {
+            if (++b >= count) return false;
+            off_b = tile_off[b];
+            if (off_b >= u_end) return false;
             P.get(b, cur);
-            b_beg = tile_off[b];
-            b_end = tile_off[b + 1];
+            w = gemm_tile_weight(cur);
+            nt_b = (tile_off[b + 1] - off_b) / w;
+            local = 0;
         }
-        const int local = t - b_beg;
+        if (off_b + local * w >= u_end) return false;
         const int ntm = (cur.m + GBM - 1) / GBM;
         r0 = (local % ntm) * GBM;
         c0 = (local / ntm) * GBN;
         d = cur;
-        ++t;
+        ++local;
         return true;
     };
     gemm_tile_stream<DMMA>(next, sm);

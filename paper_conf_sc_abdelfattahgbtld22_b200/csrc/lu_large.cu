@@ -411,7 +411,7 @@ template <bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                         const int *__restrict__ bins,
                                                         const SwapPlan *__restrict__ plans, int *queue, int j,
-                                                        int nb, int chunks_per) {
+                                                        int nb, int chunks_per, unsigned long long *ph) {
     extern __shared__ __align__(16) double st_smem[];
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
@@ -425,7 +425,15 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
     const int *list = bins + (size_t)BIN_L * a.batch;
     const long long total = (long long)count * chunks_per;
     int last_slot = -1;
+    long long t0 = (ph && tid == 0) ? clock64() : 0;
+#define ST_PHASE(k)                                                           \
+    if (ph && tid == 0) {                                                     \
+        long long t1 = clock64();                                             \
+        atomicAdd(ph + (k), (unsigned long long)(t1 - t0));                   \
+        t0 = t1;                                                              \
+    }
     for (;;) {
+        ST_PHASE(3)  // the tail of empty items
         if (tid == 0) item_s = atomicAdd(queue, 1);
         __syncthreads();
         const long long w = item_s;
@@ -449,8 +457,10 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         load_L11_async(L11, ldl, gA, ld, j, ib);
         cp_async_commit();
         __syncthreads();
+        ST_PHASE(0)
         const int W = imin(ST_COLS, vtot - vb);
-        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, j, ib, c1, sp, L11, ldl, top, bot);
+        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, j, ib, c1, sp, L11, ldl, top, bot, ph);
+        if (ph && tid == 0) t0 = clock64();
         // trailing GEMM on the strip's right-of-panel columns
         const int cbeg = (vb > j ? vb : j) + ib, cend = vb + W + ib;
         if (cbeg < cend && c1 < mi) {
@@ -472,8 +482,10 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
             };
             gemm_tile_stream<DMMA>(next, gsm);
             __syncthreads();
+            ST_PHASE(2)
         }
     }
+#undef ST_PHASE
 }
 
 static size_t strip_smem_bytes(int nb) {
@@ -609,6 +621,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     }
     const int *listL = bins + (size_t)BIN_L * a.batch;
     const bool fused = tu.panel_win && tu.strip && a.max_m <= 8 * PW_NT;
+    unsigned long long *ph = tu.phase_timing ? reinterpret_cast<unsigned long long *>(counters + CNT_PHASE0) : nullptr;
     const int st_chunks = (a.max_n + ST_COLS - 1) / ST_COLS;
     const size_t st_smem = strip_smem_bytes(nb);
     if (fused) {
@@ -630,9 +643,9 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         if (fused) {
             KScope k(K_STRIP, s);
             if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
-                                                                             counters + CNT_STRIPQ, j, nb, st_chunks);
+                                                                             counters + CNT_STRIPQ, j, nb, st_chunks, ph);
             else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
-                                                                      counters + CNT_STRIPQ, j, nb, st_chunks);
+                                                                      counters + CNT_STRIPQ, j, nb, st_chunks, ph);
             continue;
         }
         {
