@@ -27,7 +27,7 @@ size_t laswp_smem(int span);
 // defaults chosen by measurement on B200: tier M only up to
 // 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1};
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -291,6 +291,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1_dmma")) g_tuning.l1_dmma = value ? 1 : 0;
     else if (!strcmp(key, "panel_win")) g_tuning.panel_win = value ? 1 : 0;
     else if (!strcmp(key, "strip")) g_tuning.strip = value ? 1 : 0;
+    else if (!strcmp(key, "gemm_big")) g_tuning.gemm_big = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -308,6 +309,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "l1_dmma")) return g_tuning.l1_dmma;
     if (!strcmp(key, "panel_win")) return g_tuning.panel_win;
     if (!strcmp(key, "strip")) return g_tuning.strip;
+    if (!strcmp(key, "gemm_big")) return g_tuning.gemm_big;
     return -1;
 }
 

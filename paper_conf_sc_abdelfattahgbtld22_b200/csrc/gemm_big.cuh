@@ -1,0 +1,284 @@
+// gemm_big.cuh -- the large-tile FP64 tensor-core GEMM core of irrGEMM
+// (§IV-C; SURVEY §8(a) a5.3 and the TRSM recursion of a5.2).
+//
+// The partial front factorization spends 58% of its flops in F22 -= F21 F12
+// with K = n1 up to ~2000 and another 35% in the off-diagonal GEMMs of the
+// recursive TRSM ("runtime most impacted by the GEMM performance on
+// the largest nodes").  For those long-K products the 64 x 64 core
+// (gemm_core.cuh) is bound by its operand traffic; this core is sized for
+// the DMMA pipe instead:
+//   * 128 x 128 CTA tile, 256 threads = 8 warps in a 2 x 4 grid, each warp a
+//     64 x 32 tile of 8 x 4 mma.sync.m8n8k4.f64 (SASS DMMA.884) accumulators
+//     (64 doubles per lane), so one k-step is 12 fragment loads per 32 DMMA;
+//   * K chunks of 16 staged by cp.async in a 4-deep ring (one barrier per
+//     chunk), shared layouts chosen per transpose so every fragment load is
+//     bank-conflict free: k-major [k][m] with ld 132 when the operand is
+//     contiguous along m (n), m-major [m][k] with ld 20 when contiguous along k;
+//   * 1 CTA per SM (8 warps saturate DMMA: profiles/r01/microbench.txt),
+//     persistent over a device tile schedule weighted by K.
+// Epilogue reads / writes C straight from registers (each warp store covers
+// 64-byte column segments).
+#pragma once
+#include "gemm_core.cuh"
+
+namespace irr {
+
+constexpr int XBM = 128, XBN = 128, XBK = 16, X_NT = 256, XST = 4;
+constexpr int XLD_KM = 132;  // [k][m] layout: XBK rows of XBM (+4)
+constexpr int XLD_MK = 20;   // [m][k] layout: XBM rows of XBK (+4)
+constexpr int XSTAGE = 2560; // doubles per operand stage: max(16 * 132, 128 * 20)
+
+struct BigSmem {
+    double A[XST][XSTAGE];
+    double B[XST][XSTAGE];
+};
+constexpr size_t BIG_SMEM = sizeof(BigSmem);
+
+// cp.async with zero fill: src_bytes = 0 writes zeros and reads nothing
+__device__ __forceinline__ void cp_async8_zf(void *smem, const void *gmem, bool valid) {
+    unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    const int n = valid ? 8 : 0;
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+}
+
+// Stage chunk [k0, k0+16) of the (r0, c0) tile.  op(A) is m x k, op(B) k x n.
+template <int TA, int TB>
+__device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st) {
+    const int tid = threadIdx.x;
+    double *As = sm.A[st];
+    double *Bs = sm.B[st];
+#pragma unroll
+    for (int q = 0; q < (XBM * XBK) / X_NT; ++q) {
+        const int e = tid + X_NT * q;
+        int m, kk;
+        if (!TA) { m = e & (XBM - 1); kk = e >> 7; } else { kk = e & (XBK - 1); m = e >> 4; }
+        const int gm = r0 + m, gk = k0 + kk;
+        const bool ok = gm < d.m && gk < d.k;
+        const double *src = ok ? (TA ? d.A + gk + (size_t)gm * d.lda : d.A + gm + (size_t)gk * d.lda) : d.A;
+        cp_async8_zf(TA ? &As[m * XLD_MK + kk] : &As[kk * XLD_KM + m], src, ok);
+    }
+#pragma unroll
+    for (int q = 0; q < (XBN * XBK) / X_NT; ++q) {
+        const int e = tid + X_NT * q;
+        int n, kk;
+        if (!TB) { kk = e & (XBK - 1); n = e >> 4; } else { n = e & (XBN - 1); kk = e >> 7; }
+        const int gn = c0 + n, gk = k0 + kk;
+        const bool ok = gn < d.n && gk < d.k;
+        const double *src = ok ? (TB ? d.B + gn + (size_t)gk * d.ldb : d.B + gk + (size_t)gn * d.ldb) : d.B;
+        cp_async8_zf(TB ? &Bs[kk * XLD_KM + n] : &Bs[n * XLD_MK + kk], src, ok);
+    }
+}
+
+template <int TA, int TB>
+__device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double (&acc)[64]) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+    const int wm = (warp & 1) * 64, wn = (warp >> 1) * 32;
+    const double *As = sm.A[st];
+    const double *Bs = sm.B[st];
+#pragma unroll
+    for (int ks = 0; ks < XBK; ks += 4) {
+        double a[8], b[4];
+#pragma unroll
+        for (int mi = 0; mi < 8; ++mi) {
+            const int m = wm + 8 * mi + g, k = ks + t;
+            a[mi] = TA ? As[m * XLD_MK + k] : As[k * XLD_KM + m];
+        }
+#pragma unroll
+        for (int ni = 0; ni < 4; ++ni) {
+            const int n = wn + 8 * ni + g, k = ks + t;
+            b[ni] = TB ? Bs[k * XLD_KM + n] : Bs[n * XLD_MK + k];
+        }
+#pragma unroll
+        for (int mi = 0; mi < 8; ++mi)
+#pragma unroll
+            for (int ni = 0; ni < 4; ++ni)
+                dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], a[mi], b[ni]);
+    }
+}
+
+__device__ __forceinline__ void xgemm_epilogue(const GemmDesc &d, int r0, int c0, const double (&acc)[64]) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+    const int wm = (warp & 1) * 64, wn = (warp >> 1) * 32;
+    const bool rd = d.beta != 0.0;
+#pragma unroll
+    for (int mi = 0; mi < 8; ++mi) {
+        const int r = r0 + wm + 8 * mi + g;
+        if (r >= d.m) continue;
+        double cv[8];
+        if (rd) {
+#pragma unroll
+            for (int ni = 0; ni < 4; ++ni)
+#pragma unroll
+                for (int i = 0; i < 2; ++i) {
+                    const int c = c0 + wn + 8 * ni + 2 * t + i;
+                    cv[ni * 2 + i] = c < d.n ? d.C[r + (size_t)c * d.ldc] : 0.0;
+                }
+        }
+#pragma unroll
+        for (int ni = 0; ni < 4; ++ni)
+#pragma unroll
+            for (int i = 0; i < 2; ++i) {
+                const int c = c0 + wn + 8 * ni + 2 * t + i;
+                if (c >= d.n) continue;
+                double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
+                if (rd) v = fma(d.beta, cv[ni * 2 + i], v);
+                d.C[r + (size_t)c * d.ldc] = v;
+            }
+    }
+}
+
+// One tile: the whole K loop through the 4-deep ring, then the epilogue.
+template <int TA, int TB>
+__device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, BigSmem &sm) {
+    double acc[64];
+#pragma unroll
+    for (int q = 0; q < 64; ++q) acc[q] = 0.0;
+    const int nk = (d.k + XBK - 1) / XBK;
+#pragma unroll
+    for (int s = 0; s < XST - 1; ++s) {
+        if (s < nk) xgemm_issue<TA, TB>(d, r0, c0, s * XBK, sm, s);
+        cp_async_commit();
+    }
+    for (int kc = 0; kc < nk; ++kc) {
+        cp_async_wait<XST - 2>();
+        __syncthreads();
+        const int nx = kc + XST - 1;
+        if (nx < nk) xgemm_issue<TA, TB>(d, r0, c0, nx * XBK, sm, nx % XST);
+        cp_async_commit();
+        xgemm_compute<TA, TB>(sm, kc % XST, acc);
+    }
+    cp_async_wait<0>();
+    __syncthreads();  // the ring is refilled by the next tile's prologue
+    xgemm_epilogue(d, r0, c0, acc);
+}
+
+__device__ __forceinline__ int xgemm_tiles_of(const GemmDesc &d) {
+    if (d.m <= 0 || d.n <= 0) return 0;
+    return ((d.m + XBM - 1) / XBM) * ((d.n + XBN - 1) / XBN);
+}
+// work of one tile in units of 64 K (+1 for the epilogue)
+__device__ __forceinline__ int xgemm_tile_weight(const GemmDesc &d) { return 1 + (d.k > 0 ? (d.k + 63) / 64 : 0); }
+
+// tile_off[b] = weighted tiles before slot b (one CTA)
+template <class Prob>
+__global__ void __launch_bounds__(1024) xgemm_scan_kernel(Prob P, int count, const int *count_ptr, int *tile_off) {
+    __shared__ int warp_sums[32];
+    __shared__ int carry_s;
+    if (count < 0) count = *count_ptr;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) carry_s = 0;
+    __syncthreads();
+    for (int base = 0; base < count; base += 1024) {
+        const int b = base + tid;
+        int v = 0;
+        if (b < count) {
+            GemmDesc d;
+            if (P.get(b, d)) v = xgemm_tiles_of(d) * xgemm_tile_weight(d);
+        }
+        int x = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            int y = __shfl_up_sync(FULL, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) warp_sums[warp] = x;
+        __syncthreads();
+        if (warp == 0) {
+            int w = warp_sums[lane];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                int y = __shfl_up_sync(FULL, w, o);
+                if (lane >= o) w += y;
+            }
+            warp_sums[lane] = w;
+        }
+        __syncthreads();
+        const int excl = carry_s + (warp ? warp_sums[warp - 1] : 0) + x - v;
+        if (b < count) tile_off[b] = excl;
+        __syncthreads();
+        if (tid == 1023) carry_s = excl + v;
+        __syncthreads();
+    }
+    if (tid == 0) tile_off[count] = carry_s;
+}
+
+// Persistent: CTA b owns the tiles whose weighted start lies in its 1/G share.
+template <class Prob, int TA, int TB>
+__global__ void __launch_bounds__(X_NT, 1) xgemm_sched_kernel(Prob P, int count, const int *count_ptr,
+                                                             const int *__restrict__ tile_off) {
+    extern __shared__ __align__(16) unsigned char x_smem[];
+    BigSmem &sm = *reinterpret_cast<BigSmem *>(x_smem);
+    if (count < 0) count = *count_ptr;
+    if (count <= 0) return;
+    const int total = tile_off[count];
+    const long long G = gridDim.x;
+    const int u_begin = (int)((long long)blockIdx.x * total / G);
+    const int u_end = (int)((long long)(blockIdx.x + 1) * total / G);
+    if (u_begin >= u_end) return;
+    int lo = 0, hi = count - 1;
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (tile_off[mid] <= u_begin) lo = mid; else hi = mid - 1;
+    }
+    int b = lo;
+    GemmDesc cur;
+    P.get(b, cur);
+    int w = xgemm_tile_weight(cur), off_b = tile_off[b];
+    int nt_b = (tile_off[b + 1] - off_b) / w;
+    int local = u_begin > off_b ? (u_begin - off_b + w - 1) / w : 0;
+    while (true) {
+        while (local >= nt_b) {
+            if (++b >= count) return;
+            off_b = tile_off[b];
+            if (off_b >= u_end) return;
+            P.get(b, cur);
+            w = xgemm_tile_weight(cur);
+            nt_b = (tile_off[b + 1] - off_b) / w;
+            local = 0;
+        }
+        if (off_b + local * w >= u_end) return;
+        const int ntm = (cur.m + XBM - 1) / XBM;
+        xgemm_tile<TA, TB>(cur, (local % ntm) * XBM, (local / ntm) * XBN, sm);
+        ++local;
+    }
+}
+
+// Wraps a problem and keeps only the slots one of the two cores should run:
+// the big core takes products whose tile would be mostly full and whose K
+// amortises the pipeline fill.
+template <class Prob>
+struct SizeFilter {
+    Prob p;
+    int want_big;
+    __device__ static bool is_big(const GemmDesc &d) { return d.m >= 96 && d.n >= 96 && d.k >= 48; }
+    __device__ bool get(int slot, GemmDesc &d) const {
+        if (!p.get(slot, d)) return false;
+        if (want_big >= 0 && is_big(d) != (want_big != 0)) { d.m = 0; d.n = 0; d.k = 0; return false; }
+        return true;
+    }
+};
+
+template <class Prob, int TA, int TB>
+inline void xgemm_launch_t(const Prob &P, int cnt, const int *cnt_ptr, const int *tile_off, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(xgemm_sched_kernel<Prob, TA, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)BIG_SMEM);
+        attr = true;
+    }
+    xgemm_sched_kernel<Prob, TA, TB><<<num_sms(), X_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+}
+
+// one persistent CTA per SM; the transposes select the shared layouts
+template <class Prob>
+inline void launch_xgemm(const Prob &P, int ta, int tb, int cnt, const int *cnt_ptr, const int *tile_off,
+                         cudaStream_t s) {
+    if (!ta && !tb) xgemm_launch_t<Prob, 0, 0>(P, cnt, cnt_ptr, tile_off, s);
+    else if (!ta && tb) xgemm_launch_t<Prob, 0, 1>(P, cnt, cnt_ptr, tile_off, s);
+    else if (ta && !tb) xgemm_launch_t<Prob, 1, 0>(P, cnt, cnt_ptr, tile_off, s);
+    else xgemm_launch_t<Prob, 1, 1>(P, cnt, cnt_ptr, tile_off, s);
+}
+
+}  // namespace irr

@@ -2,7 +2,7 @@
 // DCWI (§IV-B): C_i <- alpha op(A_i) op(B_i) + beta C_i on
 // submatrices selected by scalar offsets, with per-matrix effective sizes
 // inferred on the device.
-#include "gemm_core.cuh"
+#include "gemm_big.cuh"
 #include "sched.cuh"
 
 namespace irr {
@@ -49,17 +49,33 @@ void launch_gemm_masked(const GemmArgs &g, const int *mask, int *counters, int *
         DcwiGemmProb P{g, mask, sl};
         const int cnt = sl.prefix ? -1 : g.batch;
         const int *cnt_ptr = sl.prefix ? sl.prefix + sl.bucket0 : nullptr;
+        // long-K products on the 128 x 128 DMMA core first, the rest on the
+        // 64 x 64 core; both passes reuse tile_off (stream-ordered)
+        const bool big = tuning().gemm_big && g.max_m >= 96 && g.max_n >= 96 && g.max_k >= 48;
+        if (big) {
+            using BP = SizeFilter<DcwiGemmProb>;
+            BP Pb{P, 1};
+            {
+                KScope k(K_GEMM_SCAN, s);
+                xgemm_scan_kernel<BP><<<1, 1024, 0, s>>>(Pb, cnt, cnt_ptr, tile_off);
+            }
+            KScope k(K_GEMM_DCWI, s);
+            launch_xgemm(Pb, g.ta, g.tb, cnt, cnt_ptr, tile_off, s);
+        }
+        using SP = SizeFilter<DcwiGemmProb>;
+        SP Ps{P, 0};
+        if (!big) Ps.want_big = -1;  // no filtering
         {
             KScope k(K_GEMM_SCAN, s);
-            gemm_scan_kernel<DcwiGemmProb><<<1, 1024, 0, s>>>(P, cnt, cnt_ptr, tile_off);
+            gemm_scan_kernel<SP><<<1, 1024, 0, s>>>(Ps, cnt, cnt_ptr, tile_off);
         }
         KScope k(K_GEMM_DCWI, s);
         if (tuning().dmma) {
-            gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb, true>);
-            gemm_sched_kernel<DcwiGemmProb, true><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+            gemm_smem_optin(gemm_sched_kernel<SP, true>);
+            gemm_sched_kernel<SP, true><<<sms * 3, G_NT, GEMM_SMEM, s>>>(Ps, cnt, cnt_ptr, tile_off);
         } else {
-            gemm_smem_optin(gemm_sched_kernel<DcwiGemmProb, false>);
-            gemm_sched_kernel<DcwiGemmProb, false><<<sms * 3, G_NT, GEMM_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+            gemm_smem_optin(gemm_sched_kernel<SP, false>);
+            gemm_sched_kernel<SP, false><<<sms * 3, G_NT, GEMM_SMEM, s>>>(Ps, cnt, cnt_ptr, tile_off);
         }
     } else {
         DcwiGemmProb P{g, mask, all_slots()};

@@ -27,6 +27,7 @@ struct Tuning {
     int l1_dmma;         // same switch for the GEMM phase inside the L1 kernel
     int panel_win;       // 1: grid-wide panels by the windowed register panel (rows <= 2048)
     int strip;           // 1: fused interchange + TRSM + GEMM per 64-column strip (needs panel_win)
+    int gemm_big;        // 1: long-K DCWI GEMMs on the 128x128 DMMA core (gemm_big.cuh)
 };
 Tuning &tuning();
 

@@ -68,6 +68,29 @@ def test_gemm_dcwi_exact(ta, tb, use_work):
         assert np.array_equal(got[i], exp), i
 
 
+@pytest.mark.parametrize("ta,tb", list(itertools.product((0, 1), (0, 1))))
+def test_gemm_big_core_exact(ta, tb):
+    """Products large enough for the 128 x 128 DMMA core (several tiles, ragged
+    edges, K not a multiple of the 16-chunk) mixed with small ones that stay
+    on the 64 x 64 core; integer data, so every entry is exact."""
+    rng = np.random.default_rng(100 + ta * 2 + tb)
+    m = np.array([300, 97, 5, 260, 130, 64]); n = np.array([257, 140, 200, 96, 7, 64])
+    k = np.array([201, 48, 300, 77, 130, 40])
+    batch = len(m)
+    As = [rng.integers(-4, 5, size=(k[i], m[i]) if ta else (m[i], k[i])).astype(float) for i in range(batch)]
+    Bs = [rng.integers(-4, 5, size=(n[i], k[i]) if tb else (k[i], n[i])).astype(float) for i in range(batch)]
+    Cs = [rng.integers(-4, 5, size=(m[i], n[i])).astype(float) for i in range(batch)]
+    dA, dB, dC = _upload(As), _upload(Bs), _upload(Cs)
+    work = torch.empty(irr.irr_gemm_workspace_size(batch), dtype=torch.uint8, device="cuda")
+    irr.irr_gemm(ta, tb, int(m.max()), int(n.max()), int(k.max()), _i32(m), _i32(n), _i32(k), -1.0, dA.ptr, 0, 0,
+                 dA.ld, dB.ptr, 0, 0, dB.ld, 0.5, dC.ptr, 0, 0, dC.ld, batch, work=work)
+    torch.cuda.synchronize()
+    got = _download(dC)
+    for i in range(batch):
+        exp = oracle.gemm(ta, tb, -1.0, As[i], Bs[i], 0.5, Cs[i])
+        assert np.array_equal(got[i], exp), i
+
+
 @pytest.mark.parametrize("side,uplo,trans,diag", list(itertools.product((0, 1), repeat=4)))
 def test_trsm_all_combinations_exact(side, uplo, trans, diag):
     """B = op(T) X0 (left) or X0 op(T) (right), dyadic T, integer X0: the

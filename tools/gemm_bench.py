@@ -20,7 +20,13 @@ ap.add_argument("--n", type=int, default=2048)
 ap.add_argument("--k", type=int, default=1024)
 ap.add_argument("--batch", type=int, default=16)
 ap.add_argument("--reps", type=int, default=5)
+ap.add_argument("--tune", action="append", default=[])
+ap.add_argument("--ta", type=int, default=0)
+ap.add_argument("--tb", type=int, default=0)
 a = ap.parse_args()
+for kv in a.tune:
+    kk, vv = kv.split("=")
+    irr.irr_set_tuning(kk, int(vv))
 b = a.batch
 A = MatrixBatch([a.m] * b, [a.k] * b, with_ipiv=False)
 B = MatrixBatch([a.k] * b, [a.n] * b, with_ipiv=False)

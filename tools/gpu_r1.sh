@@ -1,0 +1,7 @@
+set -x
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv
+python -c "import __graft_entry__ as g; g.smoke(); print('SMOKE OK')" > gpurun_out/smoke.log 2>&1
+timeout 900 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; echo pytest rc $?
+for c in C2 C3 C4 C1big; do timeout 600 python bench.py --config $c --no-cpu-baseline --no-e2e --profile-out gpurun_out/prof_$c.json > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; done
+timeout 600 python bench.py > gpurun_out/bench_default.json 2> gpurun_out/bench_default.err
+tail -3 gpurun_out/pytest_gpu.log
