@@ -156,6 +156,8 @@ def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=True):
     out = class_work(n1, n1, nb, tier_m_max, l1)
     out["gemm_dcwi"] = (float((2.0 * n1 * n2 * n2).sum()), float((8.0 * (2 * n2 * n2 + n2 * n1 + n1 * n2)).sum()))
     out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((32.0 * n1 * n2).sum()))
+    # fused a5.2 (getrs_strip.cu): 2 n1^2 n2 flops; F12 read + written, F11 read once per strip
+    out["getrs"] = (float((2.0 * n1 * n1 * n2).sum()), float((16.0 * n1 * n2 + 8.0 * n1 * n1).sum()))
     return out
 
 

@@ -23,11 +23,15 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s,
                          int *units_off, SlotList sl);
 size_t laswp_smem(int span);
+bool getrs_strip_ok(int max_n1);
+void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *const *F11, const int *ld11,
+                        double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
+                        int *queue, SlotList sl, cudaStream_t s);
 
 // defaults chosen by measurement on B200: tier M only up to
 // 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1};
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1, 0, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -67,7 +71,7 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 }
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
-                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip"};
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs"};
 
 struct DeviceInfo {
     int sms = 0;
@@ -292,6 +296,8 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "panel_win")) g_tuning.panel_win = value ? 1 : 0;
     else if (!strcmp(key, "strip")) g_tuning.strip = value ? 1 : 0;
     else if (!strcmp(key, "gemm_big")) g_tuning.gemm_big = value ? 1 : 0;
+    else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
+    else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -310,6 +316,8 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "panel_win")) return g_tuning.panel_win;
     if (!strcmp(key, "strip")) return g_tuning.strip;
     if (!strcmp(key, "gemm_big")) return g_tuning.gemm_big;
+    if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
+    if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
     return -1;
 }
 
@@ -383,7 +391,12 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     // fronts sorted by n1 (descending buckets): every building-block call
     // below visits only the fronts that still have work at its offset
     launch_size_sort(n1, batch, w.sort, s);
-    // step 2: F12 <- U^-1 L^-1 P^T F12: irrLASWP + 2 x irrTRSM (GETRS)
+    // step 2: F12 <- U^-1 L^-1 P^T F12: one fused strip kernel, or
+    // irrLASWP + 2 x irrTRSM (GETRS) as the paper composes it
+    if (tuning().getrs_fused && getrs_strip_ok(max_n1)) {
+        launch_getrs_strip(batch, n1, n2, (const double *const *)F11, ld11, F12, ld12, ipiv, info, w.tile_off,
+                           w.counters + CNT_GSQ, sorted_slots(w.sort, batch, 0), s);
+    } else {
     launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s, w.tile_off,
                         sorted_slots(w.sort, batch, 0));
     TrsmArgs t{};
@@ -394,6 +407,7 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
     t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
     run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
+    }
     // step 3: F22 <- F22 - F21 F12, F21 untouched
     GemmArgs g{};
     g.ta = 0; g.tb = 0; g.max_m = max_n2; g.max_n = max_n2; g.max_k = max_n1;

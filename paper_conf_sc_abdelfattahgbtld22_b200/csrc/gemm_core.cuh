@@ -29,6 +29,10 @@ struct GemmDesc {
     double *C; long ldc;
     int m, n, k;
     double alpha, beta;
+    // MAP variants only (the row-map CTA kernel, lu_large.cu): logical row r
+    // of op(A) and C lives at storage row rmap[r]; row k of B at kmap[k]
+    // (shared-memory lists; the pointers above then carry column offsets only)
+    const int *rmap = nullptr, *kmap = nullptr;
 };
 
 struct GemmSmem {
@@ -40,38 +44,71 @@ constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
 // Issue the cp.async copies of K chunk [k0, k0+16) of tile (r0, c0) into buffer
 // `buf` (out-of-range elements are zero-filled with plain stores).
+template <bool MAP = false>
 __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int c0, int k0, GemmSmem &sm, int buf) {
     const int tid = threadIdx.x;
+    if (MAP) {
+        // the row of op(A) (tid & 63) and of B (tid & 15) are fixed per thread:
+        // one map lookup each, all before the cp.async sequence
+        const int r = tid & 63, gr = r0 + r, kb = tid & 15, gkb = k0 + kb;
+        const bool okr = gr < d.m, okb = gkb < d.k;
+        const double *arow = d.A + (okr ? d.rmap[gr] : 0);
+        const double *brow = d.B + (okb ? d.kmap[gkb] : 0);
+#pragma unroll
+        for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
+            const int kk = (tid >> 6) + 2 * q, gk = k0 + kk;
+            double *dst = &sm.As[buf][kk][r];
+            if (okr && gk < d.k) cp_async8(dst, arow + (size_t)gk * d.lda);
+            else *dst = 0.0;
+        }
+#pragma unroll
+        for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
+            const int c = (tid >> 4) + 8 * q, gc = c0 + c;
+            double *dst = &sm.Bs[buf][kb][c];
+            if (okb && gc < d.n) cp_async8(dst, brow + (size_t)gc * d.ldb);
+            else *dst = 0.0;
+        }
+        return;
+    }
 #pragma unroll
     for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int r, kk;
-        if (!d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
+        if (MAP || !d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
         const int gr = r0 + r, gk = k0 + kk;
         double *dst = &sm.As[buf][kk][r];
-        if (gr < d.m && gk < d.k) cp_async8(dst, d.ta ? d.A + gk + (size_t)gr * d.lda : d.A + gr + (size_t)gk * d.lda);
-        else *dst = 0.0;
+        if (gr < d.m && gk < d.k) {
+            if (MAP) cp_async8(dst, d.A + d.rmap[gr] + (size_t)gk * d.lda);
+            else cp_async8(dst, d.ta ? d.A + gk + (size_t)gr * d.lda : d.A + gr + (size_t)gk * d.lda);
+        } else {
+            *dst = 0.0;
+        }
     }
 #pragma unroll
     for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int c, kk;
-        if (!d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
+        if (MAP || !d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
         const int gc = c0 + c, gk = k0 + kk;
         double *dst = &sm.Bs[buf][kk][c];
-        if (gc < d.n && gk < d.k) cp_async8(dst, d.tb ? d.B + gc + (size_t)gk * d.ldb : d.B + gk + (size_t)gc * d.ldb);
-        else *dst = 0.0;
+        if (gc < d.n && gk < d.k) {
+            if (MAP) cp_async8(dst, d.B + d.kmap[gk] + (size_t)gc * d.ldb);
+            else cp_async8(dst, d.tb ? d.B + gc + (size_t)gk * d.ldb : d.B + gk + (size_t)gc * d.ldb);
+        } else {
+            *dst = 0.0;
+        }
     }
 }
 
+template <bool MAP = false>
 __device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, GemmSmem &sm) {
     if (d.beta == 0.0) return;
     const int tid = threadIdx.x;
     const int mr = imin(GBM, d.m - r0), nc = imin(GBN, d.n - c0);
-    for (int e = tid; e < GBM * GBN; e += G_NT) {
-        const int r = e & 63, c = e >> 6;
-        if (r < mr && c < nc) cp_async8(&sm.Cs[c][r], d.C + r0 + r + (size_t)(c0 + c) * d.ldc);
-    }
+    const int r = tid & 63;  // fixed per thread (G_NT = 2 x 64)
+    if (r >= mr) return;
+    const double *cr = d.C + (MAP ? d.rmap[r0 + r] : r0 + r);
+    for (int c = tid >> 6; c < nc; c += G_NT / 64) cp_async8(&sm.Cs[c][r], cr + (size_t)(c0 + c) * d.ldc);
 }
 
 // ---- DFMA path: thread (tx, ty) owns rows tx + 8q (q < 8), cols ty + 16p (p < 4);
@@ -122,23 +159,24 @@ __device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int 
     }
 }
 
-template <bool DMMA>
+template <bool DMMA, bool MAP = false>
 __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0, const GemmSmem &sm,
                                               const double (&acc)[32]) {
     const int tid = threadIdx.x;
     if (!DMMA) {
         const int tx = tid & 7, ty = tid >> 3;
 #pragma unroll
-        for (int p = 0; p < 4; ++p) {
-            const int cl = ty + 16 * p, c = c0 + cl;
-            if (c >= d.n) continue;
+        for (int q = 0; q < 8; ++q) {
+            const int rl = tx + 8 * q, r = r0 + rl;
+            if (r >= d.m) continue;
+            const int rs = MAP ? d.rmap[r] : r;
 #pragma unroll
-            for (int q = 0; q < 8; ++q) {
-                const int rl = tx + 8 * q, r = r0 + rl;
-                if (r >= d.m) continue;
+            for (int p = 0; p < 4; ++p) {
+                const int cl = ty + 16 * p, c = c0 + cl;
+                if (c >= d.n) continue;
                 double v = d.alpha * acc[q * 4 + p];
                 if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
-                d.C[r + (size_t)c * d.ldc] = v;
+                d.C[rs + (size_t)c * d.ldc] = v;
             }
         }
     } else {
@@ -148,6 +186,7 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
         for (int mi = 0; mi < 4; ++mi) {
             const int rl = (warp & 1) * 32 + 8 * mi + g, r = r0 + rl;
             if (r >= d.m) continue;
+            const int rs = MAP ? d.rmap[r] : r;
 #pragma unroll
             for (int ni = 0; ni < 4; ++ni) {
 #pragma unroll
@@ -156,7 +195,7 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
                     if (c >= d.n) continue;
                     double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
                     if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
-                    d.C[r + (size_t)c * d.ldc] = v;
+                    d.C[rs + (size_t)c * d.ldc] = v;
                 }
             }
         }
@@ -166,17 +205,17 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
 // A stream of tiles processed by one CTA with the software pipeline described
 // above.  `next(d, r0, c0)` returns false when the CTA has no more tiles.
 // DMMA selects the FP64 tensor-core path, else DFMA.
-template <bool DMMA, class Next>
+template <bool DMMA, class Next, bool MAP = false>
 __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     GemmDesc d, dn;
     int r0, c0, rn, cn;
     if (!next(d, r0, c0)) return;
     int buf = 0;
-    if (d.k > 0) gemm_issue_chunk(d, r0, c0, 0, sm, buf);
+    if (d.k > 0) gemm_issue_chunk<MAP>(d, r0, c0, 0, sm, buf);
     cp_async_commit();
     bool have = true;
     while (have) {
-        gemm_issue_c(d, r0, c0, sm);
+        gemm_issue_c<MAP>(d, r0, c0, sm);
         cp_async_commit();
         double acc[32];
 #pragma unroll
@@ -185,10 +224,10 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         bool has_next_tile = false;
         for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
             if (c + 1 < nchunks) {
-                gemm_issue_chunk(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
+                gemm_issue_chunk<MAP>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
             } else {
                 has_next_tile = next(dn, rn, cn);
-                if (has_next_tile && dn.k > 0) gemm_issue_chunk(dn, rn, cn, 0, sm, buf ^ 1);
+                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP>(dn, rn, cn, 0, sm, buf ^ 1);
             }
             cp_async_commit();
             if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();
@@ -202,7 +241,7 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         }
         cp_async_wait<1>();
         __syncthreads();
-        gemm_epilogue<DMMA>(d, r0, c0, sm, acc);
+        gemm_epilogue<DMMA, MAP>(d, r0, c0, sm, acc);
         __syncthreads();
         have = has_next_tile;
         if (have) { d = dn; r0 = rn; c0 = cn; }

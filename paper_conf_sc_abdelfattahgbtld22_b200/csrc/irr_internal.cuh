@@ -28,6 +28,8 @@ struct Tuning {
     int panel_win;       // 1: grid-wide panels by the windowed register panel (rows <= 2048)
     int strip;           // 1: fused interchange + TRSM + GEMM per 64-column strip (needs panel_win)
     int gemm_big;        // 1: long-K DCWI GEMMs on the 128x128 DMMA core (gemm_big.cuh)
+    int l1_rowmap;       // 1: L1 kernel in row-map form (no interchanges until one final permutation)
+    int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
 };
 Tuning &tuning();
 
@@ -38,7 +40,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();
@@ -75,7 +77,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }

@@ -64,11 +64,15 @@ def test_tier_m_boundary_and_extreme_shapes():
     _run_and_check(_uniform(shapes, seed=5))
 
 
-@pytest.mark.parametrize("l1", [1, 0])
+@pytest.mark.parametrize("l1", [1, 0, "swap"])
 @pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
 def test_tier_l_forced_small_nb(nb, l1):
-    """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256,
-    l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
+    """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256 in
+    row-map form, "swap": the same with eager interchanges, l1=0: grid-wide
+    kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
+    if l1 == "swap":
+        irr.irr_set_tuning("l1_rowmap", 0)
+        l1 = 1
     irr.irr_set_tuning("tier_s", 0)
     irr.irr_set_tuning("tier_m_max", 0)
     irr.irr_set_tuning("nb", nb)
@@ -99,10 +103,12 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "L", "L2"])
+@pytest.mark.parametrize("tier", ["default", "L", "L2", "Lswap"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
-    if tier in ("L", "L2"):
+    if tier == "Lswap":
+        irr.irr_set_tuning("l1_rowmap", 0)
+    if tier in ("L", "L2", "Lswap"):
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
     if tier == "L2":

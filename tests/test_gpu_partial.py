@@ -33,9 +33,12 @@ SHAPES = [(1, 1), (5, 7), (16, 3), (31, 1), (32, 40), (33, 65), (64, 200), (120,
           (700, 300)]
 
 
-@pytest.mark.parametrize("tier", ["default", "L"])
+@pytest.mark.parametrize("tier", ["default", "L", "unfused"])
 def test_g1_front_exact(tier):
-    """G1': F12 -> X, F22 -> S bit-exactly, F11 -> the chosen L\\U."""
+    """G1': F12 -> X, F22 -> S bit-exactly, F11 -> the chosen L\\U.  "unfused":
+    step a5.2 as irrLASWP + 2 x irrTRSM instead of the fused strip kernel."""
+    if tier == "unfused":
+        irr.irr_set_tuning("getrs_fused", 0)
     if tier == "L":
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
@@ -52,7 +55,9 @@ def test_g1_front_exact(tier):
         check_partial(F, n1, Fg, ip, int(inf), exact=True, label=f"{n1}/{F.shape[0]}")
 
 
-def test_uniform_fronts_vs_oracle():
+@pytest.mark.parametrize("fused", [1, 0])
+def test_uniform_fronts_vs_oracle(fused):
+    irr.irr_set_tuning("getrs_fused", fused)
     shapes = [(1, 0), (7, 0), (3, 4), (10, 10), (17, 40), (50, 80), (97, 31), (129, 257), (400, 500)]
     fronts = [(irrgen.front_values(8, g, n1 + n2), n1) for g, (n1, n2) in enumerate(shapes)]
     out, ipivs, info = gpu_partial(fronts)
