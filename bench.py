@@ -99,22 +99,22 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ per-tier algorithmic work
-def tier_of(m, n, tier_m_max=24576, l1=True):
-    """0 = S (warp), 1 = M (CTA, in smem), 2 = L1 (CTA per matrix), 3 = L2
-    (grid-wide chain), -1 = empty; mirrors classify.cu."""
+def tier_of(m, n, tier_m_max=24576, l1=256):
+    """0 = S (warp), 1 = M (CTA, in smem), 2 = L1 (CTA per matrix, m <= l1
+    rows; 0 = off), 3 = L2 (grid-wide chain), -1 = empty; mirrors classify.cu."""
     m = np.asarray(m)
     n = np.asarray(n)
     lds = m | 1
     t = np.full(len(m), 3)
     if l1:
-        t[m <= 256] = 2
+        t[m <= l1] = 2
     t[(lds * n) <= tier_m_max] = 1
     t[(m <= 32) & (n <= 32)] = 0
     t[(m == 0) | (n == 0)] = -1
     return t
 
 
-def class_work(m, n, nb=32, tier_m_max=24576, l1=True):
+def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
     """Algorithmic (flops, bytes) per kernel class for one getrf step
     (DESIGN.md 'Roofline accounting'); tiers mirror classify.cu with the
     library's live tuning."""
@@ -150,7 +150,7 @@ def class_work(m, n, nb=32, tier_m_max=24576, l1=True):
     return out
 
 
-def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=True):
+def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=256):
     n1 = np.asarray(n1, dtype=np.int64)
     n2 = np.asarray(n2, dtype=np.int64)
     out = class_work(n1, n1, nb, tier_m_max, l1)
@@ -287,7 +287,7 @@ def main():
         ld_loc = B.ld_h
         call = lambda: B.getrf()  # noqa: E731
         cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
-                        bool(irr.irr_get_tuning("l1")))
+                        irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
         bytes_local = float(F.getrf_bytes(m_loc, n_loc).sum())
         host = B.host_buffer(pinned=True)
         hn = host.numpy()
@@ -299,7 +299,7 @@ def main():
         B = FrontBatch(m_loc, n_loc, device=dev)
         call = lambda: B.getrf_partial()  # noqa: E731
         cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
-                                bool(irr.irr_get_tuning("l1")))
+                                irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
         bytes_local = float(F.partial_bytes(m_loc, n_loc).sum())
         host = torch.empty(B.total, dtype=torch.float64, pin_memory=True)
         hn = host.numpy()
@@ -399,7 +399,14 @@ def main():
 
     # ---- roofline of the dominant kernel class (rank-local, per step)
     hbm, hbm_src = peaks()
-    dom = max(prof.items(), key=lambda kv: kv[1][0])
+    # tiers S and M run on a forked stream concurrently with the large tiers:
+    # their events also span the time spent waiting for SMs, so the dominant
+    # kernel is taken among the main-stream classes whenever a large tier ran
+    side = {"lu_small", "lu_mid"}
+    main = {k: v for k, v in prof.items() if k not in side and v[1]}
+    big_ran = any(k in main for k in ("lu_l1", "panel", "strip", "gemm_trailing"))
+    cand = main if big_ran else {k: v for k, v in prof.items() if v[1]}
+    dom = max(cand.items(), key=lambda kv: kv[1][0])
     dname, (dms, dcnt) = dom
     dms_step = dms / args.steps
     fl, by = cw.get(dname, (0.0, 0.0))

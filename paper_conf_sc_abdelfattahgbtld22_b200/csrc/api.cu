@@ -31,7 +31,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // defaults chosen by measurement on B200: tier M only up to
 // 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1, 0, 1};
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1, 0, 1, L1_MAX_ROWS};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -142,13 +142,14 @@ struct Work {
     int *bins;
     int *tile_off;
     int *sort;  // size sort (sched.cuh): sorted slots + bucket prefix
+    int *keys;  // per-matrix sort keys
     void *plans;  // getrf / partial only: one interchange plan per tier-L slot
 };
 
 static size_t work_bytes_for(int batch) {
     size_t b = (size_t)(batch > 0 ? batch : 1);
     return align256(CNT_INTS * sizeof(int)) + align256(NBINS * b * sizeof(int)) + align256((b + 1) * sizeof(int)) +
-           align256(size_sort_ints((int)b) * sizeof(int));
+           align256(size_sort_ints((int)b) * sizeof(int)) + align256(b * sizeof(int));
 }
 
 // getrf / partial: the common part plus the per-slot interchange plans of the
@@ -170,6 +171,8 @@ static Work carve(void *work, int batch) {
     p += align256((b + 1) * sizeof(int));
     w.sort = (int *)p;
     p += align256(size_sort_ints((int)b) * sizeof(int));
+    w.keys = (int *)p;
+    p += align256(b * sizeof(int));
     w.plans = p;  // valid only in a work_bytes_getrf() workspace
     return w;
 }
@@ -219,8 +222,8 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
             if (big > M2_ELEMS && mmax > M2_ELEMS) launch_lu_mid(a, w.counters, w.bins, BIN_M3, (int)mmax, side);
         }
         if (has_large) {
-            if (t.l1) launch_lu_l1(a, w.counters, w.bins, s);
-            if (!t.l1 || a.max_m > L1_MAX_ROWS) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, s);
+            if (t.l1) launch_lu_l1(a, w.counters, w.bins, w.keys, w.sort, s);
+            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, s);
         }
     }
     if (side != s) {
@@ -298,6 +301,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "gemm_big")) g_tuning.gemm_big = value ? 1 : 0;
     else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
     else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
+    else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
 }
 
 int irr_get_tuning(const char *key) {
@@ -318,6 +322,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "gemm_big")) return g_tuning.gemm_big;
     if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
     if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
+    if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
     return -1;
 }
 

@@ -33,7 +33,7 @@ __global__ void __launch_bounds__(256) classify_kernel(GetrfArgs a, int *counter
             else if (el <= M1_ELEMS && el <= tier_m_max) bin = BIN_M1;
             else if (el <= M2_ELEMS && el <= tier_m_max) bin = BIN_M2;
             else if (el <= tier_m_max) bin = BIN_M3;
-            else if (l1 && mi <= L1_MAX_ROWS) bin = BIN_L1;
+            else if (l1 && mi <= l1) bin = BIN_L1;  // l1 = max rows of the CTA-per-matrix tier
             else bin = BIN_L;
         }
     }
@@ -54,7 +54,7 @@ void launch_classify(const GetrfArgs &a, int *counters, int *bins, int keep_neg_
     const Tuning &t = tuning();
     int grid = (a.batch + 255) / 256;
     KScope k(K_CLASSIFY, s);
-    classify_kernel<<<grid, 256, 0, s>>>(a, counters, bins, keep_neg_info, t.tier_s, t.tier_m_max, t.l1);
+    classify_kernel<<<grid, 256, 0, s>>>(a, counters, bins, keep_neg_info, t.tier_s, t.tier_m_max, t.l1 ? t.l1_rows : 0);
 }
 
 // max over the batch of the local dims (only when the caller passes required

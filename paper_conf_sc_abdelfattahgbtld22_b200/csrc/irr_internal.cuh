@@ -30,6 +30,7 @@ struct Tuning {
     int gemm_big;        // 1: long-K DCWI GEMMs on the 128x128 DMMA core (gemm_big.cuh)
     int l1_rowmap;       // 1: L1 kernel in row-map form (no interchanges until one final permutation)
     int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
+    int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
 };
 Tuning &tuning();
 
@@ -66,7 +67,8 @@ struct KScope {
 // L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
 // kernels per panel iteration.
 enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, NBINS = 6 };
-constexpr int L1_MAX_ROWS = 256;
+constexpr int L1_MAX_ROWS = 256;    // panels up to this many rows are staged in shared memory
+constexpr int L1_TALL_ROWS = 1024;  // taller L1 panels: panel_win in global memory (128 threads x 8 rows)
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
 constexpr int M2_ELEMS = 12288;   // 96 KB  -> 2 CTAs / SM
 constexpr int TIER_M_MAX_DEFAULT = 24576;  // 192 KB -> 1 CTA / SM
@@ -185,7 +187,7 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
 // lu_large.cu
 constexpr size_t SWAP_PLAN_BYTES = 1040;  // sizeof(SwapPlan), checked in lu_large.cu
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, cudaStream_t s);
-void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream_t s);
+void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)
 struct GemmArgs {

@@ -22,6 +22,7 @@
 #include "gemm_core.cuh"
 #include "panel.cuh"
 #include "panel_win.cuh"
+#include "sched.cuh"
 
 namespace irr {
 
@@ -204,10 +205,25 @@ __device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni
 
 // ================================================================== L1
 // One CTA per matrix, all iterations inside (matrices with m <= L1 rows).
-template <bool DMMA>
+// tall L1 panels (257..1024 rows)
+__device__ __forceinline__ int l1_panel_tall(double *gP, long ld, int rows, int ib, int *piv,
+                                          PanelWinSmem<L1_NT / 32, 32> &pws) {
+    return rows <= 4 * L1_NT ? panel_win<L1_NT, 4, 8, 32>(gP, ld, rows, ib, piv, pws)
+                             : panel_win<L1_NT, 8, 4, 32>(gP, ld, rows, ib, piv, pws);
+}
+
+// Matrices are taken largest first (LPT): `order` is the L1 list sorted by
+// descending work (l1_key_kernel + the device size sort), `order_count` its
+// length; without a sort the classify order is used.
+// Panels of up to 256 rows are staged in shared memory and factored in
+// registers (panel_regs); taller ones (<= 1024 rows) are factored in place in
+// global memory by the windowed register panel (panel_win).
+template <bool DMMA, bool TALL>
 __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__restrict__ counters,
                                                          const int *__restrict__ bins, int nb,
-                                                         int l1_region_doubles, int phase_timing) {
+                                                         int l1_region_doubles, int phase_timing,
+                                                         const int *__restrict__ order,
+                                                         const int *__restrict__ order_count) {
     extern __shared__ __align__(16) unsigned char l1_smem[];
     __shared__ PanelScratch sc;
     __shared__ __align__(16) PanelRegScratch<L1_NT / 32, 32> prs;
@@ -216,9 +232,10 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
     __shared__ int next_s;
     double *smd = reinterpret_cast<double *>(l1_smem);
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(l1_smem);
+    PanelWinSmem<L1_NT / 32, 32> &pws = *reinterpret_cast<PanelWinSmem<L1_NT / 32, 32> *>(l1_smem);
     const int tid = threadIdx.x;
-    const int count = counters[CNT_BIN0 + BIN_L1];
-    const int *list = bins + (size_t)BIN_L1 * a.batch;
+    const int count = order ? *order_count : counters[CNT_BIN0 + BIN_L1];
+    const int *list = order ? order : bins + (size_t)BIN_L1 * a.batch;
     while (true) {
         if (tid == 0) next_s = atomicAdd(&counters[CNT_L1_NEXT], 1);
         __syncthreads();
@@ -237,18 +254,36 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
         for (int j = 0; j < K; j += nb) {
             const int ib = K - j < nb ? K - j : nb;
             const int rows = mi - j, c1 = j + ib;
-            // ---- a4.1 panel, staged in shared memory
-            double *P = smd;
-            const int ldp = rows | 1;
+            // ---- a4.1 panel, staged in shared memory (<= 256 rows) or in place
             double *gP = gA + j + (size_t)j * ld;
-            stage_block_async(P, ldp, gP, ld, rows, ib, tid, L1_NT);
-            cp_async_commit();
-            cp_async_wait<0>();
-            __syncthreads();
+            const bool staged = !TALL || rows <= L1_MAX_ROWS;
+            double *P = staged ? smd : gP;
+            const int ldp = staged ? (rows | 1) : (int)ld;
+            if (staged) {
+                stage_block_async(P, ldp, gP, ld, rows, ib, tid, L1_NT);
+                cp_async_commit();
+                cp_async_wait<0>();
+                __syncthreads();
+            }
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 3, (unsigned long long)(t1 - t0)); t0 = t1; }
             const bool regs_panel = ib <= 32;
-            const int z = regs_panel ? panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs, &sp, j)
-                                     : panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            int z;
+            if (staged) {
+                z = regs_panel ? panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs, &sp, j)
+                               : panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            } else if (TALL && regs_panel) {
+                z = l1_panel_tall(gP, ld, rows, ib, piv_s, pws);
+                // the plan in absolute rows for the interchange pass
+                if (tid < ib) sp.top_src[tid] = j + pws.plan.top_src[tid];
+                if (tid < pws.plan.nbot) {
+                    sp.bot_pos[tid] = j + pws.plan.bot_pos[tid];
+                    sp.bot_src[tid] = j + pws.plan.bot_src[tid];
+                }
+                if (tid == 0) sp.nbot = pws.plan.nbot;
+                __syncthreads();
+            } else {
+                z = panel_getf2<L1_NT>(P, ldp, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            }
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 4, (unsigned long long)(t1 - t0)); t0 = t1; }
             if (z && !info) info = j + z;
             // write the factored panel back; keep the strict lower triangle of
@@ -258,8 +293,9 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                 const int lane = tid & 31, warp = tid >> 5;
                 for (int c = warp; c < ib; c += L1_NT / 32) {
                     double *gc = gP + (size_t)c * ld;
-                    const double *pc = P + c * ldp;
-                    for (int r = lane; r < rows; r += 32) gc[r] = pc[r];
+                    const double *pc = P + (size_t)c * ldp;
+                    if (staged)
+                        for (int r = lane; r < rows; r += 32) gc[r] = pc[r];
                     double *lc = L11p + (c * (2 * ib - c - 1)) / 2 - (c + 1);
                     for (int r = c + 1 + lane; r < ib; r += 32) lc[r] = pc[r];
                 }
@@ -749,14 +785,42 @@ static size_t l1_region_bytes(int nb) {
     return (m + 15) & ~size_t(15);
 }
 
-void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream_t s) {
+// LPT key of an L1 matrix: 32 + cube root of its m n min(m,n) (>= 32, so the
+// bucketed size sort puts every L1 matrix before the zero keys of the rest)
+__global__ void l1_key_kernel(GetrfArgs a, const int *__restrict__ counters, const int *__restrict__ bins,
+                              int *__restrict__ key) {
+    const int count = counters[CNT_BIN0 + BIN_L1];
+    const int *list = bins + (size_t)BIN_L1 * a.batch;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < count; t += gridDim.x * blockDim.x) {
+        const int i = list[t];
+        const double m = a.m[i], n = a.n[i];
+        key[i] = 32 + (int)cbrt(m * n * (m < n ? m : n));
+    }
+}
+
+void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s) {
+    const int *order = nullptr, *order_count = nullptr;
+    if (keys && sort_ws) {
+        cudaMemsetAsync(keys, 0, (size_t)a.batch * sizeof(int), s);
+        {
+            KScope k(K_MISC, s);
+            int g = (a.batch + 255) / 256;
+            l1_key_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(a, counters, bins, keys);
+        }
+        launch_size_sort(keys, a.batch, sort_ws, s);
+        SlotList sl = sorted_slots(sort_ws, a.batch, 31);
+        order = sl.idx;
+        order_count = sl.prefix + sl.bucket0;
+    }
     const int nb = clamp_nb(tuning().nb);
     const size_t region = l1_region_bytes(nb);
     const size_t smem = region + (size_t)(nb * (nb - 1) / 2 + 2) * sizeof(double);
     static size_t attr = 0;
     if (smem > attr) {
-        cudaFuncSetAttribute(lu_l1_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaFuncSetAttribute(lu_l1_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_l1_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
     int per_sm = tuning().l1_ctas_per_sm;
@@ -764,7 +828,7 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     KScope k(K_LU_L1, s);
-    if (tuning().l1_rowmap && nb <= 32) {
+    if (tuning().l1_rowmap && nb <= 32 && tuning().l1_rows <= L1_MAX_ROWS) {
         const size_t smem_map = smem + (size_t)L1_MAX_ROWS * sizeof(int);
         static size_t attr_map = 0;
         if (smem_map > attr_map) {
@@ -780,12 +844,17 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, cudaStream
                                                                  tuning().phase_timing);
         return;
     }
-    if (tuning().l1_dmma)  // measured: DFMA is faster inside L1 (DMMA variant spills)
-        lu_l1_kernel<true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
-                                                     tuning().phase_timing);
-    else
-        lu_l1_kernel<false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
-                                                      tuning().phase_timing);
+    // the tall-panel variant only when the bin can hold > 256 rows (it needs
+    // more registers: the default variant keeps the lower spill count)
+    const bool tall = tuning().l1_rows > L1_MAX_ROWS;
+    const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing;
+    if (tuning().l1_dmma) {  // measured: DFMA is faster inside L1 (DMMA variant spills)
+        if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+        else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+    } else {
+        if (tall) lu_l1_kernel<false, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+        else lu_l1_kernel<false, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+    }
 }
 
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans_v,

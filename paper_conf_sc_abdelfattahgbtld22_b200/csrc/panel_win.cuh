@@ -20,25 +20,24 @@
 namespace irr {
 
 constexpr int PW_WBMAX = 16;
-constexpr int PW_LD = 65;  // row stride of the 64 x 64 shared tiles
 
-template <int NW>
+template <int NW, int NBX = 64>  // NBX: largest panel width (<= 64)
 struct PanelWinSmem {
-    double Us[64 * PW_LD];  // U rows: Us[p][k], k >= p
-    double Lb[64 * PW_LD];  // L of the pivot rows: Lb[p][s], s < p
-    double Ds[64 * PW_LD];  // L of the rows pushed below the panel block (end)
+    double Us[NBX * (NBX + 1)];  // U rows: Us[p][k], k >= p
+    double Lb[NBX * (NBX + 1)];  // L of the pivot rows: Lb[p][s], s < p
+    double Ds[NBX * (NBX + 1)];  // L of the rows pushed below the panel block (end)
     double row[2][NW][PW_WBMAX];  // published candidate rows (double-buffered)
     unsigned long long key[2][NW];
     int pos[2][NW], orig[2][NW];
-    int srcpos[64];  // original row now at pivot position p
+    int srcpos[NBX];  // original row now at pivot position p
     SwapPlan plan;
 };
 
 // One column step on the W active (shifted) columns of the window ending at
 // column bend.  Same protocol as preg_step; differs in where results go.
-template <int NT, int RPT, int WB, int W>
+template <int NT, int RPT, int WB, int W, int NBX>
 __device__ __forceinline__ void pwin_step(double (&a)[RPT][WB], int (&pos)[RPT], int c, int bend, double *gP,
-                                          long ld, int rows, int *piv, PanelWinSmem<NT / 32> &sm, int &zero_at) {
+                                          long ld, int rows, int *piv, PanelWinSmem<NT / 32, NBX> &sm, int &zero_at) {
     constexpr int NW = NT / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int par = c & 1;
@@ -91,7 +90,7 @@ __device__ __forceinline__ void pwin_step(double (&a)[RPT][WB], int (&pos)[RPT],
         piv[c] = pmin;
         sm.srcpos[c] = sm.orig[par][wbest];
     }
-    if (tid < bend - c) sm.Us[c * PW_LD + c + tid] = u[tid];  // U row c inside the window
+    if (tid < bend - c) sm.Us[c * (NBX + 1) + c + tid] = u[tid];  // U row c inside the window
 #pragma unroll
     for (int q = 0; q < RPT; ++q) {
         if (pos[q] == c) pos[q] = pmin;
@@ -142,8 +141,8 @@ __device__ __forceinline__ void pwin_step(double (&a)[RPT][WB], int (&pos)[RPT],
 // panel in LAPACK row order, piv[c] the 0-based pivot position of column c,
 // and sm.plan the interchange plan (relative rows).  Returns the 1-based column
 // of the first exact zero pivot, or 0.  All NT threads must call it.
-template <int NT, int RPT, int WB>
-__device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelWinSmem<NT / 32> &sm) {
+template <int NT, int RPT, int WB, int NBX = 64>
+__device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelWinSmem<NT / 32, NBX> &sm) {
     constexpr int NW = NT / 32;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     double a[RPT][WB];
@@ -169,22 +168,22 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
             const int p0 = b0 - WB;
             for (int s = warp; s < b0; s += NW)
                 for (int p = imax(p0, s + 1) + lane; p < b0; p += 32)
-                    sm.Lb[p * PW_LD + s] = gP[sm.srcpos[p] + (size_t)s * ld];
+                    sm.Lb[p * (NBX + 1) + s] = gP[sm.srcpos[p] + (size_t)s * ld];
             for (int k = warp; k < bw; k += NW)
-                for (int p = lane; p < b0; p += 32) sm.Us[p * PW_LD + b0 + k] = gP[sm.srcpos[p] + (size_t)(b0 + k) * ld];
+                for (int p = lane; p < b0; p += 32) sm.Us[p * (NBX + 1) + b0 + k] = gP[sm.srcpos[p] + (size_t)(b0 + k) * ld];
             __syncthreads();
             // (iii) U[0:b0, window] = L11^{-1} U[0:b0, window]: warp per column,
             // the column in registers (2 rows per lane), x_s by shuffle
             for (int k = warp; k < bw; k += NW) {
-                double x0 = lane < b0 ? sm.Us[lane * PW_LD + b0 + k] : 0.0;
-                double x1 = lane + 32 < b0 ? sm.Us[(lane + 32) * PW_LD + b0 + k] : 0.0;
+                double x0 = lane < b0 ? sm.Us[lane * (NBX + 1) + b0 + k] : 0.0;
+                double x1 = lane + 32 < b0 ? sm.Us[(lane + 32) * (NBX + 1) + b0 + k] : 0.0;
                 for (int s = 0; s < b0 - 1; ++s) {
                     const double xs = __shfl_sync(FULL, s < 32 ? x0 : x1, s & 31);
-                    if (lane > s && lane < b0) x0 = fma(-sm.Lb[lane * PW_LD + s], xs, x0);
-                    if (lane + 32 > s && lane + 32 < b0) x1 = fma(-sm.Lb[(lane + 32) * PW_LD + s], xs, x1);
+                    if (lane > s && lane < b0) x0 = fma(-sm.Lb[lane * (NBX + 1) + s], xs, x0);
+                    if (lane + 32 > s && lane + 32 < b0) x1 = fma(-sm.Lb[(lane + 32) * (NBX + 1) + s], xs, x1);
                 }
-                if (lane < b0) sm.Us[lane * PW_LD + b0 + k] = x0;
-                if (lane + 32 < b0) sm.Us[(lane + 32) * PW_LD + b0 + k] = x1;
+                if (lane < b0) sm.Us[lane * (NBX + 1) + b0 + k] = x0;
+                if (lane + 32 < b0) sm.Us[(lane + 32) * (NBX + 1) + b0 + k] = x1;
             }
             __syncthreads();
             // (iv) rows still below the pivots: a -= L(r, 0:b0) U(0:b0, window)
@@ -195,7 +194,7 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
                 double l[RPT];
 #pragma unroll
                 for (int q = 0; q < RPT; ++q) l[q] = live[q] ? gP[tid + NT * q + (size_t)s * ld] : 0.0;
-                const double *us = sm.Us + s * PW_LD + b0;
+                const double *us = sm.Us + s * (NBX + 1) + b0;
 #pragma unroll
                 for (int k = 0; k < WB; ++k) {
                     const double uk = us[k];
@@ -208,11 +207,11 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
         int c = b0;
         if (WB >= 16)
             for (; c < bend && bend - c > 8; ++c)
-                pwin_step<NT, RPT, WB, (WB >= 16 ? 16 : WB)>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
+                pwin_step<NT, RPT, WB, (WB >= 16 ? 16 : WB), NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
         if (WB >= 8)
             for (; c < bend && bend - c > 4; ++c)
-                pwin_step<NT, RPT, WB, (WB >= 8 ? 8 : WB)>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
-        for (; c < bend; ++c) pwin_step<NT, RPT, WB, 4>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
+                pwin_step<NT, RPT, WB, (WB >= 8 ? 8 : WB), NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
+        for (; c < bend; ++c) pwin_step<NT, RPT, WB, 4, NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
         __syncthreads();
     }
     // ---- the permutation: L of the last window's pivots, and of the rows
@@ -221,7 +220,7 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
         const int p0 = ((ib - 1) / WB) * WB;
         for (int s = warp; s < ib; s += NW)
             for (int p = imax(p0, s + 1) + lane; p < ib; p += 32)
-                sm.Lb[p * PW_LD + s] = gP[sm.srcpos[p] + (size_t)s * ld];
+                sm.Lb[p * (NBX + 1) + s] = gP[sm.srcpos[p] + (size_t)s * ld];
     }
 #pragma unroll
     for (int q = 0; q < RPT; ++q) {
@@ -234,7 +233,7 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
                 const int b = atomicAdd(&sm.plan.nbot, 1);
                 sm.plan.bot_pos[b] = p;
                 sm.plan.bot_src[b] = r;
-                for (int s = 0; s < ib; ++s) sm.Ds[b * PW_LD + s] = gP[r + (size_t)s * ld];
+                for (int s = 0; s < ib; ++s) sm.Ds[b * (NBX + 1) + s] = gP[r + (size_t)s * ld];
             }
         }
     }
@@ -242,8 +241,8 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
     const int nbot = sm.plan.nbot;
     for (int s = warp; s < ib; s += NW) {
         for (int p = lane; p < ib; p += 32)
-            gP[p + (size_t)s * ld] = s < p ? sm.Lb[p * PW_LD + s] : sm.Us[p * PW_LD + s];
-        for (int b = lane; b < nbot; b += 32) gP[sm.plan.bot_pos[b] + (size_t)s * ld] = sm.Ds[b * PW_LD + s];
+            gP[p + (size_t)s * ld] = s < p ? sm.Lb[p * (NBX + 1) + s] : sm.Us[p * (NBX + 1) + s];
+        for (int b = lane; b < nbot; b += 32) gP[sm.plan.bot_pos[b] + (size_t)s * ld] = sm.Ds[b * (NBX + 1) + s];
     }
     __syncthreads();
     return zero_at;

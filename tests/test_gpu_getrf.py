@@ -64,14 +64,15 @@ def test_tier_m_boundary_and_extreme_shapes():
     _run_and_check(_uniform(shapes, seed=5))
 
 
-@pytest.mark.parametrize("l1", [1, 0, "swap"])
+@pytest.mark.parametrize("l1", [1, 0, "rowmap"])
 @pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
 def test_tier_l_forced_small_nb(nb, l1):
-    """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256 in
-    row-map form, "swap": the same with eager interchanges, l1=0: grid-wide
-    kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
-    if l1 == "swap":
-        irr.irr_set_tuning("l1_rowmap", 0)
+    """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256,
+    "rowmap": the same in row-map form (interchanges as a relabelling, one
+    final permutation), l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1
+    sizes."""
+    if l1 == "rowmap":
+        irr.irr_set_tuning("l1_rowmap", 1)
         l1 = 1
     irr.irr_set_tuning("tier_s", 0)
     irr.irr_set_tuning("tier_m_max", 0)
@@ -103,12 +104,14 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "L", "L2", "Lswap"])
+@pytest.mark.parametrize("tier", ["default", "L", "L2", "Lswap", "Ltall"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
     if tier == "Lswap":
-        irr.irr_set_tuning("l1_rowmap", 0)
-    if tier in ("L", "L2", "Lswap"):
+        irr.irr_set_tuning("l1_rowmap", 1)
+    if tier == "Ltall":
+        irr.irr_set_tuning("l1_rows", 1024)
+    if tier in ("L", "L2", "Lswap", "Ltall"):
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
     if tier == "L2":
@@ -192,8 +195,12 @@ def test_c2_scaled_parity():
     assert st.get("match", 0) >= len(mats) - 3
 
 
-def test_c3_sample_parity():
-    """configs[2] shape (square U{256..1024}), a sample of 12 matrices."""
+@pytest.mark.parametrize("l1_rows", [256, 1024])
+def test_c3_sample_parity(l1_rows):
+    """configs[2] shape (square U{256..1024}), a sample of 12 matrices; with
+    l1_rows = 1024 every one is factored by the CTA-per-matrix tier, whose
+    panels above 256 rows run in place in global memory (panel_win)."""
+    irr.irr_set_tuning("l1_rows", l1_rows)
     cfg = irrgen.config("C3", scale=0.006)
     mats = [irrgen.uniform_values(cfg.seed, g, int(m), int(n)) for g, (m, n) in enumerate(zip(cfg.m, cfg.n))]
     _run_and_check(mats)
