@@ -21,7 +21,6 @@ import argparse
 import json
 import os
 import statistics
-import subprocess
 import sys
 import time
 
@@ -51,51 +50,65 @@ def peaks():
 
 # ------------------------------------------------------------------ clocks
 class ClockSampler:
-    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clock and throttle reasons sampled DURING the timed region: an NVML
+    polling thread (every ~2 ms, so short timed regions still get samples);
+    nvidia-smi is the fallback when NVML is not importable."""
+    REASONS = (("hw_slowdown", "nvmlClocksEventReasonHwSlowdown"),
+               ("hw_thermal_slowdown", "nvmlClocksEventReasonHwThermalSlowdown"),
+               ("sw_thermal_slowdown", "nvmlClocksEventReasonSwThermalSlowdown"),
+               ("sw_power_cap", "nvmlClocksEventReasonSwPowerCap"))
 
     def __init__(self, gpu_index: int):
-        self.proc = None
         self.idx = gpu_index
-        self.path = os.path.join("/tmp", f"irr_clocks_{os.getpid()}.csv")
+        self.thread = None
+        self.samples = []
+        self.reasons = set()
+        self.mx = 0.0
+
+    def _run(self):
+        import pynvml as nv
+        h = self.h
+        while not self.stop_flag:
+            try:
+                self.samples.append(float(nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)))
+                bits = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+                for name, attr in self.REASONS:
+                    if bits & getattr(nv, attr, 0):
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.002)
 
     def start(self):
+        import threading
         try:
-            self.f = open(self.path, "w")
-            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
-                                         stdout=self.f, stderr=subprocess.DEVNULL)
+            import pynvml as nv
+            nv.nvmlInit()
+            # NVML enumerates all GPUs; map through CUDA_VISIBLE_DEVICES if set
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            phys = self.idx
+            if vis:
+                toks = [t.strip() for t in vis.split(",") if t.strip()]
+                if self.idx < len(toks) and toks[self.idx].isdigit():
+                    phys = int(toks[self.idx])
+            self.h = nv.nvmlDeviceGetHandleByIndex(phys)
+            self.mx = float(nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM))
         except Exception:
-            self.proc = None
+            self.thread = None
+            return
+        self.stop_flag = False
+        self.thread = threading.Thread(target=self._run, daemon=True)
+        self.thread.start()
 
     def stop(self):
-        if self.proc is None:
+        if self.thread is None:
             return None
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
-        self.f.close()
-        sms, mx, reasons = [], 0.0, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in open(self.path):
-            parts = [x.strip() for x in line.split(",")]
-            if len(parts) < 8:
-                continue
-            try:
-                sms.append(float(parts[0]))
-                mx = max(mx, float(parts[1]))
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[4:8]):
-                if v.lower() == "active":
-                    reasons.add(nm)
-        if not sms:
+        self.stop_flag = True
+        self.thread.join(timeout=5)
+        if not self.samples:
             return None
-        return {"sm_mhz": statistics.median(sms), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sms)}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.mx,
+                "reasons": sorted(self.reasons), "samples": len(self.samples), "source": "nvml"}
 
 
 # ------------------------------------------------------------------ per-tier algorithmic work
@@ -282,6 +295,11 @@ def main():
     flops_local = float(work[mine].sum())
     flops_global = float(work.sum())
 
+    # C5 (200,000 fronts, 68 GB) is generated on the device, per rank, from
+    # the same global-id-keyed stream (irrgen.device; byte-equal to the host
+    # generator): neither a host copy nor a pristine device copy fits
+    devgen = args.config.startswith("C5")
+    host = None
     if kind == "getrf":
         B = MatrixBatch(m_loc, n_loc, device=dev)
         ld_loc = B.ld_h
@@ -289,25 +307,26 @@ def main():
         cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
                         irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
         bytes_local = float(F.getrf_bytes(m_loc, n_loc).sum())
-        host = B.host_buffer(pinned=True)
-        hn = host.numpy()
-        hn[:] = 0.0
-        # values keyed by GLOBAL id so a matrix is identical at every N
-        irrgen.fill_packed(cfg.seed, m_loc, n_loc, ld_loc, B.offsets, hn, gids=mine)
-        outs = [B.data, B.ipiv_data, B.info]
+        gm, gn = m_loc, n_loc
     else:
         B = FrontBatch(m_loc, n_loc, device=dev)
         call = lambda: B.getrf_partial()  # noqa: E731
         cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
                                 irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
         bytes_local = float(F.partial_bytes(m_loc, n_loc).sum())
+        gm = gn = B.nf_h
+    outs = [B.data, B.ipiv_data, B.info]
+    if devgen:
+        from irrgen import device as gdev
+        filler = gdev.Filler(cfg.seed, gm, gn, B.ld_h, B.offsets, mine, dev)
+        pristine = None
+    else:
         host = torch.empty(B.total, dtype=torch.float64, pin_memory=True)
         hn = host.numpy()
         hn[:] = 0.0
-        nf = B.nf_h
-        irrgen.fill_packed(cfg.seed, nf, nf, B.ld_h, B.offsets, hn, gids=mine)
-        outs = [B.data, B.ipiv_data, B.info]
-    pristine = host.to(dev)
+        # values keyed by GLOBAL id so a matrix is identical at every N
+        irrgen.fill_packed(cfg.seed, gm, gn, B.ld_h, B.offsets, hn, gids=mine)
+        pristine = host.to(dev)
     flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device=dev)   # > 126 MB L2
     stream = torch.cuda.current_stream(dev)
 
@@ -323,7 +342,10 @@ def main():
             dist.all_gather_into_tensor(gathered, status)
 
     def restore():
-        B.data.copy_(pristine)
+        if devgen:
+            filler.fill(B.data)
+        else:
+            B.data.copy_(pristine)
         flush.zero_()
 
     # ---- warm-up
@@ -370,7 +392,10 @@ def main():
 
     # ---- e2e: host buffers through the public API, H2D + compute + D2H inside the timed region
     e2e = None
-    if not args.no_e2e:
+    if devgen and not args.no_e2e:
+        e2e = {"value": None, "unit": "Gflop/s", "h2d_bytes_per_step": None, "d2h_bytes_per_step": None,
+               "note": "not measured: the batch (68 GB for C5) is generated on the device; no host copy fits"}
+    elif not args.no_e2e:
         res_host = [torch.empty(o.numel(), dtype=o.dtype, pin_memory=True) for o in outs]
         h2d = host.numel() * 8
         d2h = sum(o.numel() * o.element_size() for o in outs)
@@ -453,6 +478,8 @@ def main():
                            "batch_per_gpu": int(B.batch), "global_batch": int(len(cfg.m)),
                            "sharding": "LPT by flops" if world > 1 else "none",
                            "l2": "flushed (512 MB write) and inputs restored before every step, untimed",
+                           "inputs": "generated on the device per step (untimed)" if devgen else
+                                     "restored from a pristine device copy per step (untimed)",
                            "tuning": {k: irr.irr_get_tuning(k) for k in ("nb", "tier_m_max", "panel_rows")}},
                 "gpu_launches": int(launches), "roofline": roof, "whole_step": whole,
                 "kernel_ms_per_step": {k: v[0] / args.steps for k, v in prof.items() if v[1]},

@@ -30,8 +30,10 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 
 // defaults chosen by measurement on B200: tier M only up to
 // 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
-// grid-wide GEMMs (22.1 vs 17.5 TFLOP/s), DFMA inside L1.
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 0, 1, 1, 1, 0, 1, L1_MAX_ROWS};
+// grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
+// the deferred interchanges took the L1 kernel off its spills), deferred L1
+// left-block interchanges (6.80 -> 6.53 ms).
+static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -302,6 +304,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
     else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
+    else if (!strcmp(key, "l1_defer")) g_tuning.l1_defer = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -323,6 +326,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
     if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
+    if (!strcmp(key, "l1_defer")) return g_tuning.l1_defer;
     return -1;
 }
 

@@ -31,6 +31,7 @@ struct Tuning {
     int l1_rowmap;       // 1: L1 kernel in row-map form (no interchanges until one final permutation)
     int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
     int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
+    int l1_defer;        // 1: L1 applies the left-block interchanges once at the end (coalesced)
 };
 Tuning &tuning();
 
@@ -104,6 +105,39 @@ __device__ __forceinline__ void warp_argmax(bool cand, unsigned long long key, i
     unsigned r = __reduce_min_sync(FULL, e2 ? (unsigned)row : 0xffffffffu);
     kout = ((unsigned long long)mhi << 32) | mlo;
     rout = (int)r;  // 0xffffffff -> -1
+}
+
+// Warp arg-max as above, returning the WINNING LANE (-1: no candidate); the
+// winner knows its own key and row.  Common case: one redux on the high word
+// of the key and a ballot; the exact low-word compare and the smallest-row
+// rule run only when two candidates share the high word.
+__device__ __forceinline__ int warp_argmax_lane(bool cand, unsigned long long key, int row) {
+    const unsigned hi = cand ? (unsigned)(key >> 32) : 0u;
+    const unsigned mhi = __reduce_max_sync(FULL, hi);
+    const bool e1 = cand && hi == mhi;
+    unsigned wm = __ballot_sync(FULL, e1);
+    if (wm & (wm - 1)) {
+        const unsigned mlo = __reduce_max_sync(FULL, e1 ? (unsigned)key : 0u);
+        const bool e2 = e1 && (unsigned)key == mlo;
+        const unsigned r = __reduce_min_sync(FULL, e2 ? (unsigned)row : 0xffffffffu);
+        wm = __ballot_sync(FULL, e2 && (unsigned)row == r);
+    }
+    return wm ? __ffs(wm) - 1 : -1;
+}
+
+// 1/x for normal x whose reciprocal is normal, else 0 (the caller divides:
+// LAPACK divides below sfmin).  MUFU.RCP64H seed + one cubic Newton step:
+// error ~2^-66 before the final rounding, so the result is exact whenever
+// 1/x is representable (the dyadic test families) and within 1 ulp otherwise
+// (SURVEY Q6).  Cheap enough to run speculatively on every candidate, off the
+// pivot-search critical path.
+__device__ __forceinline__ double fast_rcp(double x) {
+    const double ax = fabs(x);
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+    const double e = fma(-x, r, 1.0);
+    r = fma(r, fma(e, e, e), r);
+    return (ax >= DBL_MIN && ax <= 0x1p1021) ? r : 0.0;
 }
 
 // Pivot scaling as LAPACK dgetf2: multiply by the reciprocal when

@@ -203,6 +203,65 @@ __device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni
     return true;
 }
 
+// Deferred left-block interchanges of the L1 kernel (a4.2).
+// The columns of panel q need, in order, the interchanges of every later
+// panel; no step of the factorization reads them again, so instead of moving
+// up to 2 ib scattered rows of the whole left block after every panel (one
+// 32-byte sector per 8-byte element) they are permuted once at the end.  With
+// g the gather map of the later panels' interchanges (column y = x[g]), panels
+// are processed right to left: g <- h_{q+1} o g, where h_{q+1} is the identity
+// with panel q+1's swaps applied in order, then the rows [j_{q+1}, m) of
+// panel q's columns are read (coalesced, cp.async) and written back permuted.
+__device__ __noinline__ void l1_left_swaps(double *__restrict__ gA, long ld, int mi, int K, int nb,
+                                           const int *__restrict__ gip, double *smd, int region_doubles) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    int *g = reinterpret_cast<int *>(smd);
+    int *h = g + L1_TALL_ROWS;
+    double *buf = smd + L1_TALL_ROWS;  // past the two int maps (2 x 1024 x 4 B)
+    const int cap = region_doubles - L1_TALL_ROWS;
+    for (int r = tid; r < mi; r += L1_NT) g[r] = r;
+    const int npan = (K + nb - 1) / nb;
+    for (int q = npan - 2; q >= 0; --q) {
+        const int js = (q + 1) * nb, ibn = imin(nb, K - js);
+        for (int r = js + tid; r < mi; r += L1_NT) h[r] = r;
+        __syncthreads();
+        if (tid == 0) {
+            for (int t = 0; t < ibn; ++t) {
+                const int p = gip[js + t] - 1;
+                if (p != js + t) {
+                    const int x = h[js + t];
+                    h[js + t] = h[p];
+                    h[p] = x;
+                }
+            }
+        }
+        __syncthreads();
+        for (int r = js + tid; r < mi; r += L1_NT) g[r] = h[g[r]];
+        __syncthreads();
+        const int rows = mi - js, c0 = q * nb;
+        int W = cap / rows;
+        W = W < 1 ? 1 : (W > nb ? nb : W);
+        for (int cb = 0; cb < nb; cb += W) {
+            const int w = imin(W, nb - cb);
+            for (int c = warp; c < w; c += L1_NT / 32) {
+                const double *gc = gA + js + (size_t)(c0 + cb + c) * ld;
+                for (int r = lane; r < rows; r += 32) cp_async8(buf + r + c * rows, gc + r);
+            }
+            cp_async_commit();
+            cp_async_wait<0>();
+            __syncthreads();
+            for (int c = warp; c < w; c += L1_NT / 32) {
+                double *gc = gA + js + (size_t)(c0 + cb + c) * ld;
+                for (int r = lane; r < rows; r += 32) {
+                    const int src = g[js + r] - js;
+                    if (src != r) gc[r] = buf[src + c * rows];
+                }
+            }
+            __syncthreads();
+        }
+    }
+}
+
 // ================================================================== L1
 // One CTA per matrix, all iterations inside (matrices with m <= L1 rows).
 // tall L1 panels (257..1024 rows)
@@ -223,7 +282,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                                                          const int *__restrict__ bins, int nb,
                                                          int l1_region_doubles, int phase_timing,
                                                          const int *__restrict__ order,
-                                                         const int *__restrict__ order_count) {
+                                                         const int *__restrict__ order_count, int defer) {
     extern __shared__ __align__(16) unsigned char l1_smem[];
     __shared__ PanelScratch sc;
     __shared__ __align__(16) PanelRegScratch<L1_NT / 32, 32> prs;
@@ -307,7 +366,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 0, (unsigned long long)(t1 - t0)); t0 = t1; }
             // ---- a4.2 + a4.3 interchanges left / right, U12 solve
-            if (j > 0 || c1 < ni) {
+            if ((j > 0 && !defer) || c1 < ni) {
                 double *top = smd;
                 double *bot = top + nb * (SW_COLS + 1);
                 if (!regs_panel) {  // panel_regs already emitted the plan
@@ -316,10 +375,13 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                 }
                 unsigned long long *phs = phase_timing ? ph : nullptr;
                 if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 1, (unsigned long long)(t1 - t0)); t0 = t1; }
-                // left block [0, j) and right block [c1, n) as one virtual range
-                const int vtot = j + (ni - c1);
+                // left block [0, j) (unless deferred) and right block [c1, n)
+                // as one virtual range
+                const int jl = defer ? 0 : j;
+                const int vtot = jl + (ni - c1);
                 for (int vb = 0; vb < vtot; vb += SW_COLS)
-                    swap_chunk(gA, ld, j, ib, vb, imin(SW_COLS, vtot - vb), j, ib, c1, sp, L11p, 0, top, bot, phs);
+                    swap_chunk(gA, ld, j, ib, vb, imin(SW_COLS, vtot - vb), jl, c1 - jl, c1, sp, L11p, 0, top, bot,
+                               phs);
             }
             if (phase_timing && tid == 0) t0 = clock64();  // chunk phases were accounted in slots 5..7
             // ---- a4.4 trailing update through the pipelined GEMM core
@@ -340,6 +402,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 2, (unsigned long long)(t1 - t0)); t0 = t1; }
         }
+        if (defer && K > nb) l1_left_swaps(gA, ld, mi, K, nb, gip, smd, l1_region_doubles);
         if (tid == 0) a.info[i] = info;
     }
 }
@@ -847,13 +910,13 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     // the tall-panel variant only when the bin can hold > 256 rows (it needs
     // more registers: the default variant keeps the lower spill count)
     const bool tall = tuning().l1_rows > L1_MAX_ROWS;
-    const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing;
-    if (tuning().l1_dmma) {  // measured: DFMA is faster inside L1 (DMMA variant spills)
-        if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
-        else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+    const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing, df = tuning().l1_defer;
+    if (tuning().l1_dmma) {  // default: DMMA (measured faster once the variant stopped spilling)
+        if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+        else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
     } else {
-        if (tall) lu_l1_kernel<false, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
-        else lu_l1_kernel<false, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count);
+        if (tall) lu_l1_kernel<false, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+        else lu_l1_kernel<false, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
     }
 }
 

@@ -3,164 +3,195 @@
 //
 // Prior work handled <= 32x32 matrices by caching in shared memory with
 // column-wise elimination; STRUMPACK's naive small kernel was
-// launch bound.  Here the whole GEPP of one matrix runs in one warp:
+// launch bound.  Here the whole GEPP of one matrix runs in one warp
+// and the matrix is read once and written once (HBM-bound, AI <= 1.33):
 //   * lane r holds row r in registers, SHIFTED so that a[0] is always the
 //     current pivot column: the rank-1 update and the shift are one FMA per
 //     register, a[c] <- a[c+1] - l * u[c+1], so every elimination step runs the
-//     same code (a loop, not a 32x32 unrolled triangle -- the unrolled form
-//     thrashed the instruction cache, ncu: 80% "no instruction" stalls);
-//   * the step width W shrinks 32 -> 16 -> 8 -> 4 as the active columns do;
-//   * pivot search: warp arg-max with the idamax tie rule (3 redux.sync);
-//     the interchange relabels lane positions, only the already-final L
-//     columns are swapped in shared memory (one lane per column);
-//   * the pivot row is broadcast through a 256-byte shared slot (STS.128 /
-//     LDS.128), U rows and L columns are written to the staged output as soon
-//     as they are final.
-// Loads are cp.async (the next matrix is in flight while the current one is
-// factored); stores are flat and fully coalesced.
+//     same code; the step width W shrinks 32 -> 16 -> 8 -> 4 with the active
+//     columns;
+//   * rows never move.  `pos` is the row's current position; an interchange
+//     is a relabelling (the winner lane takes position k, the row at k takes
+//     the winner's old position).  So nothing is swapped during the
+//     factorization: the multiplier a lane computes at step k goes to
+//     Lb[k][lane], the pivot row published at step k IS row k of U (Ub, rows
+//     packed by decreasing length), and at the end every lane writes its row
+//     once, at its final position -- for each column the warp's stores cover
+//     exactly that column, so they stay coalesced;
+//   * pivot search (idamax, ties -> smallest position): one
+//     redux.max on the high word of |a| + a ballot; only when two lanes share
+//     that high word does the full 64-bit compare + min-position run;
+//   * the next warp's matrix is prefetched into L2 while this one is factored.
+// Instruction count per matrix was the bound of the previous form (ncu: 2,625
+// warp instructions per matrix of C1big, IPC 1.6 at 12 warps/SM); this form
+// drops the per-step output bookkeeping and the smem input stage, and runs 16
+// warps per SM.
 #include "irr_internal.cuh"
 
 namespace irr {
 
 constexpr int S_WARPS = 4;
-constexpr int S_STAGE = 1024;  // doubles per stage buffer (32 x 32)
+constexpr int S_CTAS_PER_SM = 4;
+constexpr int S_UB = 544 + 32;  // packed U rows (capacities 32,32,30,30,..,2,2) + overflow pad
+
+struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 stores in every warp's slot
+    double L[32 * 32];  // L[k*32 + lane]: multiplier of the row held by `lane` at step k
+    double U[S_UB];     // row k of U (n-k values) at s_uoff(k)
+    double rcp;         // reciprocal of the pivot, published with the pivot row (0: divide)
+};
+static_assert(sizeof(SmallWarpSmem) % 16 == 0, "per-warp slots must stay 16-byte aligned");
+
+// offset of packed U row k; row k's capacity is 32 - (k & ~1) (even, so every
+// row starts 16-byte aligned for the pair stores)
+__device__ __forceinline__ int s_uoff(int k) {
+    const int t = k >> 1;
+    const int o = 2 * t * (33 - t);
+    return (k & 1) ? o + 32 - 2 * t : o;
+}
 
 template <int NC, int W>
-__device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, int m, int n,
-                                       int lane, double *__restrict__ st, double *__restrict__ prow) {
-    const bool valid = lane < m;
+__device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, bool valid,
+                                       int lane, SmallWarpSmem &sm) {
     const bool cand = valid && pos >= k;
-    unsigned long long key;
-    int pmin;
-    warp_argmax(cand, dkey(fabs(a[0])), pos, key, pmin);
-    const unsigned wmask = __ballot_sync(FULL, cand && pos == pmin);
-    const int w = __ffs(wmask) - 1;
-    if (lane == k) my_piv = pmin + 1;
+    // every lane's reciprocal of its own candidate, off the critical path of
+    // the pivot search; the winner publishes its one
+    const double myr = fast_rcp(a[0]);
+    // ---- arg-max of |a[0]| over the candidates
+    const unsigned long long key = (unsigned long long)__double_as_longlong(fabs(a[0]));
+    const unsigned hi = cand ? (unsigned)(key >> 32) : 0u;
+    const unsigned mhi = __reduce_max_sync(FULL, hi);
+    const bool e1 = cand && hi == mhi;
+    unsigned wm = __ballot_sync(FULL, e1);
+    if (wm & (wm - 1)) {  // several lanes share the high word (rare): exact compare, then smallest position
+        const unsigned mlo = __reduce_max_sync(FULL, e1 ? (unsigned)key : 0u);
+        const bool e2 = e1 && (unsigned)key == mlo;
+        const unsigned pm = __reduce_min_sync(FULL, e2 ? (unsigned)pos : 0xffffffffu);
+        wm = __ballot_sync(FULL, e2 && pos == (int)pm);
+    }
+    const int w = __ffs(wm) - 1;
+    const int pmin = __shfl_sync(FULL, pos, w);
+    // ---- the pivot row is row k of U: publish it where the output reads it
+    double *urow = sm.U + s_uoff(k);
     if (lane == w) {
 #pragma unroll
-        for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(prow + c) = make_double2(a[c], a[c + 1]);
+        for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
+        sm.rcp = myr;
     }
+    if (lane == k) my_piv = pmin + 1;
     __syncwarp();
-    const double pv = prow[0];
-    // interchange the final L columns (< k) of positions k and pmin
-    if (pmin != k && lane < k) {
-        const double x = st[k + lane * m], y = st[pmin + lane * m];
-        st[k + lane * m] = y;
-        st[pmin + lane * m] = x;
-    }
-    // U row k is final: columns k .. n-1 (n - k <= W <= 32)
-    if (lane < n - k) st[k + (k + lane) * m] = prow[lane];
+    const double pv = urow[0];
+    const double rc = sm.rcp;
+    // ---- interchange = relabel positions
     if (pos == k) pos = pmin;
     if (lane == w) pos = k;
     const bool below = valid && pos > k;
     double l = a[0];
     if (pv != 0.0) {
-        if (fabs(pv) >= DBL_MIN) l = l * (1.0 / pv);
-        else l = l / pv;
+        if (rc != 0.0) l = l * rc;
+        else l = l / pv;  // |pv| < DBL_MIN or 1/pv subnormal (LAPACK divides below sfmin)
     } else if (info == 0) {
-        info = k + 1;  // exact zero pivot: pmin == k (no interchange), no scaling
+        info = k + 1;  // exact zero pivot: every candidate is 0, pmin == k, no scaling
     }
-    if (below) st[pos + k * m] = l;
-    double u[W];
+    if (below) sm.L[k * 32 + lane] = l;
+    // ---- rank-1 update fused with the shift, u streamed in 16-byte loads
+    constexpr int CH = W < 4 ? W : 4;
 #pragma unroll
-    for (int c = 0; c < W; c += 2) {
-        const double2 v = *reinterpret_cast<const double2 *>(prow + c);
-        u[c] = v.x;
-        u[c + 1] = v.y;
+    for (int e0 = 0; e0 < W; e0 += CH) {
+        double uu[CH];
+#pragma unroll
+        for (int q = 0; q < CH; q += 2) {
+            const double2 v = *reinterpret_cast<const double2 *>(urow + e0 + q);
+            uu[q] = v.x;
+            uu[q + 1] = v.y;
+        }
+#pragma unroll
+        for (int q = 0; q < CH; ++q)
+            if (e0 + q >= 1) a[e0 + q - 1] = fma(-l, uu[q], a[e0 + q]);
     }
-#pragma unroll
-    for (int c = 0; c + 1 < W; ++c) a[c] = fma(-l, u[c + 1], a[c + 1]);
     a[W - 1] = 0.0;
-    __syncwarp();
+    // no trailing warp barrier: the next step's row k+1 starts past the n-k
+    // values of row k that are still read here, and rcp is read above
     ++k;
 }
 
 template <int NC>
 __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, int ld, int *__restrict__ gipiv,
-                                        int *__restrict__ ginfo, double *__restrict__ st,
-                                        double *__restrict__ prow, int lane) {
-    const int total = m * n;
+                                        int *__restrict__ ginfo, SmallWarpSmem &sm, int lane) {
+    const bool valid = lane < m;
     double a[NC];
+    const double *gr = gA + lane;
 #pragma unroll
-    for (int c = 0; c < NC; ++c) a[c] = (lane < m && c < n) ? st[lane + c * m] : 0.0;
-    __syncwarp();
+    for (int c = 0; c < NC; ++c) {
+        a[c] = (valid && c < n) ? *gr : 0.0;
+        gr += ld;
+    }
     int pos = lane, my_piv = 0, info = 0, k = 0;
     const int K = m < n ? m : n;
     if (NC >= 32)
-        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, m, n, lane, st, prow);
+        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
     if (NC >= 16)
-        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, m, n, lane, st, prow);
-    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, m, n, lane, st, prow);
-    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, m, n, lane, st, prow);
-    __syncwarp();
-    if (ld == m) {
-        for (int e = lane; e < total; e += 32) gA[e] = st[e];
-    } else {
-        for (int e = lane; e < total; e += 32) {
-            int c = e / m, r = e - c * m;
-            gA[r + (size_t)c * ld] = st[e];
+        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, sm);
+    __syncwarp();  // L / U rows from every lane are complete
+    // ---- write every row once, at its final position p: L(p, c) for c < p,
+    //      U(p, c) for c >= p (rows p >= K are pure L rows)
+    if (valid) {
+        double *go = gA + pos;
+        const double *ur = sm.U + s_uoff(pos < K ? pos : 0) - pos;
+        for (int c = 0; c < n; ++c) {
+            double v;
+            if (c < pos) v = sm.L[c * 32 + lane];
+            else v = ur[c];
+            go[(size_t)c * ld] = v;
         }
     }
     if (lane < K) gipiv[lane] = my_piv;
     if (lane == 0) *ginfo = info;
-    __syncwarp();  // the stage buffer is refilled by the next prefetch
+    __syncwarp();  // sm is rewritten by the next matrix
 }
 
-// Each warp walks its share of the tier-S list with a two-deep pipeline: the
-// next matrix is in flight (cp.async into the other stage buffer) while the
-// current one is factored.
-__global__ void __launch_bounds__(32 * S_WARPS) lu_small_kernel(GetrfArgs a, const int *__restrict__ counters,
-                                                                 const int *__restrict__ bins) {
+// Each warp walks its share of the tier-S list (static stride); the next
+// matrix of the warp is prefetched into L2 before the current one is loaded.
+__global__ void __launch_bounds__(32 * S_WARPS, S_CTAS_PER_SM) lu_small_kernel(GetrfArgs a,
+                                                                                const int *__restrict__ counters,
+                                                                                const int *__restrict__ bins) {
     extern __shared__ __align__(16) double s_small[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    double *stage0 = s_small + (size_t)warp * (2 * S_STAGE + 32);
-    double *prow = stage0 + 2 * S_STAGE;
+    SmallWarpSmem &sm = reinterpret_cast<SmallWarpSmem *>(s_small)[warp];
     const int count = counters[CNT_BIN0 + BIN_S];
     const int *list = bins + (size_t)BIN_S * a.batch;
     const int stride = gridDim.x * S_WARPS;
-    int t = blockIdx.x * S_WARPS + warp;
-    if (t >= count) return;
-    int i = list[t];
-    int m = a.m[i], n = a.n[i], ld = a.ld[i];
-    double *gA = a.A[i];
-    stage_block_async(stage0, m, gA, ld, m, n, lane, 32);
-    cp_async_commit();
-    int cur = 0;
-    while (true) {
+    for (int t = blockIdx.x * S_WARPS + warp; t < count; t += stride) {
+        const int i = list[t];
+        const int m = a.m[i], n = a.n[i], ld = a.ld[i];
+        double *gA = a.A[i];
         const int tn = t + stride;
-        int i2 = 0, m2 = 0, n2 = 0, ld2 = 0;
-        double *gA2 = nullptr;
         if (tn < count) {
-            i2 = list[tn];
-            m2 = a.m[i2]; n2 = a.n[i2]; ld2 = a.ld[i2];
-            gA2 = a.A[i2];
-            stage_block_async(stage0 + (cur ^ 1) * S_STAGE, m2, gA2, ld2, m2, n2, lane, 32);
+            const int i2 = list[tn];
+            const int m2 = a.m[i2], n2 = a.n[i2], ld2 = a.ld[i2];
+            const char *p2 = reinterpret_cast<const char *>(a.A[i2]);
+            const long bytes = ((long)(n2 - 1) * ld2 + m2) * 8;
+            for (long o = (long)lane * 128; o < bytes; o += 32 * 128)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + o));
         }
-        cp_async_commit();
-        cp_async_wait<1>();
-        __syncwarp();
-        double *st = stage0 + cur * S_STAGE;
         if (n <= 8)
-            lu_warp<8>(gA, m, n, ld, a.ipiv[i], a.info + i, st, prow, lane);
+            lu_warp<8>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
         else if (n <= 16)
-            lu_warp<16>(gA, m, n, ld, a.ipiv[i], a.info + i, st, prow, lane);
+            lu_warp<16>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
         else
-            lu_warp<32>(gA, m, n, ld, a.ipiv[i], a.info + i, st, prow, lane);
-        if (tn >= count) break;
-        t = tn; i = i2; m = m2; n = n2; ld = ld2; gA = gA2;
-        cur ^= 1;
+            lu_warp<32>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
     }
-    cp_async_wait<0>();
 }
 
 void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
-    const size_t smem = (size_t)S_WARPS * (2 * S_STAGE + 32) * sizeof(double);
+    const size_t smem = (size_t)S_WARPS * sizeof(SmallWarpSmem);
     static size_t attr = 0;
     if (smem > attr) {
         cudaFuncSetAttribute(lu_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
-    int grid = num_sms() * 3;  // 3 x 66 KB per SM: 12 warps / SM, 2 matrices in flight per warp
+    int grid = num_sms() * S_CTAS_PER_SM;  // 4 x 51 KB per SM: 16 warps / SM
     int need = (a.batch + S_WARPS - 1) / S_WARPS;
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;

@@ -60,6 +60,7 @@ template <int NW, int NBP>
 struct PanelRegScratch {
     double row[2][NW][NBP];  // first: 16-byte aligned for the pair stores; row[.][w][0] = signed candidate
     unsigned long long key[2][NW];
+    double rcp[2][NW];
     int pos[2][NW];
 };
 
@@ -82,10 +83,16 @@ __device__ __forceinline__ void preg_step(double (&a)[RPT][NBP], int (&pos)[RPT]
             if (bq < 0 || k > bk || (k == bk && pos[q] < bp)) { bk = k; bp = pos[q]; bq = q; }
         }
     }
-    unsigned long long wk;
-    int wp;
-    warp_argmax(bq >= 0, bk, bp, wk, wp);
-    const unsigned wm = __ballot_sync(FULL, bq >= 0 && bp == wp);
+    // speculative reciprocal of this thread's candidate (published by the winner)
+    double cv = a[0][0];
+#pragma unroll
+    for (int q = 1; q < RPT; ++q)
+        if (bq == q) cv = a[q][0];
+    const double myr = fast_rcp(cv);
+    const int wl = warp_argmax_lane(bq >= 0, bk, bp);
+    const unsigned long long wk = bk;  // the winner's own key / position
+    const int wp = bp;
+    const unsigned wm = wl < 0 ? 0u : (1u << wl);
     PT(0)
     if (wm == 0) {
         if (lane == 0) sc.pos[par][warp] = -1;
@@ -93,6 +100,7 @@ __device__ __forceinline__ void preg_step(double (&a)[RPT][NBP], int (&pos)[RPT]
         // publish the candidate row with the partial (no selects: one branch per row slot)
         sc.key[par][warp] = wk;
         sc.pos[par][warp] = wp;
+        sc.rcp[par][warp] = myr;
         double *dst = sc.row[par][warp];
 #pragma unroll
         for (int q = 0; q < RPT; ++q) {
@@ -137,8 +145,7 @@ __device__ __forceinline__ void preg_step(double (&a)[RPT][NBP], int (&pos)[RPT]
         else if (pos[q] == pmin) pos[q] = c;
     }
     if (pv == 0.0 && zero_at == 0) zero_at = c + 1;  // no interchange (pmin == c), no scaling
-    const bool use_rcp = fabs(pv) >= DBL_MIN;
-    const double rcp = (pv != 0.0 && use_rcp) ? 1.0 / pv : 0.0;
+    const double rcp = sc.rcp[par][wbest];  // 0: divide (|pv| < sfmin or 1/pv subnormal)
     PT(4)
     // ---- scale + rank-1 update + shift of my rows below position c
     double lq[RPT];
@@ -147,7 +154,7 @@ __device__ __forceinline__ void preg_step(double (&a)[RPT][NBP], int (&pos)[RPT]
     for (int q = 0; q < RPT; ++q) {
         act[q] = (tid + NT * q < rows) && pos[q] > c;
         double l = a[q][0];
-        if (pv != 0.0) l = use_rcp ? l * rcp : l / pv;
+        if (pv != 0.0) l = (rcp != 0.0) ? l * rcp : l / pv;
         lq[q] = l;
     }
     // a[e-1] <- a[e] - l u[e], e ascending; u streamed in 16-byte loads,

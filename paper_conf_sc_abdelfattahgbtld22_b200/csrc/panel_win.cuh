@@ -28,6 +28,7 @@ struct PanelWinSmem {
     double Ds[NBX * (NBX + 1)];  // L of the rows pushed below the panel block (end)
     double row[2][NW][PW_WBMAX];  // published candidate rows (double-buffered)
     unsigned long long key[2][NW];
+    double rcp[2][NW];
     int pos[2][NW], orig[2][NW];
     int srcpos[NBX];  // original row now at pivot position p
     SwapPlan plan;
@@ -51,15 +52,22 @@ __device__ __forceinline__ void pwin_step(double (&a)[RPT][WB], int (&pos)[RPT],
             if (bq < 0 || k > bk || (k == bk && pos[q] < bp)) { bk = k; bp = pos[q]; bq = q; }
         }
     }
-    unsigned long long wk;
-    int wp;
-    warp_argmax(bq >= 0, bk, bp, wk, wp);
-    const unsigned wm = __ballot_sync(FULL, bq >= 0 && bp == wp);
+    // speculative reciprocal of this thread's candidate (published by the winner)
+    double cv = a[0][0];
+#pragma unroll
+    for (int q = 1; q < RPT; ++q)
+        if (bq == q) cv = a[q][0];
+    const double myr = fast_rcp(cv);
+    const int wl = warp_argmax_lane(bq >= 0, bk, bp);
+    const unsigned long long wk = bk;  // the winner's own key / position
+    const int wp = bp;
+    const unsigned wm = wl < 0 ? 0u : (1u << wl);
     if (wm == 0) {
         if (lane == 0) sm.pos[par][warp] = -1;
     } else if (lane == __ffs(wm) - 1) {
         sm.key[par][warp] = wk;
         sm.pos[par][warp] = wp;
+        sm.rcp[par][warp] = myr;
         sm.orig[par][warp] = tid + NT * bq;
         double *dst = sm.row[par][warp];
 #pragma unroll
@@ -97,15 +105,14 @@ __device__ __forceinline__ void pwin_step(double (&a)[RPT][WB], int (&pos)[RPT],
         else if (pos[q] == pmin) pos[q] = c;
     }
     if (pv == 0.0 && zero_at == 0) zero_at = c + 1;  // no interchange (pmin == c), no scaling
-    const bool use_rcp = fabs(pv) >= DBL_MIN;
-    const double rcp = (pv != 0.0 && use_rcp) ? 1.0 / pv : 0.0;
+    const double rcp = sm.rcp[par][wbest];  // 0: divide (|pv| < sfmin or 1/pv subnormal)
     double lq[RPT];
     bool act[RPT];
 #pragma unroll
     for (int q = 0; q < RPT; ++q) {
         act[q] = (tid + NT * q < rows) && pos[q] > c;
         double l = a[q][0];
-        if (pv != 0.0) l = use_rcp ? l * rcp : l / pv;
+        if (pv != 0.0) l = (rcp != 0.0) ? l * rcp : l / pv;
         lq[q] = l;
     }
     constexpr int CH = W < 8 ? W : 8;

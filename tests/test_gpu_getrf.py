@@ -240,3 +240,51 @@ def test_grid_panel_variants_agree(win):
     irr.irr_set_tuning("l1", 0)
     irr.irr_set_tuning("panel_win", win)
     _run_and_check(_uniform([(800, 800), (300, 1000), (1000, 300)], seed=5))
+
+
+def test_device_generator_matches_host():
+    """irrgen.device (C5's on-device inputs) writes the same bytes as the host
+    generator, for ld == m and ld > m, keyed by global id."""
+    from irrgen import device as gdev
+    rng = np.random.default_rng(3)
+    m = rng.integers(0, 70, size=300)
+    n = rng.integers(0, 70, size=300)
+    ld = np.maximum(1, m) + rng.integers(0, 3, size=300) * (rng.random(300) < 0.3)
+    gids = rng.permutation(10_000)[:300]
+    off, total = irrgen.packed_offsets(ld, n)
+    host = np.full(total, 7.0)
+    irrgen.fill_packed(99, m, n, ld, off, host, gids=gids)
+    dev = torch.full((total,), 7.0, dtype=torch.float64, device="cuda")
+    gdev.Filler(99, m, n, ld, off, gids, dev.device).fill(dev)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy().view(np.uint64), host.view(np.uint64))
+
+
+@pytest.mark.parametrize("defer", [1, 0])
+def test_l1_deferred_left_interchanges(defer):
+    """L1 with the left-block interchanges applied once at the end (default)
+    and eagerly after every panel: both match the oracle, and agree bitwise
+    (the interchanges only move values)."""
+    irr.irr_set_tuning("l1_defer", defer)
+    shapes = [(256, 256), (200, 240), (256, 70), (180, 256), (129, 200), (250, 33)]
+    mats = _uniform(shapes, seed=41)
+    _run_and_check(mats)
+    irr.irr_set_tuning("l1_defer", 1 - defer)
+    other, ip_o, _, _ = gpu_getrf(mats)
+    irr.irr_set_tuning("l1_defer", defer)
+    mine, ip_m, _, _ = gpu_getrf(mats)
+    for a, b, p, q in zip(mine, other, ip_m, ip_o):
+        assert np.array_equal(a, b) and np.array_equal(p, q)
+
+
+def test_c5_sample_parity():
+    """configs[4] shapes (fronts 1..2048, heavy tail, full DGETRF): a
+    stratified sample -- the largest fronts plus a random slice."""
+    cfg = irrgen.config("C5")
+    nf = cfg.m
+    big = np.argsort(-nf)[:1]
+    rest = np.random.default_rng(5).choice(len(nf), 40, replace=False)
+    sel = np.unique(np.concatenate([big, rest]))
+    mats = [irrgen.uniform_values(cfg.seed, int(g), int(cfg.m[g]), int(cfg.n[g])) for g in sel]
+    st = _run_and_check(mats)
+    assert st.get("match", 0) >= len(mats) - 2
