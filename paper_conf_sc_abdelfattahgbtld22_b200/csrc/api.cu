@@ -304,7 +304,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
     else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
-    else if (!strcmp(key, "l1_defer")) g_tuning.l1_defer = value ? 1 : 0;
+    else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -326,7 +326,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
     if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
-    if (!strcmp(key, "l1_defer")) return g_tuning.l1_defer;
+    if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) return g_tuning.defer;
     return -1;
 }
 

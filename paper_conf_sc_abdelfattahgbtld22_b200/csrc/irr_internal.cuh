@@ -31,7 +31,7 @@ struct Tuning {
     int l1_rowmap;       // 1: L1 kernel in row-map form (no interchanges until one final permutation)
     int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
     int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
-    int l1_defer;        // 1: L1 applies the left-block interchanges once at the end (coalesced)
+    int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)
 };
 Tuning &tuning();
 
@@ -80,7 +80,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }

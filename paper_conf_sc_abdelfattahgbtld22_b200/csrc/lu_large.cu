@@ -212,18 +212,16 @@ __device__ __forceinline__ bool trailing_desc(double *A, long ld, int mi, int ni
 // are processed right to left: g <- h_{q+1} o g, where h_{q+1} is the identity
 // with panel q+1's swaps applied in order, then the rows [j_{q+1}, m) of
 // panel q's columns are read (coalesced, cp.async) and written back permuted.
-__device__ __noinline__ void l1_left_swaps(double *__restrict__ gA, long ld, int mi, int K, int nb,
-                                           const int *__restrict__ gip, double *smd, int region_doubles) {
+template <int NT>
+__device__ __forceinline__ void left_swaps_core(double *__restrict__ gA, long ld, int mi, int K, int nb,
+                                                const int *__restrict__ gip, int *g, int *h, double *buf,
+                                                int cap) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    int *g = reinterpret_cast<int *>(smd);
-    int *h = g + L1_TALL_ROWS;
-    double *buf = smd + L1_TALL_ROWS;  // past the two int maps (2 x 1024 x 4 B)
-    const int cap = region_doubles - L1_TALL_ROWS;
-    for (int r = tid; r < mi; r += L1_NT) g[r] = r;
+    for (int r = tid; r < mi; r += NT) g[r] = r;
     const int npan = (K + nb - 1) / nb;
     for (int q = npan - 2; q >= 0; --q) {
         const int js = (q + 1) * nb, ibn = imin(nb, K - js);
-        for (int r = js + tid; r < mi; r += L1_NT) h[r] = r;
+        for (int r = js + tid; r < mi; r += NT) h[r] = r;
         __syncthreads();
         if (tid == 0) {
             for (int t = 0; t < ibn; ++t) {
@@ -236,30 +234,38 @@ __device__ __noinline__ void l1_left_swaps(double *__restrict__ gA, long ld, int
             }
         }
         __syncthreads();
-        for (int r = js + tid; r < mi; r += L1_NT) g[r] = h[g[r]];
+        for (int r = js + tid; r < mi; r += NT) g[r] = h[g[r]];
         __syncthreads();
         const int rows = mi - js, c0 = q * nb;
         int W = cap / rows;
         W = W < 1 ? 1 : (W > nb ? nb : W);
         for (int cb = 0; cb < nb; cb += W) {
             const int w = imin(W, nb - cb);
-            for (int c = warp; c < w; c += L1_NT / 32) {
+            for (int c = warp; c < w; c += NT / 32) {
                 const double *gc = gA + js + (size_t)(c0 + cb + c) * ld;
-                for (int r = lane; r < rows; r += 32) cp_async8(buf + r + c * rows, gc + r);
+                for (int r = lane; r < rows; r += 32) cp_async8(buf + r + (size_t)c * rows, gc + r);
             }
             cp_async_commit();
             cp_async_wait<0>();
             __syncthreads();
-            for (int c = warp; c < w; c += L1_NT / 32) {
+            for (int c = warp; c < w; c += NT / 32) {
                 double *gc = gA + js + (size_t)(c0 + cb + c) * ld;
                 for (int r = lane; r < rows; r += 32) {
                     const int src = g[js + r] - js;
-                    if (src != r) gc[r] = buf[src + c * rows];
+                    if (src != r) gc[r] = buf[src + (size_t)c * rows];
                 }
             }
             __syncthreads();
         }
     }
+}
+
+__device__ __noinline__ void l1_left_swaps(double *__restrict__ gA, long ld, int mi, int K, int nb,
+                                           const int *__restrict__ gip, double *smd, int region_doubles) {
+    int *g = reinterpret_cast<int *>(smd);
+    // past the two int maps (2 x 1024 x 4 B)
+    left_swaps_core<L1_NT>(gA, ld, mi, K, nb, gip, g, g + L1_TALL_ROWS, smd + L1_TALL_ROWS,
+                           region_doubles - L1_TALL_ROWS);
 }
 
 // ================================================================== L1
@@ -701,7 +707,7 @@ template <bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                         const int *__restrict__ bins,
                                                         const SwapPlan *__restrict__ plans, int *queue, int j,
-                                                        int nb, int chunks_per, unsigned long long *ph) {
+                                                        int nb, int chunks_per, unsigned long long *ph, int defer) {
     extern __shared__ __align__(16) double st_smem[];
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
@@ -735,7 +741,10 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         if (j >= K) continue;
         const int ib = K - j < nb ? K - j : nb;
         const int c1 = j + ib;
-        const int vtot = ni - ib, vb = q * ST_COLS;
+        // virtual columns: the left block [0, jl) (empty when its interchanges
+        // are deferred to left_swaps_kernel) then the right block [c1, n)
+        const int jl = defer ? 0 : j;
+        const int vtot = jl + ni - c1, vb = q * ST_COLS;
         if (vb >= vtot) continue;
         double *gA = a.A[i];
         if (slot != last_slot) {
@@ -749,10 +758,10 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         __syncthreads();
         ST_PHASE(0)
         const int W = imin(ST_COLS, vtot - vb);
-        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, j, ib, c1, sp, L11, ldl, top, bot, ph);
+        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, jl, c1 - jl, c1, sp, L11, ldl, top, bot, ph);
         if (ph && tid == 0) t0 = clock64();
         // trailing GEMM on the strip's right-of-panel columns
-        const int cbeg = (vb > j ? vb : j) + ib, cend = vb + W + ib;
+        const int cbeg = (vb > jl ? vb : jl) + (c1 - jl), cend = vb + W + (c1 - jl);
         if (cbeg < cend && c1 < mi) {
             GemmDesc d0;
             d0.A = gA + c1 + (size_t)j * ld; d0.lda = ld; d0.ta = 0;
@@ -776,6 +785,33 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         }
     }
 #undef ST_PHASE
+}
+
+// The deferred left-block interchanges of the grid-wide tier: one CTA per
+// tier-L matrix (dynamic queue), after the last panel (left_swaps_core).
+constexpr int LSW_NT = 256;
+constexpr int LSW_BUF = 6144;  // doubles of column buffer (48 KB)
+__global__ void __launch_bounds__(LSW_NT) left_swaps_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                            const int *__restrict__ bins, int nb, int maps,
+                                                            int *queue) {
+    extern __shared__ __align__(16) double lsw_smem[];
+    __shared__ int item_s;
+    double *buf = lsw_smem;
+    int *g = reinterpret_cast<int *>(lsw_smem + LSW_BUF);
+    int *h = g + maps;
+    const int count = counters[CNT_BIN0 + BIN_L];
+    const int *list = bins + (size_t)BIN_L * a.batch;
+    for (;;) {
+        if (threadIdx.x == 0) item_s = atomicAdd(queue, 1);
+        __syncthreads();
+        const int t = item_s;
+        __syncthreads();
+        if (t >= count) break;
+        const int i = list[t];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        if (K > nb) left_swaps_core<LSW_NT>(a.A[i], a.ld[i], mi, K, nb, a.ipiv[i], g, h, buf, LSW_BUF);
+    }
 }
 
 static size_t strip_smem_bytes(int nb) {
@@ -910,7 +946,7 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     // the tall-panel variant only when the bin can hold > 256 rows (it needs
     // more registers: the default variant keeps the lower spill count)
     const bool tall = tuning().l1_rows > L1_MAX_ROWS;
-    const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing, df = tuning().l1_defer;
+    const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing, df = tuning().defer;
     if (tuning().l1_dmma) {  // default: DMMA (measured faster once the variant stopped spilling)
         if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
         else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
@@ -971,6 +1007,16 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
             st_attr[tu.dmma ? 1 : 0] = st_smem;
         }
     }
+    // deferred left-block interchanges (strip path only): one pass at the end
+    const size_t lsw_smem = (size_t)LSW_BUF * sizeof(double) + 2 * (size_t)a.max_m * sizeof(int);
+    const bool defer = fused && tu.defer && lsw_smem <= 200 * 1024;
+    if (defer) {
+        static size_t lsw_attr = 0;
+        if (lsw_smem > 48 * 1024 && lsw_smem > lsw_attr) {
+            cudaFuncSetAttribute(left_swaps_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsw_smem);
+            lsw_attr = lsw_smem;
+        }
+    }
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {
             KScope k(K_PANEL, s);
@@ -982,9 +1028,11 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         if (fused) {
             KScope k(K_STRIP, s);
             if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
-                                                                             counters + CNT_STRIPQ, j, nb, st_chunks, ph);
+                                                                             counters + CNT_STRIPQ, j, nb, st_chunks, ph,
+                                                                             defer);
             else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
-                                                                      counters + CNT_STRIPQ, j, nb, st_chunks, ph);
+                                                                      counters + CNT_STRIPQ, j, nb, st_chunks, ph,
+                                                                      defer);
             continue;
         }
         {
@@ -1008,6 +1056,13 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                     P, -1, counters + CNT_BIN0 + BIN_L, tile_off);
             }
         }
+    }
+    if (defer && Kmax > nb) {
+        cudaMemsetAsync(counters + CNT_LSWQ, 0, sizeof(int), s);
+        KScope k(K_SWAP_TRSM, s);
+        int grid = sms * 2;
+        if (grid > a.batch) grid = a.batch;
+        left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, nb, a.max_m, counters + CNT_LSWQ);
     }
 }
 

@@ -261,17 +261,22 @@ def test_device_generator_matches_host():
 
 
 @pytest.mark.parametrize("defer", [1, 0])
-def test_l1_deferred_left_interchanges(defer):
-    """L1 with the left-block interchanges applied once at the end (default)
-    and eagerly after every panel: both match the oracle, and agree bitwise
-    (the interchanges only move values)."""
-    irr.irr_set_tuning("l1_defer", defer)
+@pytest.mark.parametrize("l1", [1, 0])
+def test_deferred_left_interchanges(defer, l1):
+    """Left-block interchanges applied once at the end (default) and eagerly
+    after every panel, in the CTA-per-matrix tier (l1=1) and the grid-wide
+    tier (l1=0): both match the oracle and agree bitwise (interchanges only
+    move values)."""
+    irr.irr_set_tuning("l1", l1)
+    irr.irr_set_tuning("defer", defer)
     shapes = [(256, 256), (200, 240), (256, 70), (180, 256), (129, 200), (250, 33)]
+    if not l1:
+        shapes += [(700, 700), (1100, 300), (300, 900), (2000, 96)]
     mats = _uniform(shapes, seed=41)
     _run_and_check(mats)
-    irr.irr_set_tuning("l1_defer", 1 - defer)
+    irr.irr_set_tuning("defer", 1 - defer)
     other, ip_o, _, _ = gpu_getrf(mats)
-    irr.irr_set_tuning("l1_defer", defer)
+    irr.irr_set_tuning("defer", defer)
     mine, ip_m, _, _ = gpu_getrf(mats)
     for a, b, p, q in zip(mine, other, ip_m, ip_o):
         assert np.array_equal(a, b) and np.array_equal(p, q)
