@@ -165,6 +165,31 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
               const int *kcount, int *const *ipiv, int batch, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_getrs -- batched solve with the factors of irr_getrf (SURVEY §8(f)
+ * NEXT 1; the GETRS composition the paper benchmarks irrTRSM against, P:L96,
+ * L215, and the solve step of P:L77-79):
+ *      X_i <- A_i^-1 B_i = U_i^-1 L_i^-1 P_i^T B_i
+ *  trans        IRR_NO_TRANS only (IRR_TRANS -> IRR_ERR_UNSUPPORTED).
+ *  n, nrhs      int[batch]: A_i is n[i] x n[i] holding L\U and ipiv[i] as
+ *               irr_getrf left them; B_i is n[i] x nrhs[i] (column-major,
+ *               leading dimension ldb[i] >= max(1, n[i])), overwritten by X_i.
+ *               max_n / max_nrhs (host) bound them (<= 0: computed, one sync).
+ *  A, lda, ipiv, B, ldb   device pointer / int arrays as for irr_getrf.
+ *  info         int[batch] (output): 0, or -(argument position) for a bad
+ *               n (-5), nrhs (-6), NULL A_i (-7), lda (-8), NULL ipiv_i (-9),
+ *               NULL B_i (-10) or ldb (-11); those systems are skipped.  No
+ *               singularity check (LAPACK dgetrs): a zero U_ii gives IEEE
+ *               inf / NaN in X_i.
+ *  work         >= irr_getrs_workspace_size(batch) bytes (caller-owned).
+ * Host errors: -1 trans, -2 batch, -(position) for NULL arrays, as above.
+ * Asynchronous on `stream` when max_n and max_nrhs are given.
+ * ---------------------------------------------------------------------- */
+size_t irr_getrs_workspace_size(int batch);
+int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
+              const double *const *A, const int *lda, int *const *ipiv, double *const *B, const int *ldb,
+              int *info, void *work, size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * Tuning (tests and experiments; defaults are fixed by measurement and are
  * process-global, not thread-safe).  Keys: "nb" (tier-L panel width, 1..64),
  * "tier_s" (1 = enable the warp-per-matrix tier), "tier_m_max" (max padded

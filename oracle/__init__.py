@@ -50,6 +50,8 @@ def lib():
                                   dp, C.c_int, C.c_double, dp, C.c_int]
         L.oracle_trsm.argtypes = [C.c_int] * 6 + [C.c_double, dp, C.c_int, dp, C.c_int]
         L.oracle_laswp.argtypes = [C.c_int, dp, C.c_int, C.c_int, C.c_int, ip]
+        L.oracle_getrs.argtypes = [C.c_int, C.c_int, dp, C.c_int, ip, dp, C.c_int]
+        L.oracle_getrs.restype = C.c_int
         L.oracle_backward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
         L.oracle_backward_error.restype = C.c_double
         L.oracle_num_threads.restype = C.c_int
@@ -183,6 +185,22 @@ def laswp(A, k1, k2, ipiv):
     buf = A if A.size else np.zeros((1, 1), order="F")
     lib().oracle_laswp(A.shape[1], _dp(buf), max(1, A.shape[0]), int(k1), int(k2), _ip(ipiv))
     return A
+
+
+def getrs(LU, ipiv, B):
+    """X = A^-1 B from the factors of getrf (LU n x n, 1-based ipiv), on a copy of B."""
+    LU, B = _fortran(LU), _fortran(B)
+    n = LU.shape[0]
+    nrhs = B.shape[1]
+    ipiv = np.ascontiguousarray(ipiv, dtype=np.int32)
+    if ipiv.size == 0:
+        ipiv = np.zeros(1, dtype=np.int32)
+    b0 = LU if LU.size else np.zeros((1, 1), order="F")
+    b1 = B if B.size else np.zeros((1, 1), order="F")
+    r = lib().oracle_getrs(n, nrhs, _dp(b0), max(1, n), _ip(ipiv), _dp(b1), max(1, n))
+    if r < 0:
+        raise ValueError(f"oracle_getrs: bad argument {-r}")
+    return B
 
 
 def backward_error(A0, LU, ipiv):

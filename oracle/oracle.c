@@ -24,6 +24,8 @@
  *  - oracle_gemm / oracle_trsm / oracle_laswp: the building blocks of
  *    §IV-C (L171-173), §IV-D (L175-182) and §IV-F (L188-195) as their plain
  *    BLAS/LAPACK definitions.
+ *  - oracle_getrs: the solve with the factors (LAPACK dgetrs steps), the
+ *    GETRS composition the paper benchmarks irrTRSM against (L96, L215).
  *  - oracle_backward_error: ||PA - LU||_F / (||A||_F * k * eps) (north_star;
  *    SURVEY reading Q11), accumulated in long double.
  */
@@ -295,6 +297,45 @@ void oracle_laswp(int n, double *A, int lda, int k1, int k2, const int *ipiv)
                 A[p + (size_t)j * lda] = t;
             }
     }
+}
+
+/* ---------------------------------------------------------------------------
+ * GETRS with the factors of oracle_getrf (the paper's
+ * GETRS = LASWP + TRSM(L, unit) + TRSM(U)): B <- U^-1 L^-1 P^T B
+ * for an n x n L\U and n x nrhs B, as the plain steps of LAPACK dgetrs:
+ *   1. apply the swaps k = 0..n-1 in order to the rows of B;
+ *   2. forward substitution with the unit L: row i -= sum_{j<i} l_ij row j;
+ *   3. back substitution with U: row i = (row i - sum_{j>i} u_ij row j) / u_ii.
+ * Returns 0, or -(argument position) for a bad n / nrhs / ld.
+ * ------------------------------------------------------------------------- */
+int oracle_getrs(int n, int nrhs, const double *LU, int ld, const int *ipiv, double *B, int ldb)
+{
+    if (n < 0) return -1;
+    if (nrhs < 0) return -2;
+    if (ld < imax(1, n)) return -4;
+    if (ldb < imax(1, n)) return -7;
+#define LU_(i, j) LU[(size_t)(i) + (size_t)(j) * ld]
+#define B_(i, j) B[(size_t)(i) + (size_t)(j) * ldb]
+    for (int k = 0; k < n; ++k) {
+        int p = ipiv[k] - 1;
+        if (p != k)
+            for (int c = 0; c < nrhs; ++c) { double t = B_(k, c); B_(k, c) = B_(p, c); B_(p, c) = t; }
+    }
+    for (int c = 0; c < nrhs; ++c) {
+        for (int i = 0; i < n; ++i) {
+            double s = 0.0;
+            for (int j = 0; j < i; ++j) s = s + LU_(i, j) * B_(j, c);
+            B_(i, c) = B_(i, c) - s;
+        }
+        for (int i = n - 1; i >= 0; --i) {
+            double s = 0.0;
+            for (int j = i + 1; j < n; ++j) s = s + LU_(i, j) * B_(j, c);
+            B_(i, c) = (B_(i, c) - s) / LU_(i, i);
+        }
+    }
+#undef LU_
+#undef B_
+    return 0;
 }
 
 /* ||PA - LU||_F / (||A||_F * max(1, min(m,n)) * eps)  (north_star).

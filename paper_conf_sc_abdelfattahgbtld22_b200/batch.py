@@ -83,6 +83,20 @@ class MatrixBatch:
                              self.ipiv, self.info, self.workspace(), stream)
 
 
+    def getrs(self, rhs: "MatrixBatch", info=None, stream=None):
+        """irr_getrs: rhs.data[i] <- A_i^-1 rhs_i with this batch's factors
+        (square matrices; rhs.m must equal this batch's n).  Returns the
+        per-system argument status (int32 device tensor)."""
+        if info is None:
+            info = torch.zeros(max(1, self.batch), dtype=torch.int32, device=self.device)
+        nb = irr.irr_getrs_workspace_size(self.batch)
+        work = torch.empty(max(256, nb), dtype=torch.uint8, device=self.device)
+        irr.irr_getrs(irr.IRR_NO_TRANS, self.batch, self.max_n, rhs.max_n, self.n, rhs.n, self.ptr, self.ld,
+                      self.ipiv, rhs.ptr, rhs.ld, info, work, stream)
+        self._getrs_keep = work
+        return info
+
+
 class FrontBatch:
     """Fronts F = [F11 F12; F21 F22], one nf x nf block each (ld = nf)."""
 

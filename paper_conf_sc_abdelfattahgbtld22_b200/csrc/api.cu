@@ -428,6 +428,64 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 
+// Step a5.2 of the partial front on its own: X <- U^-1 L^-1 P^T B with the
+// factors of irr_getrf (the fused strip kernel, or irrLASWP + 2 x irrTRSM).
+static void getrs_core(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs, const double *const *A,
+                       const int *lda, int *const *ipiv, double *const *B, const int *ldb, const int *mask,
+                       const Work &w, cudaStream_t s) {
+    // systems sorted by n (descending buckets): every building-block call
+    // visits only the systems that still have work at its offset
+    launch_size_sort(n, batch, w.sort, s);
+    if (tuning().getrs_fused && getrs_strip_ok(max_n)) {
+        launch_getrs_strip(batch, n, nrhs, A, lda, B, ldb, ipiv, mask, w.tile_off, w.counters + CNT_GSQ,
+                           sorted_slots(w.sort, batch, 0), s);
+        return;
+    }
+    launch_laswp_masked(max_nrhs, nrhs, B, 0, 0, ldb, 0, max_n, n, ipiv, batch, mask, s, w.tile_off,
+                        sorted_slots(w.sort, batch, 0));
+    TrsmArgs t{};
+    t.side = IRR_LEFT; t.uplo = IRR_LOWER; t.trans = IRR_NO_TRANS; t.diag = IRR_UNIT;
+    t.max_m = max_n; t.max_n = max_nrhs; t.m = n; t.n = nrhs; t.alpha = 1.0;
+    t.T = A; t.Ti = 0; t.Tj = 0; t.ldt = lda;
+    t.B = B; t.Bi = 0; t.Bj = 0; t.ldb = ldb; t.batch = batch;
+    run_trsm_masked(t, mask, w.counters, w.tile_off, s, w.sort);
+    t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
+    run_trsm_masked(t, mask, w.counters, w.tile_off, s, w.sort);
+}
+
+size_t irr_getrs_workspace_size(int batch) { return work_bytes_getrf(batch); }
+
+int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
+              const double *const *A, const int *lda, int *const *ipiv, double *const *B, const int *ldb,
+              int *info, void *work, size_t work_bytes, irr_stream_t stream) {
+    if (trans != IRR_NO_TRANS && trans != IRR_TRANS) return -1;
+    if (batch < 0) return -2;
+    if (trans == IRR_TRANS) return IRR_ERR_UNSUPPORTED;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!n) return -5;
+    if (!nrhs) return -6;
+    if (!A) return -7;
+    if (!lda) return -8;
+    if (!ipiv) return -9;
+    if (!B) return -10;
+    if (!ldb) return -11;
+    if (!info) return -12;
+    if (!work) return -13;
+    if (work_bytes < work_bytes_getrf(batch)) return IRR_ERR_WORKSPACE;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    Work w = carve(work, batch);
+    rc = resolve_max_dims(batch, max_n, max_nrhs, n, nrhs, w.counters, s);
+    if (rc) return rc;
+    if (max_n > 0 && laswp_smem(max_n) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
+    launch_getrs_validate(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, s);
+    if (max_n <= 0 || max_nrhs <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+    IRR_CUDA_TRY(cudaMemsetAsync(w.counters, 0, CNT_INTS * sizeof(int), s));
+    getrs_core(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, w, s);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
 size_t irr_gemm_workspace_size(int batch) { return work_bytes_for(batch); }
 
 int irr_gemm(irr_trans_t ta, irr_trans_t tb, int max_m, int max_n, int max_k, const int *m, const int *n,

@@ -44,7 +44,7 @@ constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
 // Issue the cp.async copies of K chunk [k0, k0+16) of tile (r0, c0) into buffer
 // `buf` (out-of-range elements are zero-filled with plain stores).
-template <bool MAP = false>
+template <bool MAP = false, bool BRES = false>
 __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int c0, int k0, GemmSmem &sm, int buf) {
     const int tid = threadIdx.x;
     if (MAP) {
@@ -84,6 +84,7 @@ __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int 
             *dst = 0.0;
         }
     }
+    if (BRES) return;  // B already resident in sm.Bs (the caller staged all K rows)
 #pragma unroll
     for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
@@ -113,7 +114,9 @@ __device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, 
 
 // ---- DFMA path: thread (tx, ty) owns rows tx + 8q (q < 8), cols ty + 16p (p < 4);
 //      acc[q * 4 + p].  12 shared-memory wavefronts per 32 DFMA per warp.
-__device__ __forceinline__ void gemm_compute_chunk_dfma(const GemmSmem &sm, int buf, double (&acc)[32]) {
+__device__ __forceinline__ void gemm_compute_chunk_dfma(const GemmSmem &sm, int buf, double (&acc)[32],
+                                                        int bbuf = -1) {
+    if (bbuf < 0) bbuf = buf;
     const int tid = threadIdx.x, tx = tid & 7, ty = tid >> 3;
 #pragma unroll
     for (int kk = 0; kk < GBK; ++kk) {
@@ -121,7 +124,7 @@ __device__ __forceinline__ void gemm_compute_chunk_dfma(const GemmSmem &sm, int 
 #pragma unroll
         for (int q = 0; q < 8; ++q) a[q] = sm.As[buf][kk][tx + 8 * q];
 #pragma unroll
-        for (int p = 0; p < 4; ++p) b[p] = sm.Bs[buf][kk][ty + 16 * p];
+        for (int p = 0; p < 4; ++p) b[p] = sm.Bs[bbuf][kk][ty + 16 * p];
 #pragma unroll
         for (int q = 0; q < 8; ++q)
 #pragma unroll
@@ -140,7 +143,9 @@ __device__ __forceinline__ void dmma_8x8x4(double &c0, double &c1, double a, dou
                  : "d"(a), "d"(b));
 }
 
-__device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int buf, double (&acc)[32]) {
+__device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int buf, double (&acc)[32],
+                                                        int bbuf = -1) {
+    if (bbuf < 0) bbuf = buf;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int g = lane >> 2, t = lane & 3;
     const int rb = (warp & 1) * 32 + g, cb = (warp >> 1) * 32 + g;
@@ -150,12 +155,58 @@ __device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int 
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi) a[mi] = sm.As[buf][ks + t][rb + 8 * mi];
 #pragma unroll
-        for (int ni = 0; ni < 4; ++ni) b[ni] = sm.Bs[buf][ks + t][cb + 8 * ni];
+        for (int ni = 0; ni < 4; ++ni) b[ni] = sm.Bs[bbuf][ks + t][cb + 8 * ni];
 #pragma unroll
         for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
             for (int ni = 0; ni < 4; ++ni)
                 dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], a[mi], b[ni]);
+    }
+}
+
+// DMMA path without a shared-memory C stage: this lane's 32 C values go
+// straight from global memory into registers, issued at the start of the tile
+// and consumed by the epilogue (ncu, strip kernel on C3: the epilogue's wait
+// on the staged C tile was the largest stall, 16%).  Measured SLOWER on B200
+// (C3 strip 57.8 -> 60.4 ms, C2 6.44 -> 6.54 ms), so off by default (CREG_OK).
+__device__ __forceinline__ void gemm_load_c_regs(const GemmDesc &d, int r0, int c0, double (&cr)[32]) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+    const bool rd = d.beta != 0.0;
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+        const int r = r0 + (warp & 1) * 32 + 8 * mi + g;
+#pragma unroll
+        for (int ni = 0; ni < 4; ++ni) {
+#pragma unroll
+            for (int i = 0; i < 2; ++i) {
+                const int c = c0 + (warp >> 1) * 32 + 8 * ni + 2 * t + i;
+                cr[(mi * 4 + ni) * 2 + i] = (rd && r < d.m && c < d.n) ? d.C[r + (size_t)c * d.ldc] : 0.0;
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ void gemm_epilogue_creg(const GemmDesc &d, int r0, int c0, const double (&acc)[32],
+                                                   const double (&cr)[32]) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane >> 2, t = lane & 3;
+#pragma unroll
+    for (int mi = 0; mi < 4; ++mi) {
+        const int r = r0 + (warp & 1) * 32 + 8 * mi + g;
+        if (r >= d.m) continue;
+#pragma unroll
+        for (int ni = 0; ni < 4; ++ni) {
+#pragma unroll
+            for (int i = 0; i < 2; ++i) {
+                const int c = c0 + (warp >> 1) * 32 + 8 * ni + 2 * t + i;
+                if (c >= d.n) continue;
+                const int q = (mi * 4 + ni) * 2 + i;
+                double v = d.alpha * acc[q];
+                if (d.beta != 0.0) v = fma(d.beta, cr[q], v);
+                d.C[r + (size_t)c * d.ldc] = v;
+            }
+        }
     }
 }
 
@@ -205,17 +256,23 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
 // A stream of tiles processed by one CTA with the software pipeline described
 // above.  `next(d, r0, c0)` returns false when the CTA has no more tiles.
 // DMMA selects the FP64 tensor-core path, else DFMA.
-template <bool DMMA, class Next, bool MAP = false>
+// BRES: op(B) (k <= 2 GBK rows) is resident in sm.Bs for every tile of the
+// stream -- chunk c reads Bs[c] -- and is never loaded (the strip kernel's
+// U12, solved in place there).
+template <bool DMMA, class Next, bool MAP = false, bool CREG_OK = false, bool BRES = false>
 __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     GemmDesc d, dn;
     int r0, c0, rn, cn;
     if (!next(d, r0, c0)) return;
     int buf = 0;
-    if (d.k > 0) gemm_issue_chunk<MAP>(d, r0, c0, 0, sm, buf);
+    if (d.k > 0) gemm_issue_chunk<MAP, BRES>(d, r0, c0, 0, sm, buf);
     cp_async_commit();
     bool have = true;
+    constexpr bool CREG = DMMA && !MAP && CREG_OK;  // C in registers (the commit below is then an empty group)
     while (have) {
-        gemm_issue_c<MAP>(d, r0, c0, sm);
+        double cr[32];
+        if (CREG) gemm_load_c_regs(d, r0, c0, cr);
+        else gemm_issue_c<MAP>(d, r0, c0, sm);
         cp_async_commit();
         double acc[32];
 #pragma unroll
@@ -224,25 +281,29 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         bool has_next_tile = false;
         for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
             if (c + 1 < nchunks) {
-                gemm_issue_chunk<MAP>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
+                gemm_issue_chunk<MAP, BRES>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
             } else {
                 has_next_tile = next(dn, rn, cn);
-                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP>(dn, rn, cn, 0, sm, buf ^ 1);
+                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP, BRES>(dn, rn, cn, 0, sm, buf ^ 1);
             }
             cp_async_commit();
             if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();
             __syncthreads();
             if (nchunks > 0) {
-                if (DMMA) gemm_compute_chunk_dmma(sm, buf, acc);
-                else gemm_compute_chunk_dfma(sm, buf, acc);
+                if (DMMA) gemm_compute_chunk_dmma(sm, buf, acc, BRES ? c : buf);
+                else gemm_compute_chunk_dfma(sm, buf, acc, BRES ? c : buf);
             }
             __syncthreads();
             buf ^= 1;
         }
-        cp_async_wait<1>();
-        __syncthreads();
-        gemm_epilogue<DMMA, MAP>(d, r0, c0, sm, acc);
-        __syncthreads();
+        if (CREG) {
+            gemm_epilogue_creg(d, r0, c0, acc, cr);
+        } else {
+            cp_async_wait<1>();
+            __syncthreads();
+            gemm_epilogue<DMMA, MAP>(d, r0, c0, sm, acc);
+            __syncthreads();
+        }
         have = has_next_tile;
         if (have) { d = dn; r0 = rn; c0 = cn; }
     }
@@ -261,6 +322,12 @@ __device__ __forceinline__ int gemm_tile_weight(const GemmDesc &d) { return 1 + 
 
 // count: number of problem slots, from *count_ptr when count < 0.
 // tile_off[b] = weighted work before slot b (gemm_tile_weight units).
+// C fragments in registers for the DMMA epilogue (gemm_load_c_regs) where the
+// problem's descriptor code leaves the register room (the DCWI descriptor
+// spills with it); specialised next to the problem types that opt in.
+template <class Prob>
+struct gemm_creg_ok { static constexpr bool value = false; };
+
 template <class Prob>
 __global__ void __launch_bounds__(1024) gemm_scan_kernel(Prob P, int count, const int *count_ptr, int *tile_off) {
     __shared__ int warp_sums[32];
@@ -346,7 +413,7 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, 
         ++local;
         return true;
     };
-    gemm_tile_stream<DMMA>(next, sm);
+    gemm_tile_stream<DMMA, decltype(next), false, gemm_creg_ok<Prob>::value>(next, sm);
 }
 
 // DCWI-grid fallback (no workspace): virtual tiles over the required dims,

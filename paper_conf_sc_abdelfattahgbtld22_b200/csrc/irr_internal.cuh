@@ -67,7 +67,7 @@ struct KScope {
 // L = blocked right-looking LU with one kernel chain per panel iteration.
 // L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
 // kernels per panel iteration.
-enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, NBINS = 6 };
+enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, BIN_S16 = 6, BIN_S8 = 7, NBINS = 8 };
 constexpr int L1_MAX_ROWS = 256;    // panels up to this many rows are staged in shared memory
 constexpr int L1_TALL_ROWS = 1024;  // taller L1 panels: panel_win in global memory (128 threads x 8 rows)
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
@@ -255,6 +255,10 @@ void launch_partial_validate(int batch, int max_n1, int max_n2, const int *n1, c
                              const int *ld11, const int *ld12, const int *ld21, const int *ld22,
                              double *const *F11, double *const *F12, const double *const *F21,
                              double *const *F22, int *const *ipiv, int *info, cudaStream_t s);
+
+void launch_getrs_validate(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
+                           const double *const *A, const int *lda, int *const *ipiv, double *const *B,
+                           const int *ldb, int *info, cudaStream_t s);
 
 int num_sms();
 }  // namespace irr

@@ -711,9 +711,14 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
     extern __shared__ __align__(16) double st_smem[];
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
-    double *L11 = st_smem;
-    double *top = L11 + nb * ldl;
-    double *bot = top + nb * (ST_COLS + 1);
+    // nb <= 32: the solved U12 rows (top) ARE the GEMM's resident B operand
+    // (gsm.Bs: 2 x 16 rows of GPAD = ST_COLS + 1), and L11 / bot sit in the C
+    // stage (dead during the interchange + TRSM, filled only by the GEMM
+    // tiles afterwards); else the original layout
+    const bool bres = DMMA && nb <= 2 * GBK;
+    double *top = bres ? &gsm.Bs[0][0][0] : st_smem + nb * ldl;
+    double *L11 = bres ? &gsm.Cs[0][0] : st_smem;
+    double *bot = bres ? L11 + nb * ldl : top + nb * (ST_COLS + 1);
     __shared__ SwapPlan sp;
     __shared__ int item_s;
     const int tid = threadIdx.x;
@@ -779,7 +784,16 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
                 ++tt;
                 return true;
             };
-            gemm_tile_stream<DMMA>(next, gsm);
+            if (bres && vb >= jl) {  // the GEMM's columns start at top's column 0
+                // B rows >= ib of the resident operand must be zero (A is
+                // zero-filled there, but stale shared memory may hold NaNs)
+                if (ib < 2 * GBK)
+                    for (int e = tid; e < (2 * GBK - ib) * (ST_COLS + 1); e += G_NT) top[ib * (ST_COLS + 1) + e] = 0.0;
+                __syncthreads();
+                gemm_tile_stream<DMMA, decltype(next), false, false, true>(next, gsm);
+            } else {
+                gemm_tile_stream<DMMA>(next, gsm);
+            }
             __syncthreads();
             ST_PHASE(2)
         }
@@ -871,6 +885,9 @@ struct TrailingProb {
         return trailing_desc(a.A[i], a.ld[i], a.m[i], a.n[i], j, nb, d);
     }
 };
+template <>
+struct gemm_creg_ok<TrailingProb> { static constexpr bool value = false; };  // measured: staged C is faster
+
 
 static int clamp_nb(int nb) { return nb < 1 ? 1 : (nb > NBMAX ? NBMAX : nb); }
 

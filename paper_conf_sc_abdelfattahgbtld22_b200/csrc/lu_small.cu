@@ -31,27 +31,42 @@
 namespace irr {
 
 constexpr int S_WARPS = 4;
-constexpr int S_CTAS_PER_SM = 4;
-constexpr int S_UB = 544 + 32;  // packed U rows (capacities 32,32,30,30,..,2,2) + overflow pad
 
-struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 stores in every warp's slot
-    double L[32 * 32];  // L[k*32 + lane]: multiplier of the row held by `lane` at step k
-    double U[S_UB];     // row k of U (n-k values) at s_uoff(k)
-    double rcp;         // reciprocal of the pivot, published with the pivot row (0: divide)
-};
-static_assert(sizeof(SmallWarpSmem) % 16 == 0, "per-warp slots must stay 16-byte aligned");
+// Width classes n <= 8 / 16 / 32 are separate bins and separate kernels
+// (classify.cu), so the narrow ones run at their own register and
+// shared-memory budgets: more resident warps to hide the per-step latency
+// chain (redux -> ballot -> shfl -> publish -> LDS -> DMUL -> DFMA).
+template <int NC>
+struct SmallCfg;
+template <>
+struct SmallCfg<32> { static constexpr int ctas = 4, bin = BIN_S; };    // 128 regs, 16 warps / SM
+template <>
+struct SmallCfg<16> { static constexpr int ctas = 6, bin = BIN_S16; };  // 80 regs, 24 warps / SM
+template <>
+struct SmallCfg<8> { static constexpr int ctas = 8, bin = BIN_S8; };    // 64 regs, 32 warps / SM
 
-// offset of packed U row k; row k's capacity is 32 - (k & ~1) (even, so every
+// offset of packed U row k; row k's capacity is NC - (k & ~1) (even, so every
 // row starts 16-byte aligned for the pair stores)
-__device__ __forceinline__ int s_uoff(int k) {
-    const int t = k >> 1;
-    const int o = 2 * t * (33 - t);
-    return (k & 1) ? o + 32 - 2 * t : o;
+template <int NC>
+__host__ __device__ constexpr int s_uoff(int k) {
+    return (k & 1) ? 2 * (k >> 1) * (NC + 1 - (k >> 1)) + NC - 2 * (k >> 1)
+                   : 2 * (k >> 1) * (NC + 1 - (k >> 1));
 }
+
+template <int NC>
+struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 stores in every warp's slot
+    double L[NC * 32];             // L[k*32 + lane]: multiplier of the row held by `lane` at step k
+    double U[s_uoff<NC>(NC) + NC];  // row k of U (n-k values) at s_uoff(k), + overflow pad
+    double rcp[2];                 // reciprocal of the pivot, published with the pivot row (0: divide)
+};
+static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<16>) % 16 == 0 &&
+                  sizeof(SmallWarpSmem<8>) % 16 == 0,
+              "per-warp slots must stay 16-byte aligned");
+static_assert(s_uoff<32>(32) == 544 && s_uoff<32>(3) == 94, "packed U offsets");
 
 template <int NC, int W>
 __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, bool valid,
-                                       int lane, SmallWarpSmem &sm) {
+                                       int lane, SmallWarpSmem<NC> &sm) {
     const bool cand = valid && pos >= k;
     // every lane's reciprocal of its own candidate, off the critical path of
     // the pivot search; the winner publishes its one
@@ -71,16 +86,16 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
     const int w = __ffs(wm) - 1;
     const int pmin = __shfl_sync(FULL, pos, w);
     // ---- the pivot row is row k of U: publish it where the output reads it
-    double *urow = sm.U + s_uoff(k);
+    double *urow = sm.U + s_uoff<NC>(k);
     if (lane == w) {
 #pragma unroll
         for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
-        sm.rcp = myr;
+        sm.rcp[0] = myr;
     }
     if (lane == k) my_piv = pmin + 1;
     __syncwarp();
     const double pv = urow[0];
-    const double rc = sm.rcp;
+    const double rc = sm.rcp[0];
     // ---- interchange = relabel positions
     if (pos == k) pos = pmin;
     if (lane == w) pos = k;
@@ -116,7 +131,7 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
 
 template <int NC>
 __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, int ld, int *__restrict__ gipiv,
-                                        int *__restrict__ ginfo, SmallWarpSmem &sm, int lane) {
+                                        int *__restrict__ ginfo, SmallWarpSmem<NC> &sm, int lane) {
     const bool valid = lane < m;
     double a[NC];
     const double *gr = gA + lane;
@@ -138,7 +153,7 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     //      U(p, c) for c >= p (rows p >= K are pure L rows)
     if (valid) {
         double *go = gA + pos;
-        const double *ur = sm.U + s_uoff(pos < K ? pos : 0) - pos;
+        const double *ur = sm.U + s_uoff<NC>(pos < K ? pos : 0) - pos;
         for (int c = 0; c < n; ++c) {
             double v;
             if (c < pos) v = sm.L[c * 32 + lane];
@@ -151,16 +166,18 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     __syncwarp();  // sm is rewritten by the next matrix
 }
 
-// Each warp walks its share of the tier-S list (static stride); the next
-// matrix of the warp is prefetched into L2 before the current one is loaded.
-__global__ void __launch_bounds__(32 * S_WARPS, S_CTAS_PER_SM) lu_small_kernel(GetrfArgs a,
-                                                                                const int *__restrict__ counters,
-                                                                                const int *__restrict__ bins) {
+// Each warp walks its share of the width class's list (static stride); the
+// next matrix of the warp is prefetched into L2 before the current one is
+// loaded.
+template <int NC>
+__global__ void __launch_bounds__(32 * S_WARPS, SmallCfg<NC>::ctas) lu_small_kernel(GetrfArgs a,
+                                                                                    const int *__restrict__ counters,
+                                                                                    const int *__restrict__ bins) {
     extern __shared__ __align__(16) double s_small[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    SmallWarpSmem &sm = reinterpret_cast<SmallWarpSmem *>(s_small)[warp];
-    const int count = counters[CNT_BIN0 + BIN_S];
-    const int *list = bins + (size_t)BIN_S * a.batch;
+    SmallWarpSmem<NC> &sm = reinterpret_cast<SmallWarpSmem<NC> *>(s_small)[warp];
+    const int count = counters[CNT_BIN0 + SmallCfg<NC>::bin];
+    const int *list = bins + (size_t)SmallCfg<NC>::bin * a.batch;
     const int stride = gridDim.x * S_WARPS;
     for (int t = blockIdx.x * S_WARPS + warp; t < count; t += stride) {
         const int i = list[t];
@@ -175,28 +192,34 @@ __global__ void __launch_bounds__(32 * S_WARPS, S_CTAS_PER_SM) lu_small_kernel(G
             for (long o = (long)lane * 128; o < bytes; o += 32 * 128)
                 asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + o));
         }
-        if (n <= 8)
-            lu_warp<8>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
-        else if (n <= 16)
-            lu_warp<16>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
-        else
-            lu_warp<32>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
+        lu_warp<NC>(gA, m, n, ld, a.ipiv[i], a.info + i, sm, lane);
     }
 }
 
-void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
-    const size_t smem = (size_t)S_WARPS * sizeof(SmallWarpSmem);
+template <int NC>
+static void launch_class(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
+    const size_t smem = (size_t)S_WARPS * sizeof(SmallWarpSmem<NC>);
     static size_t attr = 0;
     if (smem > attr) {
-        cudaFuncSetAttribute(lu_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaFuncSetAttribute(lu_small_kernel<NC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         attr = smem;
     }
-    int grid = num_sms() * S_CTAS_PER_SM;  // 4 x 51 KB per SM: 16 warps / SM
+    int grid = num_sms() * SmallCfg<NC>::ctas;
     int need = (a.batch + S_WARPS - 1) / S_WARPS;
     if (grid > need) grid = need;
     if (grid < 1) grid = 1;
     KScope k(K_LU_SMALL, s);
-    lu_small_kernel<<<grid, 32 * S_WARPS, smem, s>>>(a, counters, bins);
+    lu_small_kernel<NC><<<grid, 32 * S_WARPS, smem, s>>>(a, counters, bins);
+}
+
+// widest class first: it has the most work per matrix, the narrow kernels
+// fill in behind it
+void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
+    launch_class<32>(a, counters, bins, s);
+    if (a.max_n > 0) {
+        launch_class<16>(a, counters, bins, s);
+        launch_class<8>(a, counters, bins, s);
+    }
 }
 
 }  // namespace irr

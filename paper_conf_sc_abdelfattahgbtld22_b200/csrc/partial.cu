@@ -36,4 +36,30 @@ void launch_partial_validate(int batch, int max_n1, int max_n2, const int *n1, c
                                                                ld22, F11, F12, F21, F22, ipiv, info);
 }
 
+// irr_getrs argument check (LAPACK positions of the irr_getrs call)
+__global__ void getrs_validate_kernel(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
+                                      const double *const *A, const int *lda, int *const *ipiv,
+                                      double *const *B, const int *ldb, int *info) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= batch) return;
+    const int a = n[i], b = nrhs[i];
+    int e = 0;
+    if (a < 0 || a > max_n) e = -5;
+    else if (b < 0 || b > max_nrhs) e = -6;
+    else if (a > 0 && A[i] == nullptr) e = -7;
+    else if (lda[i] < (a > 1 ? a : 1)) e = -8;
+    else if (a > 0 && ipiv[i] == nullptr) e = -9;
+    else if (a > 0 && b > 0 && B[i] == nullptr) e = -10;
+    else if (ldb[i] < (a > 1 ? a : 1)) e = -11;
+    info[i] = e;
+}
+
+void launch_getrs_validate(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
+                           const double *const *A, const int *lda, int *const *ipiv, double *const *B,
+                           const int *ldb, int *info, cudaStream_t s) {
+    KScope k(K_MISC, s);
+    getrs_validate_kernel<<<(batch + 255) / 256, 256, 0, s>>>(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B,
+                                                             ldb, info);
+}
+
 }  // namespace irr

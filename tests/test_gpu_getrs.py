@@ -1,0 +1,119 @@
+"""GPU parity of irr_getrs (the solve with the factors,
+the GETRS composition of P:L96, L215) through the C ABI against the oracle's
+plain dgetrs steps, on the GPU's own factors (so the comparison isolates the
+solve), plus the residual of A X = B and the exact dyadic family."""
+import numpy as np
+import pytest
+
+import irrgen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("no CUDA device", allow_module_level=True)
+
+from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
+from paper_conf_sc_abdelfattahgbtld22_b200.batch import MatrixBatch  # noqa: E402
+
+EPS = np.finfo(np.float64).eps
+
+
+@pytest.fixture(autouse=True)
+def _reset_tuning():
+    irr.irr_reset_tuning()
+    yield
+    irr.irr_reset_tuning()
+
+
+def _load(B, mats):
+    host = np.zeros(B.total)
+    for i, M in enumerate(mats):
+        if M.size:
+            B.matrix(i, host)[:, :] = M
+    B.data.copy_(torch.from_numpy(host))
+
+
+def _solve(As, Bs, fused=1):
+    irr.irr_set_tuning("getrs_fused", fused)
+    n = [A.shape[0] for A in As]
+    nrhs = [X.shape[1] for X in Bs]
+    FA = MatrixBatch(n, n)
+    RB = MatrixBatch(n, nrhs)
+    _load(FA, As)
+    _load(RB, Bs)
+    FA.getrf()
+    st = FA.getrs(RB)
+    torch.cuda.synchronize()
+    fa, ip, rb = FA.data.cpu().numpy(), FA.ipiv_data.cpu().numpy(), RB.data.cpu().numpy()
+    LUs = [np.array(FA.matrix(i, fa)) for i in range(FA.batch)]
+    ipivs = [np.array(FA.ipiv_of(i, ip)) for i in range(FA.batch)]
+    Xs = [np.array(RB.matrix(i, rb)) for i in range(RB.batch)]
+    return LUs, ipivs, Xs, st.cpu().numpy()[: FA.batch]
+
+
+@pytest.mark.parametrize("fused", [1, 0])
+def test_getrs_matches_oracle_mixed_sizes(fused):
+    """Every tier of the factorization and both solve paths (fused strip
+    kernel / irrLASWP + 2 x irrTRSM), ragged n and nrhs, nrhs = 0 and n = 0."""
+    rng = np.random.default_rng(17)
+    shapes = [(0, 3), (1, 1), (5, 0), (7, 3), (32, 32), (33, 1), (100, 17), (128, 200), (257, 64), (300, 5),
+              (600, 40)] + [(int(a), int(b)) for a, b in zip(rng.integers(1, 200, 20), rng.integers(1, 90, 20))]
+    As = [irrgen.uniform_values(5, g, n, n) for g, (n, _) in enumerate(shapes)]
+    Bs = [irrgen.uniform_values(6, g, n, r) for g, (n, r) in enumerate(shapes)]
+    LUs, ipivs, Xs, st = _solve(As, Bs, fused)
+    assert (st == 0).all()
+    for (n, r), A, B, LU, ip, X in zip(shapes, As, Bs, LUs, ipivs, Xs):
+        if n == 0 or r == 0:
+            continue
+        Xo = oracle.getrs(LU, ip, B)
+        dev = np.abs(X - Xo).max() / max(1e-300, np.abs(Xo).max())
+        assert dev <= 1e-10, f"{n}x{r}: deviation {dev}"
+        res = np.abs(A @ X - B).max() / (np.abs(A).max() * np.abs(X).max() * n * EPS)
+        assert res <= 10.0, f"{n}x{r}: residual {res}"
+
+
+def test_getrs_exact_dyadic():
+    """G1 factors with power-of-two pivots and integer X: X is recovered bit-exactly."""
+    shapes = [(6, 2), (40, 9), (64, 64), (150, 3)]
+    As, Xt = [], []
+    for g, (n, r) in enumerate(shapes):
+        A = irrgen.g1_exact(9, 500 + g, n, n)[0]
+        X = np.asfortranarray(np.random.default_rng(g).integers(-8, 9, size=(n, r)).astype(np.float64))
+        As.append(A)
+        Xt.append(X)
+    Bs = [np.asfortranarray(A @ X) for A, X in zip(As, Xt)]
+    _, _, Xs, st = _solve(As, Bs)
+    assert (st == 0).all()
+    for X, Xg in zip(Xt, Xs):
+        assert np.array_equal(X, Xg)
+
+
+def test_getrs_bad_arguments_are_skipped():
+    """ldb < n is reported per system (-11) and that system is untouched."""
+    n = [8, 8]
+    FA = MatrixBatch(n, n)
+    RB = MatrixBatch([8, 8], [2, 2], ld=[8, 8])
+    _load(FA, [irrgen.uniform_values(1, g, 8, 8) for g in range(2)])
+    B0 = [irrgen.uniform_values(2, g, 8, 2) for g in range(2)]
+    _load(RB, B0)
+    FA.getrf()
+    RB.ld = torch.tensor([8, 3], dtype=torch.int32, device=RB.device)
+    st = FA.getrs(RB).cpu().numpy()
+    torch.cuda.synchronize()
+    assert st[0] == 0 and st[1] == -11
+    rb = RB.data.cpu().numpy()
+    assert np.array_equal(np.array(RB.matrix(1, rb)), B0[1])
+
+
+def test_getrs_host_argument_errors():
+    FA = MatrixBatch([4], [4])
+    work = torch.empty(irr.irr_getrs_workspace_size(1), dtype=torch.uint8, device="cuda")
+    info = torch.zeros(1, dtype=torch.int32, device="cuda")
+    rc = irr.irr_getrs(irr.IRR_TRANS, 1, 4, 1, FA.n, FA.n, FA.ptr, FA.ld, FA.ipiv, FA.ptr, FA.ld, info, work,
+                       check=False)
+    assert rc == irr.IRR_ERR_UNSUPPORTED
+    rc = irr.irr_getrs(irr.IRR_NO_TRANS, -1, 4, 1, FA.n, FA.n, FA.ptr, FA.ld, FA.ipiv, FA.ptr, FA.ld, info, work,
+                       check=False)
+    assert rc == -2

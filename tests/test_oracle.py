@@ -387,3 +387,43 @@ def test_flops_formula():
     assert flops.getrf_flops(1, 1) == 1.0
     # partial: getrf(n1) + two triangular solves n1^2 n2 each + Schur GEMM 2 n1 n2^2
     assert flops.partial_flops(3, 2) == pytest.approx(count_gepp_ops(3, 3) + 2 * 9 * 2 + 2 * 3 * 4)
+
+
+# ---------------------------------------------------------------- GETRS pins
+def test_getrs_hand_2x2(orc):
+    """A = [[1, 2], [3, 4]]: GEPP swaps rows (ipiv = [2, 2]), L = [[1,0],[1/3,1]],
+    U = [[3, 4], [0, 2/3]]; A x = [5, 11] has x = [1, 2] (worked by hand)."""
+    A = np.array([[1.0, 2.0], [3.0, 4.0]], order="F")
+    LU, ipiv, info, _ = orc.getrf(A)
+    assert list(ipiv) == [2, 2] and info == 0
+    X = orc.getrs(LU, ipiv, np.array([[5.0], [11.0]], order="F"))
+    assert np.abs(X[:, 0] - [1.0, 2.0]).max() <= 4 * EPS
+
+
+@pytest.mark.parametrize("n,nrhs", [(1, 1), (5, 3), (17, 1), (40, 9), (64, 64)])
+def test_getrs_exact_dyadic(orc, n, nrhs):
+    """G1: A = P L U from dyadic factors with power-of-two pivots, X dyadic,
+    B = A X formed exactly (integers scaled by powers of two) -> GETRS returns X
+    bit-exactly (every step of the solve is exact on this family)."""
+    A, L, U, ipiv, info = irrgen.g1_exact(9, n + 13 * nrhs, n, n)
+    rng = np.random.default_rng(n * 100 + nrhs)
+    X = np.asfortranarray(rng.integers(-8, 9, size=(n, nrhs)).astype(np.float64))
+    B = np.asfortranarray(A @ X)
+    LU, oipiv, _, _ = orc.getrf(A)
+    assert np.array_equal(oipiv, ipiv)
+    got = orc.getrs(LU, oipiv, B)
+    assert np.array_equal(got, X)
+
+
+@pytest.mark.parametrize("n,nrhs", [(3, 2), (33, 5), (100, 17)])
+def test_getrs_vs_lapack(orc, n, nrhs):
+    """Cross-check against LAPACK dgetrs (scipy lu_solve on the oracle's own
+    factors): same factors in, same solution out to rounding."""
+    A = irrgen.uniform_values(12, n, n, n)
+    B = irrgen.uniform_values(13, n, n, nrhs)
+    LU, ipiv, _, _ = orc.getrf(A)
+    got = orc.getrs(LU, ipiv, B)
+    ref = sl.lu_solve((LU, ipiv - 1), B)
+    assert np.abs(got - ref).max() <= 1e-9 * max(1.0, np.abs(ref).max())
+    res = np.abs(A @ got - B).max() / (np.abs(A).max() * np.abs(got).max() * n * EPS)
+    assert res <= 10.0
