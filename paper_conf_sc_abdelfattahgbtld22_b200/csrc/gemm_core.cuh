@@ -35,10 +35,12 @@ struct GemmDesc {
     const int *rmap = nullptr, *kmap = nullptr;
 };
 
+constexpr int CPAD = GBM + 2;  // even: 16-byte row pairs of the C stage stay aligned (cp.async16)
+
 struct GemmSmem {
     double As[2][GBK][GPAD];
     double Bs[2][GBK][GPAD];
-    double Cs[GBN][GPAD];
+    double Cs[GBN][CPAD];
 };
 constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
@@ -106,6 +108,24 @@ __device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, 
     if (d.beta == 0.0) return;
     const int tid = threadIdx.x;
     const int mr = imin(GBM, d.m - r0), nc = imin(GBN, d.n - c0);
+    if (!MAP) {
+        // row pair (2p, 2p+1) per thread: one 16-byte copy where the column's
+        // pair is 16-byte aligned in global memory (parity of r0 + c ldc), else two
+        const int p2 = 2 * (tid & 31);
+        if (p2 >= mr) return;
+        const bool two = p2 + 1 < mr;
+        for (int c = tid >> 5; c < nc; c += G_NT / 32) {
+            const double *src = d.C + r0 + p2 + (size_t)(c0 + c) * d.ldc;
+            double *dst = &sm.Cs[c][p2];
+            if (two && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+                cp_async16(dst, src);
+            } else {
+                cp_async8(dst, src);
+                if (two) cp_async8(dst + 1, src + 1);
+            }
+        }
+        return;
+    }
     const int r = tid & 63;  // fixed per thread (G_NT = 2 x 64)
     if (r >= mr) return;
     const double *cr = d.C + (MAP ? d.rmap[r0 + r] : r0 + r);
@@ -134,9 +154,11 @@ __device__ __forceinline__ void gemm_compute_chunk_dfma(const GemmSmem &sm, int 
 
 // ---- DMMA path (FP64 tensor core, mma.sync m8n8k4 -> SASS DMMA.8x8x4):
 //      warp w computes the 32x32 sub-tile (rows 32 (w&1), cols 32 (w>>1)) as
-//      4 x 4 mma tiles; lane (g = lane>>2, t = lane&3) holds A(g, t), B(t, g)
-//      and C(g, 2t + i).  acc[(mi * 4 + ni) * 2 + i].  One DMMA = 256 FMA, so
-//      the operand traffic is two 8-byte loads per lane per 16 DMMA.
+//      4 x 4 mma tiles; lane (g = lane>>2, t = lane&3) loads A(g, t) and B(t, g)
+//      and the mma runs TRANSPOSED (C^T = B^T A^T: B's fragment as the row
+//      operand), so acc[(mi * 4 + ni) * 2 + i] = C(8 mi + 2t + i, 8 ni + g):
+//      two adjacent rows of one column, i.e. one 16-byte global access in the
+//      column-major C.  One DMMA = 256 FMA; two 8-byte loads per lane per 16 DMMA.
 __device__ __forceinline__ void dmma_8x8x4(double &c0, double &c1, double a, double b) {
     asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
                  : "+d"(c0), "+d"(c1)
@@ -160,7 +182,7 @@ __device__ __forceinline__ void gemm_compute_chunk_dmma(const GemmSmem &sm, int 
         for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
             for (int ni = 0; ni < 4; ++ni)
-                dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], a[mi], b[ni]);
+                dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], b[ni], a[mi]);
     }
 }
 
@@ -175,12 +197,12 @@ __device__ __forceinline__ void gemm_load_c_regs(const GemmDesc &d, int r0, int 
     const bool rd = d.beta != 0.0;
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi) {
-        const int r = r0 + (warp & 1) * 32 + 8 * mi + g;
 #pragma unroll
         for (int ni = 0; ni < 4; ++ni) {
+            const int c = c0 + (warp >> 1) * 32 + 8 * ni + g;
 #pragma unroll
             for (int i = 0; i < 2; ++i) {
-                const int c = c0 + (warp >> 1) * 32 + 8 * ni + 2 * t + i;
+                const int r = r0 + (warp & 1) * 32 + 8 * mi + 2 * t + i;
                 cr[(mi * 4 + ni) * 2 + i] = (rd && r < d.m && c < d.n) ? d.C[r + (size_t)c * d.ldc] : 0.0;
             }
         }
@@ -193,14 +215,14 @@ __device__ __forceinline__ void gemm_epilogue_creg(const GemmDesc &d, int r0, in
     const int g = lane >> 2, t = lane & 3;
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi) {
-        const int r = r0 + (warp & 1) * 32 + 8 * mi + g;
-        if (r >= d.m) continue;
 #pragma unroll
         for (int ni = 0; ni < 4; ++ni) {
+            const int c = c0 + (warp >> 1) * 32 + 8 * ni + g;
+            if (c >= d.n) continue;
 #pragma unroll
             for (int i = 0; i < 2; ++i) {
-                const int c = c0 + (warp >> 1) * 32 + 8 * ni + 2 * t + i;
-                if (c >= d.n) continue;
+                const int r = r0 + (warp & 1) * 32 + 8 * mi + 2 * t + i;
+                if (r >= d.m) continue;
                 const int q = (mi * 4 + ni) * 2 + i;
                 double v = d.alpha * acc[q];
                 if (d.beta != 0.0) v = fma(d.beta, cr[q], v);
@@ -231,22 +253,36 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
             }
         }
     } else {
+        // lane holds C(rl, cl) and C(rl + 1, cl): one 16-byte store where the
+        // pair is aligned and both rows exist, else two 8-byte stores
         const int lane = tid & 31, warp = tid >> 5;
         const int g = lane >> 2, t = lane & 3;
+        const bool rdc = d.beta != 0.0;
 #pragma unroll
-        for (int mi = 0; mi < 4; ++mi) {
-            const int rl = (warp & 1) * 32 + 8 * mi + g, r = r0 + rl;
-            if (r >= d.m) continue;
-            const int rs = MAP ? d.rmap[r] : r;
+        for (int ni = 0; ni < 4; ++ni) {
+            const int cl = (warp >> 1) * 32 + 8 * ni + g, c = c0 + cl;
+            if (c >= d.n) continue;
 #pragma unroll
-            for (int ni = 0; ni < 4; ++ni) {
-#pragma unroll
-                for (int i = 0; i < 2; ++i) {
-                    const int cl = (warp >> 1) * 32 + 8 * ni + 2 * t + i, c = c0 + cl;
-                    if (c >= d.n) continue;
-                    double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
-                    if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
-                    d.C[rs + (size_t)c * d.ldc] = v;
+            for (int mi = 0; mi < 4; ++mi) {
+                const int rl = (warp & 1) * 32 + 8 * mi + 2 * t, r = r0 + rl;
+                if (r >= d.m) continue;
+                const int q = (mi * 4 + ni) * 2;
+                double v0 = d.alpha * acc[q], v1 = d.alpha * acc[q + 1];
+                if (rdc) {
+                    v0 = fma(d.beta, sm.Cs[cl][rl], v0);
+                    v1 = fma(d.beta, sm.Cs[cl][rl + 1], v1);
+                }
+                if (MAP) {
+                    d.C[d.rmap[r] + (size_t)c * d.ldc] = v0;
+                    if (r + 1 < d.m) d.C[d.rmap[r + 1] + (size_t)c * d.ldc] = v1;
+                } else {
+                    double *dst = d.C + r + (size_t)c * d.ldc;
+                    if (r + 1 < d.m && ((reinterpret_cast<uintptr_t>(dst) & 15) == 0)) {
+                        *reinterpret_cast<double2 *>(dst) = make_double2(v0, v1);
+                    } else {
+                        dst[0] = v0;
+                        if (r + 1 < d.m) dst[1] = v1;
+                    }
                 }
             }
         }
