@@ -21,7 +21,7 @@
 namespace irr {
 
 constexpr int GBM = 64, GBN = 64, GBK = 16, G_NT = 128;
-constexpr int GPAD = GBM + 1;
+constexpr int GPAD = GBM + 2;  // even: 16-byte row pairs of the A stage stay aligned; 2-way (not 4-way) fragment conflicts
 
 struct GemmDesc {
     const double *A; long lda; int ta;
@@ -46,7 +46,7 @@ constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
 // Issue the cp.async copies of K chunk [k0, k0+16) of tile (r0, c0) into buffer
 // `buf` (out-of-range elements are zero-filled with plain stores).
-template <bool MAP = false, bool BRES = false>
+template <bool MAP = false, bool BRES = false, bool APAIR = true>
 __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int c0, int k0, GemmSmem &sm, int buf) {
     const int tid = threadIdx.x;
     if (MAP) {
@@ -72,6 +72,25 @@ __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int 
         }
         return;
     }
+    if (APAIR && !MAP && !d.ta) {
+        // op(A) = A column-major: row pairs (2p, 2p+1) of column kk, one
+        // 16-byte copy where the pair is aligned in global memory, else two
+#pragma unroll
+        for (int q = 0; q < (GBM * GBK) / (2 * G_NT); ++q) {
+            const int e = tid + G_NT * q;
+            const int r = 2 * (e & 31), kk = e >> 5;
+            const int gr = r0 + r, gk = k0 + kk;
+            double *dst = &sm.As[buf][kk][r];
+            const double *src = d.A + gr + (size_t)gk * d.lda;
+            const bool okk = gk < d.k;
+            if (okk && gr + 1 < d.m && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+                cp_async16(dst, src);
+            } else {
+                if (okk && gr < d.m) cp_async8(dst, src); else dst[0] = 0.0;
+                if (okk && gr + 1 < d.m) cp_async8(dst + 1, src + 1); else dst[1] = 0.0;
+            }
+        }
+    } else {
 #pragma unroll
     for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
@@ -85,6 +104,7 @@ __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int 
         } else {
             *dst = 0.0;
         }
+    }
     }
     if (BRES) return;  // B already resident in sm.Bs (the caller staged all K rows)
 #pragma unroll
@@ -295,13 +315,14 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
 // BRES: op(B) (k <= 2 GBK rows) is resident in sm.Bs for every tile of the
 // stream -- chunk c reads Bs[c] -- and is never loaded (the strip kernel's
 // U12, solved in place there).
-template <bool DMMA, class Next, bool MAP = false, bool CREG_OK = false, bool BRES = false>
+// APAIR: 16-byte row-pair copies of op(A) (off where the extra registers spill).
+template <bool DMMA, class Next, bool MAP = false, bool CREG_OK = false, bool BRES = false, bool APAIR = true>
 __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     GemmDesc d, dn;
     int r0, c0, rn, cn;
     if (!next(d, r0, c0)) return;
     int buf = 0;
-    if (d.k > 0) gemm_issue_chunk<MAP, BRES>(d, r0, c0, 0, sm, buf);
+    if (d.k > 0) gemm_issue_chunk<MAP, BRES, APAIR>(d, r0, c0, 0, sm, buf);
     cp_async_commit();
     bool have = true;
     constexpr bool CREG = DMMA && !MAP && CREG_OK;  // C in registers (the commit below is then an empty group)
@@ -317,10 +338,10 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         bool has_next_tile = false;
         for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
             if (c + 1 < nchunks) {
-                gemm_issue_chunk<MAP, BRES>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
+                gemm_issue_chunk<MAP, BRES, APAIR>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
             } else {
                 has_next_tile = next(dn, rn, cn);
-                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP, BRES>(dn, rn, cn, 0, sm, buf ^ 1);
+                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP, BRES, APAIR>(dn, rn, cn, 0, sm, buf ^ 1);
             }
             cp_async_commit();
             if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();

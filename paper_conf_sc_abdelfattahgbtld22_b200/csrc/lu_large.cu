@@ -124,7 +124,7 @@ __device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const 
 // solve_from also get U12 <- L11^-1 (rows j..j+ib-1), L11 in shared memory in
 // the layouts of trsm_col_regs.  top / bot: shared buffers of nb x
 // (SW_COLS+1).  SW_NT threads.
-template <int COLS = SW_COLS>
+template <int COLS = SW_COLS, int LT = COLS + 1>
 __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int j, int ib, int vbeg, int W,
                                            int jsplit, int shift, int solve_from, const SwapPlan &sp,
                                            const double *L11, int ldl, double *top, double *bot,
@@ -137,7 +137,6 @@ __device__ __forceinline__ void swap_chunk(double *__restrict__ gA, long ld, int
         atomicAdd(ph + (k), (unsigned long long)(t1 - tq));                   \
         tq = t1;                                                              \
     }
-    constexpr int LT = COLS + 1;
     constexpr int NWS = SW_NT / 32;
     const int nbot = sp.nbot;
     // warps over columns, lanes over the (<= 64) moved rows: no integer division
@@ -403,7 +402,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                     ++tt;
                     return true;
                 };
-                gemm_tile_stream<DMMA>(next, gsm);
+                gemm_tile_stream<DMMA, decltype(next), false, false, false, false>(next, gsm);
             }
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 2, (unsigned long long)(t1 - t0)); t0 = t1; }
@@ -712,13 +711,13 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
     // nb <= 32: the solved U12 rows (top) ARE the GEMM's resident B operand
-    // (gsm.Bs: 2 x 16 rows of GPAD = ST_COLS + 1), and L11 / bot sit in the C
+    // (gsm.Bs: 2 x 16 rows of stride GPAD), and L11 / bot sit in the C
     // stage (dead during the interchange + TRSM, filled only by the GEMM
     // tiles afterwards); else the original layout
     const bool bres = DMMA && nb <= 2 * GBK;
     double *top = bres ? &gsm.Bs[0][0][0] : st_smem + nb * ldl;
     double *L11 = bres ? &gsm.Cs[0][0] : st_smem;
-    double *bot = bres ? L11 + nb * ldl : top + nb * (ST_COLS + 1);
+    double *bot = bres ? L11 + nb * ldl : top + nb * GPAD;
     __shared__ SwapPlan sp;
     __shared__ int item_s;
     const int tid = threadIdx.x;
@@ -763,7 +762,8 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         __syncthreads();
         ST_PHASE(0)
         const int W = imin(ST_COLS, vtot - vb);
-        swap_chunk<ST_COLS>(gA, ld, j, ib, vb, W, jl, c1 - jl, c1, sp, L11, ldl, top, bot, ph);
+        // row stride GPAD: top doubles as the GEMM's resident B stage
+        swap_chunk<ST_COLS, GPAD>(gA, ld, j, ib, vb, W, jl, c1 - jl, c1, sp, L11, ldl, top, bot, ph);
         if (ph && tid == 0) t0 = clock64();
         // trailing GEMM on the strip's right-of-panel columns
         const int cbeg = (vb > jl ? vb : jl) + (c1 - jl), cend = vb + W + (c1 - jl);
@@ -788,7 +788,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
                 // B rows >= ib of the resident operand must be zero (A is
                 // zero-filled there, but stale shared memory may hold NaNs)
                 if (ib < 2 * GBK)
-                    for (int e = tid; e < (2 * GBK - ib) * (ST_COLS + 1); e += G_NT) top[ib * (ST_COLS + 1) + e] = 0.0;
+                    for (int e = tid; e < (2 * GBK - ib) * GPAD; e += G_NT) top[ib * GPAD + e] = 0.0;
                 __syncthreads();
                 gemm_tile_stream<DMMA, decltype(next), false, false, true>(next, gsm);
             } else {
@@ -829,7 +829,7 @@ __global__ void __launch_bounds__(LSW_NT) left_swaps_kernel(GetrfArgs a, const i
 }
 
 static size_t strip_smem_bytes(int nb) {
-    size_t sw = (size_t)(nb * (nb + 1) + 2 * nb * (ST_COLS + 1)) * sizeof(double);
+    size_t sw = (size_t)(nb * (nb + 1) + 2 * nb * GPAD) * sizeof(double);
     size_t m = sw > GEMM_SMEM ? sw : GEMM_SMEM;
     return (m + 15) & ~size_t(15);
 }
