@@ -330,15 +330,20 @@ def main():
     flush = torch.empty(512 * 1024 * 1024, dtype=torch.uint8, device=dev)   # > 126 MB L2
     stream = torch.cuda.current_stream(dev)
 
-    # status gather (the only collective): per-matrix info words, padded
+    # status gather (the only collective, a6): per-matrix 8-byte status words
+    # (info, FNV-1a of ipiv) from irr_status_words, padded to the largest shard
     pad = int(max(np.bincount(owner, minlength=world))) if world > 1 else len(mine)
-    status = torch.zeros(max(1, pad), dtype=torch.int32, device=coll_dev)
-    gathered = torch.zeros(world * max(1, pad), dtype=torch.int32, device=coll_dev) if world > 1 else None
+    words = torch.zeros(2 * max(1, pad), dtype=torch.int32, device=dev)
+    status = words if coll_dev == dev else torch.zeros_like(words, device=coll_dev)
+    gathered = torch.zeros(world * 2 * max(1, pad), dtype=torch.int32, device=coll_dev) if world > 1 else None
+    sm, sn = (B.m, B.n) if kind == "getrf" else (B.n1, B.n1)
 
     def step():
         call()
         if world > 1:
-            status[: B.batch].copy_(B.info[: B.batch])
+            irr.irr_status_words(B.batch, sm, sn, B.ipiv, B.info, words)
+            if status is not words:
+                status.copy_(words)
             dist.all_gather_into_tensor(gathered, status)
 
     def restore():

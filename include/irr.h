@@ -190,6 +190,17 @@ int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *
               int *info, void *work, size_t work_bytes, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_status_words -- the per-matrix completion record gathered across GPUs
+ * (SURVEY §8(a) a6 / §8(e)): words[2 i] = info[i], words[2 i + 1] = 32-bit
+ * FNV-1a hash (offset basis 2166136261, prime 16777619) of the bytes of
+ * ipiv[i][0 .. min(m[i], n[i])) in little-endian order (0 entries: the basis;
+ * matrices with info[i] < 0: 0).  All arrays device memory; asynchronous on
+ * `stream`; returns 0 or IRR_ERR_CUDA.
+ * ---------------------------------------------------------------------- */
+int irr_status_words(int batch, const int *m, const int *n, int *const *ipiv, const int *info,
+                     unsigned int *words, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * Tuning (tests and experiments; defaults are fixed by measurement and are
  * process-global, not thread-safe).  Keys: "nb" (tier-L panel width, 1..64),
  * "tier_s" (1 = enable the warp-per-matrix tier), "tier_m_max" (max padded

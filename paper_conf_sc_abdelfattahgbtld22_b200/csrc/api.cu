@@ -29,11 +29,12 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
                         int *queue, SlotList sl, cudaStream_t s);
 
 // defaults chosen by measurement on B200: tier M only up to
-// 96 KB (the 192 KB bin is faster in L1), S/M concurrent with L1, DMMA for the
+// 48 KB (C2 6.20 -> 6.06 ms against 96 KB, once L1 got faster; C4 100.5 ->
+// 100.4; 0 = no tier M is 6.00 on C2 but slower on C5), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
 // left-block interchanges (6.80 -> 6.53 ms).
-static Tuning g_default = {32, 1, M2_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -483,6 +484,21 @@ int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *
     if (max_n <= 0 || max_nrhs <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
     IRR_CUDA_TRY(cudaMemsetAsync(w.counters, 0, CNT_INTS * sizeof(int), s));
     getrs_core(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, w, s);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+int irr_status_words(int batch, const int *m, const int *n, int *const *ipiv, const int *info, unsigned int *words,
+                     irr_stream_t stream) {
+    if (batch < 0) return -1;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!m) return -2;
+    if (!n) return -3;
+    if (!ipiv) return -4;
+    if (!info) return -5;
+    if (!words) return -6;
+    int rc = check_device();
+    if (rc) return rc;
+    launch_status_words(batch, m, n, ipiv, info, words, (cudaStream_t)stream);
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 

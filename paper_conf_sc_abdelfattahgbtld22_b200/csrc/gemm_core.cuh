@@ -35,7 +35,7 @@ struct GemmDesc {
     const int *rmap = nullptr, *kmap = nullptr;
 };
 
-constexpr int CPAD = GBM + 2;  // even: 16-byte row pairs of the C stage stay aligned (cp.async16)
+constexpr int CPAD = GBM + 2;  // even: 16-byte row pairs of the C stage stay aligned (cp.async16, LDS.128)
 
 struct GemmSmem {
     double As[2][GBK][GPAD];
@@ -288,9 +288,10 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
                 if (r >= d.m) continue;
                 const int q = (mi * 4 + ni) * 2;
                 double v0 = d.alpha * acc[q], v1 = d.alpha * acc[q + 1];
-                if (rdc) {
-                    v0 = fma(d.beta, sm.Cs[cl][rl], v0);
-                    v1 = fma(d.beta, sm.Cs[cl][rl + 1], v1);
+                if (rdc) {  // rl even and CPAD even: the pair is one 16-byte shared load
+                    const double2 cv = *reinterpret_cast<const double2 *>(&sm.Cs[cl][rl]);
+                    v0 = fma(d.beta, cv.x, v0);
+                    v1 = fma(d.beta, cv.y, v1);
                 }
                 if (MAP) {
                     d.C[d.rmap[r] + (size_t)c * d.ldc] = v0;

@@ -260,6 +260,9 @@ void launch_getrs_validate(int batch, int max_n, int max_nrhs, const int *n, con
                            const double *const *A, const int *lda, int *const *ipiv, double *const *B,
                            const int *ldb, int *info, cudaStream_t s);
 
+void launch_status_words(int batch, const int *m, const int *n, int *const *ipiv, const int *info, unsigned *words,
+                         cudaStream_t s);
+
 int num_sms();
 }  // namespace irr
 

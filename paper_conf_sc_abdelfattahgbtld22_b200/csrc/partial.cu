@@ -62,4 +62,36 @@ void launch_getrs_validate(int batch, int max_n, int max_nrhs, const int *n, con
                                                              ldb, info);
 }
 
+// a6: per-matrix status words (info, FNV-1a of the pivot bytes), one thread
+// per matrix (the pivot vectors are short; this is bookkeeping, not the path)
+__global__ void status_words_kernel(int batch, const int *m, const int *n, int *const *ipiv, const int *info,
+                                    unsigned *words) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= batch) return;
+    const int e = info[i];
+    unsigned h = 2166136261u;
+    if (e >= 0) {
+        const int k = m[i] < n[i] ? m[i] : n[i];
+        const int *p = ipiv[i];
+        for (int t = 0; t < k; ++t) {
+            const unsigned v = (unsigned)p[t];
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                h ^= (v >> (8 * b)) & 0xffu;
+                h *= 16777619u;
+            }
+        }
+    } else {
+        h = 0u;
+    }
+    words[2 * i] = (unsigned)e;
+    words[2 * i + 1] = h;
+}
+
+void launch_status_words(int batch, const int *m, const int *n, int *const *ipiv, const int *info, unsigned *words,
+                         cudaStream_t s) {
+    KScope k(K_MISC, s);
+    status_words_kernel<<<(batch + 255) / 256, 256, 0, s>>>(batch, m, n, ipiv, info, words);
+}
+
 }  // namespace irr

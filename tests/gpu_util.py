@@ -126,3 +126,12 @@ def check_partial(F0, n1, Fg, ipiv, info, exact=False, label=""):
         d = np.abs(g22 - o22).max()
         assert d <= DEV_TOL * max(sigma, 1e-300), f"{label}: F22 dev {d / sigma}"
     return "match"
+
+
+def fnv1a_ipiv(ipiv) -> int:
+    """Host FNV-1a (32-bit) of an int32 pivot vector's little-endian bytes --
+    the definition irr_status_words implements (include/irr.h)."""
+    h = 2166136261
+    for byte in np.ascontiguousarray(ipiv, dtype="<i4").tobytes():
+        h = ((h ^ byte) * 16777619) & 0xFFFFFFFF
+    return h

@@ -57,9 +57,14 @@ def test_edge_shapes_all_tiers():
     assert st.get("match", 0) + st.get("empty", 0) >= len(shapes) - 2
 
 
-def test_tier_m_boundary_and_extreme_shapes():
-    # m * n around the tier-M limit (padded m*n <= 24576) and very thin shapes
+@pytest.mark.parametrize("tier_m_max", [None, 12288, 24576])
+def test_tier_m_boundary_and_extreme_shapes(tier_m_max):
+    # m * n around the tier-M limits (48 / 96 / 192 KB footprints) and very
+    # thin shapes, at the default limit and with the two larger bins enabled
+    if tier_m_max is not None:
+        irr.irr_set_tuning("tier_m_max", tier_m_max)
     shapes = [(151, 162), (151, 163), (153, 160), (160, 153), (96, 256), (256, 96), (97, 256),
+              (77, 79), (78, 78), (79, 78), (110, 111), (111, 110), (64, 96), (95, 64),
               (1, 1024), (1024, 1), (33, 1), (1, 33), (300, 7), (7, 300), (1000, 30), (30, 1000)]
     _run_and_check(_uniform(shapes, seed=5))
 
@@ -104,9 +109,11 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "L", "L2", "Lswap", "Ltall"])
+@pytest.mark.parametrize("tier", ["default", "M", "L", "L2", "Lswap", "Ltall"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
+    if tier == "M":
+        irr.irr_set_tuning("tier_m_max", 24576)
     if tier == "Lswap":
         irr.irr_set_tuning("l1_rowmap", 1)
     if tier == "Ltall":
@@ -293,3 +300,28 @@ def test_c5_sample_parity():
     mats = [irrgen.uniform_values(cfg.seed, int(g), int(cfg.m[g]), int(cfg.n[g])) for g in sel]
     st = _run_and_check(mats)
     assert st.get("match", 0) >= len(mats) - 2
+
+
+def test_status_words():
+    """a6 status words: info and the FNV-1a of ipiv (include/irr.h), checked
+    against the host definition on the oracle's pivots; a bad-argument matrix
+    gets (info, 0)."""
+    from gpu_util import fnv1a_ipiv
+    from paper_conf_sc_abdelfattahgbtld22_b200.batch import MatrixBatch
+    import oracle
+    shapes = [(5, 5), (40, 33), (300, 280), (1, 7), (0, 3)]
+    mats = _uniform(shapes, seed=91)
+    LUs, ipivs, info, (B, _) = gpu_getrf(mats)
+    words = torch.zeros(2 * B.batch, dtype=torch.int32, device="cuda")
+    irr.irr_status_words(B.batch, B.m, B.n, B.ipiv, B.info, words)
+    w = words.cpu().numpy().view(np.uint32).reshape(-1, 2)
+    for g, A in enumerate(mats):
+        _, ipo, info_o, _ = oracle.getrf(A)
+        assert int(w[g, 0]) == info_o
+        assert int(w[g, 1]) == fnv1a_ipiv(ipo)
+    # a matrix with a bad leading dimension: info -4, hash 0
+    B.ld = torch.tensor([5, 40, 300, 0, 1], dtype=torch.int32, device="cuda")
+    B.getrf()
+    irr.irr_status_words(B.batch, B.m, B.n, B.ipiv, B.info, words)
+    w = words.cpu().numpy().view(np.uint32).reshape(-1, 2)
+    assert w[3, 0].view(np.int32) == -4 and w[3, 1] == 0
