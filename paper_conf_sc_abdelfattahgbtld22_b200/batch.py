@@ -152,3 +152,118 @@ class FrontBatch:
         return irr.irr_getrf_partial(self.batch, self.max_n1, self.max_n2, self.n1, self.n2, self.F11, self.ld11,
                                      self.F12, self.ld12, self.F21, self.ld21, self.F22, self.ld22, self.ipiv,
                                      self.info, self.workspace(), stream)
+
+
+# ---------------------------------------------------------------------------
+# End to end with HOST buffers: the batch is streamed through the GPU in
+# contiguous chunks of matrices, so the host->device copy of chunk c+1, the
+# factorization of chunk c and the device->host copy of chunk c-1 overlap (two
+# copy streams -- B200 has copy engines in both directions -- and one compute
+# stream; every library call stays on the compute stream, so the library's
+# own forked side stream is never shared by two concurrent calls).  Matrices
+# are independent, so a chunk is just a sub-batch: views of the size / pointer
+# / ipiv / info arrays at an offset, no copies.
+# ---------------------------------------------------------------------------
+def _chunk_bounds(offsets, total, count, chunks):
+    """Matrix index boundaries splitting the flat buffer into ~equal byte ranges."""
+    if count == 0:
+        return [0, 0]
+    chunks = max(1, min(chunks, count))
+    ends = np.append(np.asarray(offsets[1:], dtype=np.int64), total)
+    cuts = [0]
+    for c in range(1, chunks):
+        i = int(np.searchsorted(ends, total * c / chunks, side="left")) + 1
+        if cuts[-1] < i < count:
+            cuts.append(i)
+    cuts.append(count)
+    return cuts
+
+
+class _Pipe:
+    def __init__(self, device):
+        self.h2d = torch.cuda.Stream(device)
+        self.d2h = torch.cuda.Stream(device)
+
+    def run(self, cuts, elem_range, data, host_in, host_out, compute, extra_out):
+        """elem_range(i0, i1) -> (e0, e1) flat element range of matrices [i0, i1);
+        compute(i0, i1, stream) factors that sub-batch; extra_out: list of
+        (device tensor, host tensor, range_fn) copied back per chunk."""
+        cur = torch.cuda.current_stream(data.device)
+        self.h2d.wait_stream(cur)
+        self.d2h.wait_stream(cur)
+        loaded, done = [], []
+        for i0, i1 in zip(cuts[:-1], cuts[1:]):
+            e0, e1 = elem_range(i0, i1)
+            with torch.cuda.stream(self.h2d):
+                data[e0:e1].copy_(host_in[e0:e1], non_blocking=True)
+                ev = torch.cuda.Event()
+                ev.record(self.h2d)
+            loaded.append(ev)
+        for (i0, i1), ev in zip(zip(cuts[:-1], cuts[1:]), loaded):
+            cur.wait_event(ev)
+            compute(i0, i1, cur)
+            evc = torch.cuda.Event()
+            evc.record(cur)
+            done.append(evc)
+        for (i0, i1), evc in zip(zip(cuts[:-1], cuts[1:]), done):
+            self.d2h.wait_event(evc)
+            e0, e1 = elem_range(i0, i1)
+            with torch.cuda.stream(self.d2h):
+                host_out[e0:e1].copy_(data[e0:e1], non_blocking=True)
+                for dev_t, host_t, rng in extra_out:
+                    a, b = rng(i0, i1)
+                    host_t[a:b].copy_(dev_t[a:b], non_blocking=True)
+        cur.wait_stream(self.d2h)
+
+
+def _sub(t, i0, i1):
+    return t[i0:i1]
+
+
+def getrf_host(B: "MatrixBatch", host_in, host_out, ipiv_out, info_out, chunks=8, pipe=None):
+    """irr_getrf end to end from pinned host buffers (flat layout of B):
+    host_out <- factors, ipiv_out <- pivots (flat), info_out <- info.  Ordered
+    on torch's current stream (the caller synchronises to read the results)."""
+    pipe = pipe or _Pipe(B.device)
+    cuts = _chunk_bounds(B.offsets, B.total, B.batch, chunks)
+    ends = np.append(B.offsets[1:], B.total) if B.batch else np.zeros(0, dtype=np.int64)
+    pends = np.append(B.ipiv_off[1:], B.ipiv_data.numel()) if B.batch else np.zeros(0, dtype=np.int64)
+
+    def rng(i0, i1):
+        return int(B.offsets[i0]), int(ends[i1 - 1])
+
+    def prng(i0, i1):
+        return int(B.ipiv_off[i0]), int(pends[i1 - 1])
+
+    def compute(i0, i1, s):
+        irr.irr_getrf(i1 - i0, int(B.m_h[i0:i1].max()), int(B.n_h[i0:i1].max()), _sub(B.m, i0, i1),
+                      _sub(B.n, i0, i1), _sub(B.ptr, i0, i1), _sub(B.ld, i0, i1), _sub(B.ipiv, i0, i1),
+                      _sub(B.info, i0, i1), B.workspace(), s)
+
+    pipe.run(cuts, rng, B.data, host_in, host_out, compute,
+             [(B.ipiv_data, ipiv_out, prng), (B.info, info_out, lambda a, b: (a, b))])
+    return pipe
+
+
+def getrf_partial_host(F: "FrontBatch", host_in, host_out, ipiv_out, info_out, chunks=8, pipe=None):
+    """irr_getrf_partial end to end from pinned host buffers (flat layout of F)."""
+    pipe = pipe or _Pipe(F.device)
+    cuts = _chunk_bounds(F.offsets, F.total, F.batch, chunks)
+    ends = np.append(F.offsets[1:], F.total) if F.batch else np.zeros(0, dtype=np.int64)
+    pends = np.append(F.ipiv_off[1:], F.ipiv_data.numel()) if F.batch else np.zeros(0, dtype=np.int64)
+
+    def rng(i0, i1):
+        return int(F.offsets[i0]), int(ends[i1 - 1])
+
+    def prng(i0, i1):
+        return int(F.ipiv_off[i0]), int(pends[i1 - 1])
+
+    def compute(i0, i1, s):
+        S = lambda t: _sub(t, i0, i1)  # noqa: E731
+        irr.irr_getrf_partial(i1 - i0, int(F.n1_h[i0:i1].max()), int(F.n2_h[i0:i1].max()), S(F.n1), S(F.n2),
+                              S(F.F11), S(F.ld11), S(F.F12), S(F.ld12), S(F.F21), S(F.ld21), S(F.F22),
+                              S(F.ld22), S(F.ipiv), S(F.info), F.workspace(), s)
+
+    pipe.run(cuts, rng, F.data, host_in, host_out, compute,
+             [(F.ipiv_data, ipiv_out, prng), (F.info, info_out, lambda a, b: (a, b))])
+    return pipe

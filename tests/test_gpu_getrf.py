@@ -325,3 +325,37 @@ def test_status_words():
     irr.irr_status_words(B.batch, B.m, B.n, B.ipiv, B.info, words)
     w = words.cpu().numpy().view(np.uint32).reshape(-1, 2)
     assert w[3, 0].view(np.int32) == -4 and w[3, 1] == 0
+
+
+@pytest.mark.parametrize("chunks", [1, 3, 16])
+def test_pipelined_host_entry_points(chunks):
+    """getrf_host / getrf_partial_host (pinned host in -> host out, chunked
+    H2D / getrf / D2H overlap) give bitwise the results of the device path."""
+    from paper_conf_sc_abdelfattahgbtld22_b200.batch import (FrontBatch, MatrixBatch, getrf_host,
+                                                             getrf_partial_host)
+    cfg = irrgen.config("C2", scale=0.03)
+    B = MatrixBatch(cfg.m, cfg.n)
+    host = torch.zeros(B.total, dtype=torch.float64, pin_memory=True)
+    irrgen.fill_packed(cfg.seed, cfg.m, cfg.n, B.ld_h, B.offsets, host.numpy())
+    outs = [torch.empty(t.numel(), dtype=t.dtype, pin_memory=True) for t in (B.data, B.ipiv_data, B.info)]
+    getrf_host(B, host, *outs, chunks=chunks)
+    torch.cuda.synchronize()
+    B.data.copy_(host)
+    B.ipiv_data.zero_()
+    B.getrf()
+    torch.cuda.synchronize()
+    assert np.array_equal(outs[0].numpy(), B.data.cpu().numpy())
+    assert np.array_equal(outs[1].numpy(), B.ipiv_data.cpu().numpy())
+    assert np.array_equal(outs[2].numpy(), B.info.cpu().numpy())
+    n1, n2 = [3, 40, 0, 100, 7], [5, 60, 9, 30, 0]
+    F = FrontBatch(n1, n2)
+    fh = torch.zeros(F.total, dtype=torch.float64, pin_memory=True)
+    irrgen.fill_packed(7, F.nf_h, F.nf_h, F.ld_h, F.offsets, fh.numpy())
+    fo = [torch.empty(t.numel(), dtype=t.dtype, pin_memory=True) for t in (F.data, F.ipiv_data, F.info)]
+    getrf_partial_host(F, fh, *fo, chunks=chunks)
+    torch.cuda.synchronize()
+    F.data.copy_(fh)
+    F.getrf_partial()
+    torch.cuda.synchronize()
+    assert np.array_equal(fo[0].numpy(), F.data.cpu().numpy())
+    assert np.array_equal(fo[2].numpy(), F.info.cpu().numpy())

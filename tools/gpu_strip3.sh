@@ -1,0 +1,2 @@
+ncu --set full --clock-control none --import-source on -k regex:strip_kernel -c 1 -o gpurun_out/prof_strip_C3b python tools/prof_one.py --config C3 --scale 0.5 --reps 1 > gpurun_out/ncu_strip.log 2>&1
+python tools/phase_time.py --config C3 --scale 0.5 > gpurun_out/phase_C3.txt 2>&1; cat gpurun_out/phase_C3.txt
