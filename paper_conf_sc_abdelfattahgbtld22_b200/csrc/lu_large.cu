@@ -95,26 +95,40 @@ __device__ __forceinline__ void plan_swaps_from(const int *piv_abs, int j, int i
 // column-major with leading dimension ldl, or, when ldl == 0, its strict lower
 // triangle packed by columns (column s = rows s+1..ib-1 at s(2ib-s-1)/2).
 // Shift-register form (as in tier S): v[0] is always the next solution
-// entry, so the loop body is the same for every step (O(NBX) code, no local
-// memory) and each step is NBX-1 independent FMAs.
+// entry, so the loop body is the same for every step (O(W) code, no local
+// memory) and each step is W-1 independent FMAs, W shrinking 32 -> 4.
+// trsm_col_step: one substitution step on the W leading registers (the
+// remaining rows of the column fit in W: ib - s <= W).
+template <int NBX, int W>
+__device__ __forceinline__ void trsm_col_step(double (&v)[NBX], double *x, int ldx, int ib, int s,
+                                              const double *L11, int ldl) {
+    const double xs = v[0];
+    x[s * ldx] = xs;
+    // column s of L11 below the diagonal is contiguous in both layouts
+    const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
+    const int cnt = ib - s - 1;
+#pragma unroll
+    for (int q = 0; q + 1 < W; ++q) {
+        const double l = (q < cnt) ? Ls[q] : 0.0;
+        v[q] = fma(-l, xs, v[q + 1]);
+    }
+    v[W - 1] = 0.0;
+}
+
 template <int NBX>
 __device__ __forceinline__ void trsm_col_regs(double *x, int ldx, int ib, const double *L11, int ldl) {
     double v[NBX];
 #pragma unroll
     for (int r = 0; r < NBX; ++r) v[r] = (r < ib) ? x[r * ldx] : 0.0;
-    for (int s = 0; s < ib; ++s) {
-        const double xs = v[0];
-        x[s * ldx] = xs;
-        // column s of L11 below the diagonal is contiguous in both layouts
-        const double *Ls = L11 + (ldl ? s + 1 + s * ldl : (s * (2 * ib - s - 1)) / 2);
-        const int cnt = ib - s - 1;
-#pragma unroll
-        for (int q = 0; q + 1 < NBX; ++q) {
-            const double l = (q < cnt) ? Ls[q] : 0.0;
-            v[q] = fma(-l, xs, v[q + 1]);
-        }
-        v[NBX - 1] = 0.0;
-    }
+    // the active width shrinks with the remaining rows (as in the panel):
+    // about half the FMAs and L loads of a fixed-width sweep
+    int s = 0;
+    if (NBX >= 32)
+        for (; ib - s > 16; ++s) trsm_col_step<NBX, (NBX >= 32 ? 32 : NBX)>(v, x, ldx, ib, s, L11, ldl);
+    if (NBX >= 16)
+        for (; ib - s > 8; ++s) trsm_col_step<NBX, (NBX >= 16 ? 16 : NBX)>(v, x, ldx, ib, s, L11, ldl);
+    for (; ib - s > 4; ++s) trsm_col_step<NBX, (NBX >= 8 ? 8 : NBX)>(v, x, ldx, ib, s, L11, ldl);
+    for (; s < ib; ++s) trsm_col_step<NBX, 4>(v, x, ldx, ib, s, L11, ldl);
 }
 
 // Apply the plan to W columns of one matrix given as a VIRTUAL range
