@@ -8,8 +8,8 @@
 //   * lane r holds row r in registers, SHIFTED so that a[0] is always the
 //     current pivot column: the rank-1 update and the shift are one FMA per
 //     register, a[c] <- a[c+1] - l * u[c+1], so every elimination step runs the
-//     same code; the step width W shrinks 32 -> 16 -> 8 -> 4 with the active
-//     columns;
+//     same code; the step width W shrinks 32 -> 24 -> 16 -> 12 -> 8 -> 4
+//     with the active columns;
 //   * rows never move.  `pos` is the row's current position; an interchange
 //     is a relabelling (the winner lane takes position k, the row at k takes
 //     the winner's old position).  So nothing is swapped during the
@@ -142,10 +142,16 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     }
     int pos = lane, my_piv = 0, info = 0, k = 0;
     const int K = m < n ? m : n;
-    if (NC >= 32)
-        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
-    if (NC >= 16)
-        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+    // active width W >= n - k in steps of 32 / 24 / 16 / 12 / 8 / 4 (the
+    // FMAs, pivot-row loads and publish stores of a step scale with W)
+    if (NC >= 32) {
+        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+    }
+    if (NC >= 16) {
+        while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+    }
     while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
     while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, sm);
     __syncwarp();  // L / U rows from every lane are complete
