@@ -250,7 +250,7 @@ def main():
     ap.add_argument("--config", default="C2", choices=irrgen.CONFIG_NAMES)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--e2e-chunks", type=int, default=32, help="chunks of the pipelined end-to-end call")
+    ap.add_argument("--e2e-chunks", type=int, default=8, help="chunks of the pipelined end-to-end call")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--ref-seconds", type=float, default=5.0)
