@@ -25,6 +25,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
          "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC]
+# experiments only (A/B of build-time switches, e.g. -DIRR_S32_CTAS=5); empty by default
+FLAGS += [f for f in os.environ.get("IRR_NVCC_EXTRA", "").split() if f]
 
 
 def _deps():
