@@ -42,6 +42,7 @@ struct GsRing {
 struct GsSolve {
     double T[GS_BR * GS_LDT];  // diagonal triangle, column-major
     double X[GS_SW * GS_LDT];  // the block being solved: X[c * GS_LDT + r]
+    double rd[GS_BR];          // upper solve: reciprocals of the diagonal
 };
 // The ring (update GEMM) and the solve buffers are used one after the other
 // and share the same bytes; the permutation phase (perm + ipiv ints and a
@@ -178,6 +179,13 @@ __device__ __forceinline__ void gs_block(const double *T, long ldt, double *X, l
             }
     cp_async_wait<0>();
     __syncthreads();
+    if (!LOWER) {
+        // one true division per diagonal entry, then multiplies in the
+        // substitution (ncu: the per-step division was 14% of the kernel's
+        // stall samples and 13% of its instructions)
+        if (tid < GS_BR) sv.rd[tid] = 1.0 / sv.T[tid * GS_LDT + tid];
+        __syncthreads();
+    }
     // substitution: column c = tid >> 2; lane q4 = tid & 3 owns rows q4 + 4k
     // (interleaved, so the four lanes of a column read four consecutive T
     // entries: conflict-free); x_s comes from lane s & 3 by shuffle
@@ -210,7 +218,7 @@ __device__ __forceinline__ void gs_block(const double *T, long ldt, double *X, l
 #pragma unroll
                 for (int ss = 15; ss >= 0; --ss) {
                     const int s = s0 + ss;
-                    if (q4 == (s & 3)) x[s >> 2] = x[s >> 2] / sv.T[s * GS_LDT + s];
+                    if (q4 == (s & 3)) x[s >> 2] = x[s >> 2] * sv.rd[s];
                     const double xs = __shfl_sync(FULL, x[s >> 2], base | (s & 3));
                     const double *Ts = sv.T + s * GS_LDT + q4;
 #pragma unroll
@@ -269,26 +277,31 @@ __global__ void __launch_bounds__(GS_NT, 2) getrs_strip_kernel(GsArgs g, SlotLis
             bool moved = false;
             for (int r = tid; r < n1; r += GS_NT) moved |= perm[r] != r;
             if (__syncthreads_or(moved)) {
-                for (int cc = 0; cc < W; cc += 2) {
-                    const int nc = imin(2, W - cc);
-                    for (int c = 0; c < nc; ++c) {
+                // as many columns per round as the buffer holds (was 2: the
+                // rounds' load latency was ~20% of the kernel's stall samples)
+                constexpr int CAP = (int)((GS_SMEM - 2 * GS_N1MAX * sizeof(int)) / sizeof(double));
+                const int per = imax(1, imin(W, CAP / n1));
+                for (int cc = 0; cc < W; cc += per) {
+                    const int nc = imin(per, W - cc);
+                    for (int c = warp; c < nc; c += GS_NT / 32) {
                         const double *col = X + (size_t)(c0 + cc + c) * ld12;
-                        for (int r = tid; r < n1; r += GS_NT) colbuf[c * GS_N1MAX + r] = col[r];
+                        for (int r = lane; r < n1; r += 32) cp_async8(&colbuf[(size_t)c * n1 + r], col + r);
                     }
+                    cp_async_commit();
+                    cp_async_wait<0>();
                     __syncthreads();
-                    for (int c = 0; c < nc; ++c) {
+                    for (int c = warp; c < nc; c += GS_NT / 32) {
                         double *col = X + (size_t)(c0 + cc + c) * ld12;
-                        for (int r = tid; r < n1; r += GS_NT) {
+                        for (int r = lane; r < n1; r += 32) {
                             const int p = perm[r];
-                            if (p != r) col[r] = colbuf[c * GS_N1MAX + p];
+                            if (p != r) col[r] = colbuf[(size_t)c * n1 + p];
                         }
                     }
                     __syncthreads();
                 }
             }
         }
-        (void)lane; (void)warp;
-        // ---- 2. L^-1 (unit lower), blocks top to bottom
+            // ---- 2. L^-1 (unit lower), blocks top to bottom
         for (int r0 = 0; r0 < n1; r0 += GS_BR) gs_block<true>(F11, ld11, X, ld12, n1, c0, W, r0, rg, sv);
         // ---- 3. U^-1 (non-unit upper), blocks bottom to top
         const int last = ((n1 - 1) / GS_BR) * GS_BR;
