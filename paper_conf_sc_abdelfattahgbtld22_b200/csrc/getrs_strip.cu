@@ -73,26 +73,39 @@ struct GsUnits {
 //      -= T(rows r0.., cols k0..k0+K) * X(rows k0..k0+K, strip)
 __device__ __forceinline__ void gs_issue(const double *T, long ldt, int r0, int rb, const double *X, long ldx,
                                          int c0, int W, int kbeg, int k0, int kend, GsRing &rg, int st) {
+    // pairs of consecutive elements (rows of T, k of X): one 16-byte copy
+    // where the pair is aligned in global memory, else two 8-byte copies
+    // (ncu: the per-element copies were ~10% of the kernel's stall samples)
     const int tid = threadIdx.x;
 #pragma unroll
-    for (int q = 0; q < (GS_BR * GS_BK) / GS_NT; ++q) {
+    for (int q = 0; q < (GS_BR * GS_BK) / (2 * GS_NT); ++q) {
         const int e = tid + GS_NT * q;
-        const int m = e & (GS_BR - 1), kk = e >> 6;
+        const int m = 2 * (e & (GS_BR / 2 - 1)), kk = e / (GS_BR / 2);
         const int gk = k0 + kk;
-        const bool ok = m < rb && gk < kend;
         double *dst = &rg.A[st][kk * GS_LDA + m];
-        if (ok) cp_async8(dst, T + r0 + m + (size_t)gk * ldt);
-        else *dst = 0.0;
+        const double *src = T + r0 + m + (size_t)gk * ldt;
+        const bool okk = gk < kend;
+        if (okk && m + 1 < rb && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+            cp_async16(dst, src);
+        } else {
+            if (okk && m < rb) cp_async8(dst, src); else dst[0] = 0.0;
+            if (okk && m + 1 < rb) cp_async8(dst + 1, src + 1); else dst[1] = 0.0;
+        }
     }
 #pragma unroll
-    for (int q = 0; q < (GS_SW * GS_BK) / GS_NT; ++q) {
+    for (int q = 0; q < (GS_SW * GS_BK) / (2 * GS_NT); ++q) {
         const int e = tid + GS_NT * q;
-        const int kk = e & (GS_BK - 1), n = e >> 4;
+        const int kk = 2 * (e & (GS_BK / 2 - 1)), n = e / (GS_BK / 2);
         const int gk = k0 + kk;
-        const bool ok = n < W && gk < kend;
         double *dst = &rg.B[st][n * GS_LDB + kk];
-        if (ok) cp_async8(dst, X + gk + (size_t)(c0 + n) * ldx);
-        else *dst = 0.0;
+        const double *src = X + gk + (size_t)(c0 + n) * ldx;
+        const bool okn = n < W;
+        if (okn && gk + 1 < kend && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+            cp_async16(dst, src);
+        } else {
+            if (okn && gk < kend) cp_async8(dst, src); else dst[0] = 0.0;
+            if (okn && gk + 1 < kend) cp_async8(dst + 1, src + 1); else dst[1] = 0.0;
+        }
     }
     (void)kbeg;
 }
