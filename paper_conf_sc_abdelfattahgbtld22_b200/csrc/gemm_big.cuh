@@ -41,31 +41,60 @@ __device__ __forceinline__ void cp_async8_zf(void *smem, const void *gmem, bool 
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(n) : "memory");
 }
 
+// 16-byte copy of elements (i, i+1) along the operand's contiguous dimension
+// when both exist and the source pair is aligned, else 8-byte copies / zeros
+// (`base`: an in-bounds address for the zero-filling copies, never read)
+__device__ __forceinline__ void x_pair(double *dst, const double *src, bool ok0, bool ok1, const double *base) {
+    if (ok0 && ok1 && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+        cp_async16(dst, src);
+    } else {
+        cp_async8_zf(dst, ok0 ? src : base, ok0);
+        cp_async8_zf(dst + 1, ok1 ? src + 1 : base, ok1);
+    }
+}
+
 // Stage chunk [k0, k0+16) of the (r0, c0) tile.  op(A) is m x k, op(B) k x n.
+// Element pairs along each operand's contiguous dimension (m for A, k for
+// A^T, k for B, n for B^T): both shared layouts keep such pairs 16-byte
+// aligned (even leading dimensions 132 / 20).
 template <int TA, int TB>
 __device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st) {
     const int tid = threadIdx.x;
     double *As = sm.A[st];
     double *Bs = sm.B[st];
 #pragma unroll
-    for (int q = 0; q < (XBM * XBK) / X_NT; ++q) {
+    for (int q = 0; q < (XBM * XBK) / (2 * X_NT); ++q) {
         const int e = tid + X_NT * q;
-        int m, kk;
-        if (!TA) { m = e & (XBM - 1); kk = e >> 7; } else { kk = e & (XBK - 1); m = e >> 4; }
-        const int gm = r0 + m, gk = k0 + kk;
-        const bool ok = gm < d.m && gk < d.k;
-        const double *src = ok ? (TA ? d.A + gk + (size_t)gm * d.lda : d.A + gm + (size_t)gk * d.lda) : d.A;
-        cp_async8_zf(TA ? &As[m * XLD_MK + kk] : &As[kk * XLD_KM + m], src, ok);
+        if (!TA) {  // A(m, k) at A + m + k lda: pairs along m
+            const int m = 2 * (e & (XBM / 2 - 1)), kk = e / (XBM / 2);
+            const int gm = r0 + m, gk = k0 + kk;
+            const bool okk = gk < d.k;
+            x_pair(&As[kk * XLD_KM + m], d.A + gm + (size_t)(okk ? gk : 0) * d.lda, okk && gm < d.m,
+                   okk && gm + 1 < d.m, d.A);
+        } else {    // A(k, m) at A + k + m lda: pairs along k
+            const int kk = 2 * (e & (XBK / 2 - 1)), m = e / (XBK / 2);
+            const int gm = r0 + m, gk = k0 + kk;
+            const bool okm = gm < d.m;
+            x_pair(&As[m * XLD_MK + kk], d.A + gk + (size_t)(okm ? gm : 0) * d.lda, okm && gk < d.k,
+                   okm && gk + 1 < d.k, d.A);
+        }
     }
 #pragma unroll
-    for (int q = 0; q < (XBN * XBK) / X_NT; ++q) {
+    for (int q = 0; q < (XBN * XBK) / (2 * X_NT); ++q) {
         const int e = tid + X_NT * q;
-        int n, kk;
-        if (!TB) { kk = e & (XBK - 1); n = e >> 4; } else { n = e & (XBN - 1); kk = e >> 7; }
-        const int gn = c0 + n, gk = k0 + kk;
-        const bool ok = gn < d.n && gk < d.k;
-        const double *src = ok ? (TB ? d.B + gn + (size_t)gk * d.ldb : d.B + gk + (size_t)gn * d.ldb) : d.B;
-        cp_async8_zf(TB ? &Bs[kk * XLD_KM + n] : &Bs[n * XLD_MK + kk], src, ok);
+        if (!TB) {  // B(k, n) at B + k + n ldb: pairs along k
+            const int kk = 2 * (e & (XBK / 2 - 1)), n = e / (XBK / 2);
+            const int gn = c0 + n, gk = k0 + kk;
+            const bool okn = gn < d.n;
+            x_pair(&Bs[n * XLD_MK + kk], d.B + gk + (size_t)(okn ? gn : 0) * d.ldb, okn && gk < d.k,
+                   okn && gk + 1 < d.k, d.B);
+        } else {    // B(n, k) at B + n + k ldb: pairs along n
+            const int n = 2 * (e & (XBN / 2 - 1)), kk = e / (XBN / 2);
+            const int gn = c0 + n, gk = k0 + kk;
+            const bool okk = gk < d.k;
+            x_pair(&Bs[kk * XLD_KM + n], d.B + gn + (size_t)(okk ? gk : 0) * d.ldb, okk && gn < d.n,
+                   okk && gn + 1 < d.n, d.B);
+        }
     }
 }
 
