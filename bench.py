@@ -462,7 +462,9 @@ def main():
     roof["kernel"] = dname
     roof["share_of_step"] = dms_step / (total_ms / args.steps)
     roof["launches_per_step"] = dcnt / args.steps
-    roof["peak_source"] = (hbm_src + " MEASURED_PEAKS.json hbm_gbs") if roof["bound"] == "hbm" else \
+    roof["peak_source"] = ("measured: MEASURED_PEAKS.json hbm_gbs" if hbm_src == "measured" else
+                           "fallback 6,650 GB/s (B200_PROFILING.md; MEASURED_PEAKS.json absent)") \
+        if roof["bound"] == "hbm" else \
         "derived: 148 SM x 64 DFMA/clk x 2 flop x 1.965 GHz"
     roof["traffic"] = _ncu_traffic(args.config, dname, dcnt / args.steps)
     whole = {"flops": flops_local, "bytes": bytes_local,
