@@ -305,3 +305,34 @@ def fill_packed(seed: int, m, n, ld, offsets, out: np.ndarray, gid_base: int = 0
             out[offsets[gid] + i + j * ld[gid]] = vals
         g0 = g1
     return out
+
+
+def extend_add_level(seed: int, n_parents: int, np_max: int, children_per_parent: int = 2,
+                     frac_lo: float = 0.25, frac_hi: float = 0.75):
+    """One level of a synthetic binary assembly tree for the extend-add.
+
+    Parent p has order np_p ~ U[1, np_max]; each of its children has a Schur
+    complement of order n2_c ~ U[frac_lo, frac_hi] * np_p (at least 1, at most
+    np_p) whose rows / columns map to a sorted random subset rel_c of the
+    parent's indices (nested dissection: a child's separator variables appear
+    in its parent front, in order).  Children are listed parent by parent
+    (child 0 of parent 0, child 1 of parent 0, ...).  Values from
+    uniform_values.  Returns (np_sizes, parent_of_child, n2, rel list,
+    F22 list, Fp list) -- no arithmetic of the method.
+    """
+    rng = np.random.default_rng(seed)
+    np_sizes = rng.integers(1, np_max + 1, size=n_parents).astype(np.int32)
+    parent, n2, rel, F22 = [], [], [], []
+    Fp = [uniform_values(seed, 1_000_000 + p, int(s), int(s)) for p, s in enumerate(np_sizes)]
+    gid = 0
+    for p, s in enumerate(np_sizes):
+        for _ in range(children_per_parent):
+            k = int(rng.integers(max(1, int(frac_lo * s)), max(1, int(frac_hi * s)) + 1))
+            k = min(max(k, 1), int(s))
+            r = np.sort(rng.choice(int(s), size=k, replace=False)).astype(np.int32)
+            parent.append(p)
+            n2.append(k)
+            rel.append(r)
+            F22.append(uniform_values(seed, gid, k, k))
+            gid += 1
+    return np_sizes, np.array(parent, dtype=np.int32), np.array(n2, dtype=np.int32), rel, F22, Fp

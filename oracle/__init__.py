@@ -52,6 +52,8 @@ def lib():
         L.oracle_laswp.argtypes = [C.c_int, dp, C.c_int, C.c_int, C.c_int, ip]
         L.oracle_getrs.argtypes = [C.c_int, C.c_int, dp, C.c_int, ip, dp, C.c_int]
         L.oracle_getrs.restype = C.c_int
+        L.oracle_extend_add.argtypes = [C.c_int, dp, C.c_int, ip, C.c_int, dp, C.c_int]
+        L.oracle_extend_add.restype = C.c_int
         L.oracle_backward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
         L.oracle_backward_error.restype = C.c_double
         L.oracle_num_threads.restype = C.c_int
@@ -201,6 +203,20 @@ def getrs(LU, ipiv, B):
     if r < 0:
         raise ValueError(f"oracle_getrs: bad argument {-r}")
     return B
+
+
+def extend_add(Fp, F22, rel):
+    """Fp[rel_i, rel_j] += F22[i, j], on a copy of the np x np parent front Fp."""
+    Fp, F22 = _fortran(Fp), _fortran(F22)
+    n2, npp = F22.shape[0], Fp.shape[0]
+    rel = np.ascontiguousarray(rel, dtype=np.int32)
+    r0 = rel if rel.size else np.zeros(1, dtype=np.int32)
+    b0 = F22 if F22.size else np.zeros((1, 1), order="F")
+    b1 = Fp if Fp.size else np.zeros((1, 1), order="F")
+    r = lib().oracle_extend_add(n2, _dp(b0), max(1, n2), _ip(r0), npp, _dp(b1), max(1, npp))
+    if r < 0:
+        raise ValueError(f"oracle_extend_add: bad argument {-r}")
+    return Fp
 
 
 def backward_error(A0, LU, ipiv):

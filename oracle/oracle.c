@@ -26,6 +26,10 @@
  *    BLAS/LAPACK definitions.
  *  - oracle_getrs: the solve with the factors (LAPACK dgetrs steps), the
  *    GETRS composition the paper benchmarks irrTRSM against (L96, L215).
+ *  - oracle_extend_add: the extend-add of a child's Schur complement into
+ *    its parent front (L99 §III-A: "the Schur complement F_{r:22} is added
+ *    into the parent frontal matrix ... this requires a scatter operation"),
+ *    as its plain definition Fp[rel_i, rel_j] += F22[i, j].
  *  - oracle_backward_error: ||PA - LU||_F / (||A||_F * k * eps) (north_star;
  *    SURVEY reading Q11), accumulated in long double.
  */
@@ -335,6 +339,30 @@ int oracle_getrs(int n, int nrhs, const double *LU, int ld, const int *ipiv, dou
     }
 #undef LU_
 #undef B_
+    return 0;
+}
+
+/* ---------------------------------------------------------------------------
+ * Extend-add: the child's n2 x n2 Schur
+ * complement F22 is scattered into its parent front Fp (np x np) through the
+ * index map rel (0-based parent row / column of each child row / column):
+ *     Fp[rel[i], rel[j]] = Fp[rel[i], rel[j]] + F22[i, j]   for all i, j < n2.
+ * Returns 0, or -(argument position) for a bad n2 / ld22 / rel entry / np /
+ * ldp (then Fp is untouched).  Several children of one parent are applied by
+ * calling this once per child, in the caller's order.
+ * ------------------------------------------------------------------------- */
+int oracle_extend_add(int n2, const double *F22, int ld22, const int *rel, int np, double *Fp, int ldp)
+{
+    if (n2 < 0) return -1;
+    if (ld22 < imax(1, n2)) return -3;
+    if (np < 0) return -5;
+    if (ldp < imax(1, np)) return -7;
+    for (int i = 0; i < n2; ++i)
+        if (rel[i] < 0 || rel[i] >= np) return -4;
+    for (int j = 0; j < n2; ++j)
+        for (int i = 0; i < n2; ++i)
+            Fp[(size_t)rel[i] + (size_t)rel[j] * ldp] = Fp[(size_t)rel[i] + (size_t)rel[j] * ldp] +
+                                                        F22[(size_t)i + (size_t)j * ld22];
     return 0;
 }
 
