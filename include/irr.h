@@ -201,6 +201,38 @@ int irr_status_words(int batch, const int *m, const int *n, int *const *ipiv, co
                      unsigned int *words, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_extend_add -- batched extend-add of child Schur complements into their
+ * parent fronts.  PAPER.md L99 §III-A: "After these
+ * operations are applied to front F_r, the Schur complement F_{r:22} is added
+ * into the parent frontal matrix ... this requires a scatter operation";
+ * L102: all fronts of one tree level are handled concurrently.  For child c:
+ *     Fp_c[rel_c[i], rel_c[j]] += F22_c[i, j]     0 <= i, j < n2[c]
+ *  batch        number of children (>= 0)                               (host)
+ *  max_n2       >= every n2[c]; 0 => nothing to do                      (host)
+ *  n2[batch]    order of each child's Schur complement
+ *  F22[batch]   -> column-major n2 x n2 Schur complement (read only), ld22[c]
+ *  rel[batch]   -> int[n2[c]]: 0-based row / column of the parent front that
+ *               the child's row / column i maps to (distinct entries)
+ *  np[batch]    order of the parent front of child c
+ *  Fp[batch]    -> column-major np x np parent front of child c (several
+ *               children may point at the same parent), ldp[c]
+ *  info[batch]  0, or -(argument position) of the first bad per-child value:
+ *               -3 n2 < 0 or > max_n2, -5 ld22 < max(1, n2), -6 a rel entry
+ *               outside [0, np), -7 np < 0, -9 ldp < max(1, np), -4 / -8 NULL
+ *               F22 / Fp with n2 > 0; such a child adds nothing.
+ * The adds are atomic (FP64 reductions in L2): children sharing a parent may
+ * be in one call; an entry hit by one child per call gets exactly
+ * fl(Fp + F22) (bit-identical to a sequential sum), an entry hit by several
+ * children of one call gets their sum in an unspecified order.  Call once per
+ * sibling round (child 0s, then child 1s) for a result independent of
+ * scheduling.  All arrays device memory, caller-owned; asynchronous on
+ * `stream`.  Host errors: -1 batch, -2 max_n2, -(position) for NULL arrays.
+ * ---------------------------------------------------------------------- */
+int irr_extend_add(int batch, int max_n2, const int *n2, const double *const *F22, const int *ld22,
+                   const int *const *rel, const int *np, double *const *Fp, const int *ldp, int *info,
+                   irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * Tuning (tests and experiments; defaults are fixed by measurement and are
  * process-global, not thread-safe).  Keys: "nb" (tier-L panel width, 1..64),
  * "tier_s" (1 = enable the warp-per-matrix tier), "tier_m_max" (max padded

@@ -74,7 +74,7 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 }
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
-                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs"};
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs", "extend_add"};
 
 struct DeviceInfo {
     int sms = 0;
@@ -499,6 +499,26 @@ int irr_status_words(int batch, const int *m, const int *n, int *const *ipiv, co
     int rc = check_device();
     if (rc) return rc;
     launch_status_words(batch, m, n, ipiv, info, words, (cudaStream_t)stream);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+int irr_extend_add(int batch, int max_n2, const int *n2, const double *const *F22, const int *ld22,
+                   const int *const *rel, const int *np, double *const *Fp, const int *ldp, int *info,
+                   irr_stream_t stream) {
+    if (batch < 0) return -1;
+    if (max_n2 < 0) return -2;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!n2) return -3;
+    if (!F22) return -4;
+    if (!ld22) return -5;
+    if (!rel) return -6;
+    if (!np) return -7;
+    if (!Fp) return -8;
+    if (!ldp) return -9;
+    if (!info) return -10;
+    int rc = check_device();
+    if (rc) return rc;
+    launch_extend_add(batch, max_n2, n2, F22, ld22, rel, np, Fp, ldp, info, (cudaStream_t)stream);
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 

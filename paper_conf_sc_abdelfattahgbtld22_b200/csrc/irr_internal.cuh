@@ -42,7 +42,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, K_EXTEND_ADD, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();
@@ -210,6 +210,9 @@ struct GetrfArgs {
 };
 
 // classify.cu
+void launch_extend_add(int batch, int max_n2, const int *n2, const double *const *F22, const int *ld22,
+                       const int *const *rel, const int *np, double *const *Fp, const int *ldp, int *info,
+                       cudaStream_t s);
 void launch_classify(const GetrfArgs &a, int *counters, int *bins, int keep_neg_info, cudaStream_t s);
 void launch_max_dims(int batch, const int *m, const int *n, int *counters, cudaStream_t s);
 

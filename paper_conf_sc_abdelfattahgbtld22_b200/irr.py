@@ -26,7 +26,7 @@ IRR_SUCCESS, IRR_ERR_CUDA, IRR_ERR_WORKSPACE, IRR_ERR_UNSUPPORTED, IRR_ERR_DEVIC
 EXPORTED = (
     "irr_getrf_workspace_size", "irr_getrf", "irr_getrf_partial_workspace_size", "irr_getrf_partial",
     "irr_gemm_workspace_size", "irr_gemm", "irr_trsm_workspace_size", "irr_trsm", "irr_laswp",
-    "irr_getrs_workspace_size", "irr_getrs", "irr_status_words",
+    "irr_getrs_workspace_size", "irr_getrs", "irr_status_words", "irr_extend_add",
     "irr_set_tuning", "irr_get_tuning", "irr_reset_tuning", "irr_launch_count", "irr_version",
     "irr_profile_enable", "irr_profile_collect", "irr_profile_num_classes", "irr_profile_class_name",
 )
@@ -71,6 +71,8 @@ def load(path: str | None = None):
     L.irr_getrs_workspace_size.restype = sz
     L.irr_getrs.argtypes = [i, i, i, i, vp, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
     L.irr_getrs.restype = i
+    L.irr_extend_add.argtypes = [i, i, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+    L.irr_extend_add.restype = i
     L.irr_status_words.argtypes = [i, vp, vp, vp, vp, vp, vp]
     L.irr_status_words.restype = i
     L.irr_set_tuning.argtypes = [C.c_char_p, i]
@@ -152,6 +154,12 @@ def irr_getrs(trans, batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info
     rc = load().irr_getrs(trans, batch, max_n, max_nrhs, _p(n), _p(nrhs), _p(A), _p(lda), _p(ipiv), _p(B),
                           _p(ldb), _p(info), _p(work), _nbytes(work), _stream(stream))
     return _check(rc, "irr_getrs") if check else rc
+
+
+def irr_extend_add(batch, max_n2, n2, F22, ld22, rel, np_, Fp, ldp, info, stream=None, check=True):
+    rc = load().irr_extend_add(batch, max_n2, _p(n2), _p(F22), _p(ld22), _p(rel), _p(np_), _p(Fp), _p(ldp),
+                               _p(info), _stream(stream))
+    return _check(rc, "irr_extend_add") if check else rc
 
 
 def irr_status_words(batch, m, n, ipiv, info, words, stream=None, check=True):
