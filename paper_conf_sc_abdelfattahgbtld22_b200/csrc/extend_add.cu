@@ -21,6 +21,12 @@ constexpr int EA_THREADS = 256;
 constexpr int EA_REL_SMEM = 4096;  // 16 KB of rel entries per CTA
 constexpr int EA_MAX_Y = 64;
 
+// fire-and-forget FP64 reduction (atomicAdd with an unused result compiles to
+// ATOM, whose return the warp waits for: 88% long-scoreboard stalls in ncu)
+__device__ __forceinline__ void red_add_f64(double *p, double v) {
+    asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(p), "d"(v) : "memory");
+}
+
 __global__ void __launch_bounds__(EA_THREADS)
     extend_add_kernel(int max_n2, const int *__restrict__ n2, const double *const *__restrict__ F22,
                       const int *__restrict__ ld22, const int *const *__restrict__ rel, const int *__restrict__ np,
@@ -66,7 +72,7 @@ __global__ void __launch_bounds__(EA_THREADS)
         const int ri = i < EA_REL_SMEM ? srel[i] : __ldg(r + i);
         const int rj = j < EA_REL_SMEM ? srel[j] : __ldg(r + j);
         const double v = __ldg(A + (size_t)i + (size_t)j * l22);
-        atomicAdd(P + (size_t)ri + (size_t)rj * lp, v);
+        red_add_f64(P + (size_t)ri + (size_t)rj * lp, v);
         i += di;
         q += dq;
         if (i >= nc) {
