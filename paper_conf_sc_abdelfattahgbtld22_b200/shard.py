@@ -51,3 +51,33 @@ def merge_status(gathered: np.ndarray, shards) -> np.ndarray:
     for r, idx in enumerate(shards):
         out[idx] = gathered[r, : len(idx)]
     return out
+
+
+def sibling_rounds(parent_of_child) -> list:
+    """Split one tree level's children into rounds for irr_extend_add:
+    round r holds the r-th child (in batch order) of every parent, so no two
+    children of one round share a parent and each call adds at most one
+    contribution per parent entry (bit-identical to the sequential order,
+    include/irr.h).  Returns a list of ascending index arrays."""
+    parent = np.asarray(parent_of_child, dtype=np.int64)
+    if len(parent) == 0:
+        return []
+    order = np.argsort(parent, kind="stable")
+    ps = parent[order]
+    first = np.r_[0, np.nonzero(np.diff(ps))[0] + 1]
+    rank = np.arange(len(ps)) - np.repeat(first, np.diff(np.r_[first, len(ps)]))
+    r_of = np.empty(len(parent), dtype=np.int64)
+    r_of[order] = rank
+    return [np.nonzero(r_of == r)[0] for r in range(int(r_of.max()) + 1)]
+
+
+def shard_level(parent_of_child, n2, parts: int) -> np.ndarray:
+    """Owner rank of each child of one extend-add level: a parent front and
+    all its children stay on one GPU (the scatter needs no exchange), parents
+    LPT-balanced by the bytes their children move (sum of n2^2)."""
+    parent = np.asarray(parent_of_child, dtype=np.int64)
+    if len(parent) == 0:
+        return np.zeros(0, dtype=np.int64)
+    n2 = np.asarray(n2, dtype=np.float64)
+    work = np.bincount(parent, weights=n2 * n2)
+    return lpt_partition(work, parts)[parent]

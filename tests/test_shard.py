@@ -77,3 +77,24 @@ def test_gloo_two_ranks_gather_and_merge():
         assert p.exitcode == 0
     assert merged == list(range(total))           # every matrix's word lands at its global id
     assert tmax == 2.0
+
+
+def test_sibling_rounds_and_level_shard():
+    from paper_conf_sc_abdelfattahgbtld22_b200.shard import shard_level, sibling_rounds
+    import irrgen
+    nps, parent, n2, rel, F22, Fp = irrgen.extend_add_level(2, 50, 64, children_per_parent=3)
+    perm = np.random.default_rng(0).permutation(len(parent))      # children in any order
+    parent, n2 = parent[perm], n2[perm]
+    rounds = sibling_rounds(parent)
+    assert len(rounds) == 3
+    assert sorted(np.concatenate(rounds).tolist()) == list(range(len(parent)))
+    for r in rounds:
+        assert len(np.unique(parent[r])) == len(r)                 # no shared parent in a round
+    # round r holds the r-th occurrence of each parent in batch order
+    for c in range(len(parent)):
+        k = int((parent[:c] == parent[c]).sum())
+        assert c in rounds[k]
+    owner = shard_level(parent, n2, 4)
+    for p in np.unique(parent):
+        assert len(np.unique(owner[parent == p])) == 1              # a parent and its children on one rank
+    assert sibling_rounds([]) == [] and len(shard_level([], [], 2)) == 0
