@@ -24,6 +24,9 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          int *units_off, SlotList sl);
 size_t laswp_smem(int span);
 bool getrs_strip_ok(int max_n1);
+bool getrs_vec_ok(int max_n);
+void launch_getrs_vec(int batch, int max_n, const int *n, const int *nrhs, const double *const *A, const int *lda,
+                      int *const *ipiv, double *const *B, const int *ldb, const int *mask, cudaStream_t s);
 void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *const *F11, const int *ld11,
                         double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
                         int *queue, SlotList sl, cudaStream_t s);
@@ -34,7 +37,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
 // left-block interchanges (6.80 -> 6.53 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -304,6 +307,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "gemm_big")) g_tuning.gemm_big = value ? 1 : 0;
     else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
     else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
+    else if (!strcmp(key, "getrs_vec")) g_tuning.getrs_vec = value ? 1 : 0;
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
     else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
 }
@@ -326,6 +330,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "gemm_big")) return g_tuning.gemm_big;
     if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
     if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
+    if (!strcmp(key, "getrs_vec")) return g_tuning.getrs_vec;
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
     if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) return g_tuning.defer;
     return -1;
@@ -482,6 +487,10 @@ int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *
     if (max_n > 0 && laswp_smem(max_n) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     launch_getrs_validate(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, s);
     if (max_n <= 0 || max_nrhs <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+    if (max_nrhs == 1 && tuning().getrs_vec && getrs_vec_ok(max_n)) {
+        launch_getrs_vec(batch, max_n, n, nrhs, A, lda, ipiv, B, ldb, info, s);  // one RHS: CTA per system
+        return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+    }
     IRR_CUDA_TRY(cudaMemsetAsync(w.counters, 0, CNT_INTS * sizeof(int), s));
     getrs_core(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, w, s);
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;

@@ -117,3 +117,38 @@ def test_getrs_host_argument_errors():
     rc = irr.irr_getrs(irr.IRR_NO_TRANS, -1, 4, 1, FA.n, FA.n, FA.ptr, FA.ld, FA.ipiv, FA.ptr, FA.ld, info, work,
                        check=False)
     assert rc == -2
+
+
+@pytest.mark.parametrize("vec", [1, 0])
+def test_getrs_single_rhs_paths(vec):
+    """max_nrhs == 1: the CTA-per-system kernel (getrs_vec) and the strip path
+    against the oracle; sizes span one 32-column block, ragged tails, > 256
+    rows (several rows per thread) and n = 1."""
+    irr.irr_set_tuning("getrs_vec", vec)
+    rng = np.random.default_rng(23)
+    ns = [1, 2, 31, 32, 33, 64, 100, 257, 300, 513] + [int(v) for v in rng.integers(1, 260, 30)]
+    As = [irrgen.uniform_values(8, g, n, n) for g, n in enumerate(ns)]
+    Bs = [irrgen.uniform_values(9, g, n, 1) for g, n in enumerate(ns)]
+    LUs, ipivs, Xs, st = _solve(As, Bs)
+    assert (st == 0).all()
+    for n, A, B, LU, ip, X in zip(ns, As, Bs, LUs, ipivs, Xs):
+        Xo = oracle.getrs(LU, ip, B)
+        dev = np.abs(X - Xo).max() / max(1e-300, np.abs(Xo).max())
+        assert dev <= 1e-10, f"n={n}: deviation {dev}"
+        res = np.abs(A @ X - B).max() / (np.abs(A).max() * np.abs(X).max() * n * EPS)
+        assert res <= 10.0, f"n={n}: residual {res}"
+
+
+def test_getrs_single_rhs_exact():
+    """Integer X through G1 factors is recovered bit-exactly by the single-RHS kernel."""
+    irr.irr_set_tuning("getrs_vec", 1)
+    ns = [6, 40, 64, 150]
+    As, Xt = [], []
+    for g, n in enumerate(ns):
+        As.append(irrgen.g1_exact(9, 700 + g, n, n)[0])
+        Xt.append(np.asfortranarray(np.random.default_rng(g).integers(-8, 9, size=(n, 1)).astype(np.float64)))
+    Bs = [np.asfortranarray(A @ X) for A, X in zip(As, Xt)]
+    _, _, Xs, st = _solve(As, Bs)
+    assert (st == 0).all()
+    for X, Xg in zip(Xt, Xs):
+        assert np.array_equal(X, Xg)

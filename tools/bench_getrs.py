@@ -35,7 +35,12 @@ def main():
     ap.add_argument("--nrhs", type=int, default=0)
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--seed", type=int, default=3)
+    ap.add_argument("--tune", action="append", default=[], help="irr_set_tuning key=value")
     a = ap.parse_args()
+    from paper_conf_sc_abdelfattahgbtld22_b200 import irr
+    for kv in a.tune:
+        k, v = kv.split("=")
+        irr.irr_set_tuning(k, int(v))
     rng = np.random.default_rng(a.seed)
     n = rng.integers(1, a.n_max + 1, size=a.batch)
     nrhs = n if a.nrhs == 0 else np.full(a.batch, a.nrhs)
@@ -63,7 +68,7 @@ def main():
     peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
     gf = flops / (ms * 1e-3) / 1e9
     gbs = byts / (ms * 1e-3) / 1e9
-    print(json.dumps({"kernel": "getrs", "batch": a.batch, "n_max": a.n_max, "nrhs": a.nrhs or "n_i",
+    print(json.dumps({"kernel": "getrs", "batch": a.batch, "n_max": a.n_max, "nrhs": a.nrhs or "n_i", "tune": a.tune,
                       "ms_per_solve": round(ms, 4), "gflops": round(gf, 1), "fp64_frac": round(gf * 1e9 / FP64_PEAK, 3),
                       "achieved_gbs": round(gbs, 1), "hbm_frac": round(gbs / peak, 3), "alg_flops": flops,
                       "alg_bytes": byts}))
