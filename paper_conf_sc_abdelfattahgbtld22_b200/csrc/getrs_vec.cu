@@ -9,8 +9,9 @@
 //   * b and ipiv staged in shared memory, the interchanges applied in order by
 //     one thread (smem only);
 //   * substitution in 32-column blocks: warp 0 solves the 32 x 32 diagonal
-//     triangle with x in registers (lane i = row i of the block, shuffles
-//     broadcast the solved entry), then every thread updates its rows below
+//     triangle (staged in shared memory one block ahead) with x in registers
+//     (lane i = row i of the block, shuffles broadcast the solved entry),
+//     then every thread updates its rows below
 //     (L) / above (U) with the block's 32 columns -- for a fixed column,
 //     consecutive threads read consecutive rows (coalesced, each element of
 //     L\U read exactly once).  Two barriers per 32 columns.
@@ -20,8 +21,11 @@
 namespace irr {
 
 constexpr int GV_THREADS = 128;
+#ifndef GV_MINB
+#define GV_MINB 8  // 64 registers: 8 CTAs (32 warps) per SM
+#endif
 
-__global__ void __launch_bounds__(GV_THREADS, 4)
+__global__ void __launch_bounds__(GV_THREADS, GV_MINB)
     getrs_vec_kernel(const int *__restrict__ n_, const int *__restrict__ nrhs_, const double *const *__restrict__ A,
                      const int *__restrict__ lda_, int *const *__restrict__ ipiv_, double *const *__restrict__ B,
                      const int *__restrict__ ldb_, const int *__restrict__ mask) {
@@ -50,20 +54,28 @@ __global__ void __launch_bounds__(GV_THREADS, 4)
             }
         }
     __syncthreads();
-    // forward: L unit lower
+    // forward: L unit lower.  The 32 x 32 diagonal tile of the next block is
+    // staged in shared memory by all threads together with the current
+    // block's trailing update (both only read L\U), so warp 0's dependent
+    // chain reads it from shared memory and the registers stay low.
+    __shared__ double tri[32 * 33];
+    auto stage = [&](int jb, int w, bool lower) {
+        for (int e = t; e < 32 * 32; e += GV_THREADS) {
+            const int r = e & 31, k = e >> 5;
+            const bool in = r < w && k < w && (lower ? k < r : k >= r);
+            tri[r * 33 + k] = in ? LU[(size_t)(jb + r) + (size_t)(jb + k) * lda] : 0.0;
+        }
+    };
+    stage(0, min(32, n), true);
+    __syncthreads();
     for (int jb = 0; jb < n; jb += 32) {
         const int w = min(32, n - jb);
         if (warp == 0) {
-            // the lane's row of the 32 x 32 diagonal block, loaded up front
-            double lr[32];
-#pragma unroll
-            for (int k = 0; k < 32; ++k)
-                lr[k] = (lane < w && k < lane) ? LU[(size_t)(jb + lane) + (size_t)(jb + k) * lda] : 0.0;
             double xi = lane < w ? x[jb + lane] : 0.0;
 #pragma unroll
             for (int k = 0; k < 31; ++k) {
                 const double xk = __shfl_sync(0xffffffffu, xi, k);
-                xi -= lr[k] * xk;  // lr[k] = 0 unless k < lane < w
+                xi -= tri[lane * 33 + k] * xk;  // 0 unless k < lane < w
             }
             if (lane < w) x[jb + lane] = xi;
         }
@@ -75,24 +87,23 @@ __global__ void __launch_bounds__(GV_THREADS, 4)
             for (int k = 0; k < w; ++k) acc -= col[(size_t)k * lda] * x[jb + k];
             x[i] = acc;
         }
+        if (jb + 32 < n) stage(jb + 32, min(32, n - jb - 32), true);
         __syncthreads();
     }
     // backward: U upper, non-unit; blocks from the bottom
     const int nblk = (n + 31) / 32;
+    stage((nblk - 1) * 32, n - (nblk - 1) * 32, false);
+    __syncthreads();
     for (int q = nblk - 1; q >= 0; --q) {
         const int jb = q * 32, w = min(32, n - jb);
         if (warp == 0) {
-            double ur[32];
-#pragma unroll
-            for (int k = 0; k < 32; ++k)
-                ur[k] = (lane < w && k >= lane && k < w) ? LU[(size_t)(jb + lane) + (size_t)(jb + k) * lda] : 0.0;
             double xi = lane < w ? x[jb + lane] : 0.0;
 #pragma unroll
             for (int k = 31; k >= 0; --k) {
                 if (k < w) {
-                    if (lane == k) xi = xi / ur[k];
+                    if (lane == k) xi = xi / tri[k * 33 + k];
                     const double xk = __shfl_sync(0xffffffffu, xi, k);
-                    if (lane < k) xi -= ur[k] * xk;
+                    if (lane < k) xi -= tri[lane * 33 + k] * xk;
                 }
             }
             if (lane < w) x[jb + lane] = xi;
@@ -105,6 +116,7 @@ __global__ void __launch_bounds__(GV_THREADS, 4)
             for (int k = 0; k < w; ++k) acc -= col[(size_t)k * lda] * x[jb + k];
             x[i] = acc;
         }
+        if (q > 0) stage(jb - 32, 32, false);
         __syncthreads();
     }
     for (int i = t; i < n; i += GV_THREADS) b[i] = x[i];
