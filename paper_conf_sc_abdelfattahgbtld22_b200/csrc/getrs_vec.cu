@@ -21,6 +21,10 @@
 namespace irr {
 
 constexpr int GV_THREADS = 128;
+#ifndef GV_UNROLL
+#define GV_UNROLL 8  // loads in flight per thread in the column updates
+#endif
+constexpr int kGvUnroll = GV_UNROLL;
 #ifndef GV_MINB
 #define GV_MINB 8  // 64 registers: 8 CTAs (32 warps) per SM
 #endif
@@ -83,7 +87,7 @@ __global__ void __launch_bounds__(GV_THREADS, GV_MINB)
         for (int i = jb + w + t; i < n; i += GV_THREADS) {
             double acc = x[i];
             const double *col = LU + (size_t)i + (size_t)jb * lda;
-#pragma unroll 8
+#pragma unroll kGvUnroll
             for (int k = 0; k < w; ++k) acc -= col[(size_t)k * lda] * x[jb + k];
             x[i] = acc;
         }
@@ -112,7 +116,7 @@ __global__ void __launch_bounds__(GV_THREADS, GV_MINB)
         for (int i = t; i < jb; i += GV_THREADS) {
             double acc = x[i];
             const double *col = LU + (size_t)i + (size_t)jb * lda;
-#pragma unroll 8
+#pragma unroll kGvUnroll
             for (int k = 0; k < w; ++k) acc -= col[(size_t)k * lda] * x[jb + k];
             x[i] = acc;
         }
