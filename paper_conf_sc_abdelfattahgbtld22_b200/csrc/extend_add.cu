@@ -20,6 +20,9 @@ namespace irr {
 constexpr int EA_THREADS = 256;
 constexpr int EA_REL_SMEM = 4096;  // 16 KB of rel entries per CTA
 constexpr int EA_MAX_Y = 64;
+#ifndef EA_PER_CTA
+#define EA_PER_CTA 16384  // target child elements per CTA of the largest child
+#endif
 
 // fire-and-forget FP64 reduction (atomicAdd with an unused result compiles to
 // ATOM, whose return the warp waits for: 88% long-scoreboard stalls in ncu)
@@ -82,14 +85,71 @@ __global__ void __launch_bounds__(EA_THREADS)
     }
 }
 
+// Small children (max_n2 <= 64): one warp per child, 8 children per CTA, rel
+// held in two registers per lane and broadcast by shuffles -- no shared
+// memory stage and no CTA barrier per child (the CTA-per-child kernel spends
+// its time on that prologue when a child has only a few hundred elements).
+constexpr int EA_SMALL_N2 = 64;
+__global__ void __launch_bounds__(256)
+    extend_add_small_kernel(int batch, int max_n2, const int *__restrict__ n2, const double *const *__restrict__ F22,
+                            const int *__restrict__ ld22, const int *const *__restrict__ rel,
+                            const int *__restrict__ np, double *const *__restrict__ Fp, const int *__restrict__ ldp,
+                            int *__restrict__ info) {
+    const int lane = threadIdx.x & 31;
+    const int c = blockIdx.x * 8 + (threadIdx.x >> 5);
+    if (c >= batch) return;
+    const int nc = n2[c], npc = np[c], l22 = ld22[c], lp = ldp[c];
+    int code = 0;
+    if (nc < 0 || nc > max_n2) code = -3;
+    else if (l22 < max(1, nc)) code = -5;
+    else if (npc < 0) code = -7;
+    else if (lp < max(1, npc)) code = -9;
+    else if (nc > 0 && !F22[c]) code = -4;
+    else if (nc > 0 && !Fp[c]) code = -8;
+    else if (nc > 0 && !rel[c]) code = -6;
+    if (code != 0 || nc == 0) {
+        if (lane == 0) info[c] = code;
+        return;
+    }
+    const int *r = rel[c];
+    const int r0 = lane < nc ? __ldg(r + lane) : 0;
+    const int r1 = lane + 32 < nc ? __ldg(r + lane + 32) : 0;
+    const bool bad = __any_sync(0xffffffffu, r0 < 0 || r0 >= npc || r1 < 0 || r1 >= npc);
+    if (lane == 0) info[c] = bad ? -6 : 0;
+    if (bad) return;
+    const double *A = F22[c];
+    double *P = Fp[c];
+    const int total = nc * nc;
+    int j = lane / nc, i = lane - j * nc;
+    const int dj = 32 / nc, di = 32 - dj * nc;
+    for (int e = lane; e - lane < total; e += 32) {  // whole warp iterates (shuffles)
+        const int a0 = __shfl_sync(0xffffffffu, r0, i & 31), a1 = __shfl_sync(0xffffffffu, r1, i & 31);
+        const int b0 = __shfl_sync(0xffffffffu, r0, j & 31), b1 = __shfl_sync(0xffffffffu, r1, j & 31);
+        if (e < total) {
+            const int ri = i < 32 ? a0 : a1, rj = j < 32 ? b0 : b1;
+            red_add_f64(P + (size_t)ri + (size_t)rj * lp, __ldg(A + (size_t)i + (size_t)j * l22));
+        }
+        i += di;
+        j += dj;
+        if (i >= nc) {
+            i -= nc;
+            ++j;
+        }
+    }
+}
+
 void launch_extend_add(int batch, int max_n2, const int *n2, const double *const *F22, const int *ld22,
                        const int *const *rel, const int *np, double *const *Fp, const int *ldp, int *info,
                        cudaStream_t s) {
     // about 16 K elements per CTA of the largest child, at most EA_MAX_Y column groups
     long long per = (long long)max_n2 * max_n2;
-    int Y = (int)std::min<long long>(EA_MAX_Y, std::max<long long>(1, (per + 16383) / 16384));
+    int Y = (int)std::min<long long>(EA_MAX_Y, std::max<long long>(1, (per + EA_PER_CTA - 1) / EA_PER_CTA));
     Y = std::max(1, std::min(Y, std::max(1, max_n2)));
     KScope k(K_EXTEND_ADD, s);
+    if (max_n2 <= EA_SMALL_N2) {
+        extend_add_small_kernel<<<(batch + 7) / 8, 256, 0, s>>>(batch, max_n2, n2, F22, ld22, rel, np, Fp, ldp, info);
+        return;
+    }
     extend_add_kernel<<<dim3(batch, Y), EA_THREADS, 0, s>>>(max_n2, n2, F22, ld22, rel, np, Fp, ldp, info);
 }
 

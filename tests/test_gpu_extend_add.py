@@ -43,10 +43,13 @@ def _oracle(lvl, order):
     return out
 
 
+@pytest.mark.parametrize("np_max", [300, 85])
 @pytest.mark.parametrize("ld_extra", [0, 3])
-def test_sibling_rounds_bit_exact(ld_extra):
-    """Round r = the r-th child of every parent: one add per entry per call."""
-    lvl = irrgen.extend_add_level(11, 40, 300)
+def test_sibling_rounds_bit_exact(ld_extra, np_max):
+    """Round r = the r-th child of every parent: one add per entry per call.
+    np_max 85 keeps every child <= 64 (the warp-per-child kernel, both rel
+    registers in use); 300 takes the CTA-per-child kernel."""
+    lvl = irrgen.extend_add_level(11, 40, np_max)
     nps, parent, n2, rel, F22, Fp = lvl
     L = Level(*lvl, ld_extra=ld_extra)
     kids = np.arange(len(parent))
