@@ -24,9 +24,10 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          int *units_off, SlotList sl);
 size_t laswp_smem(int span);
 bool getrs_strip_ok(int max_n1);
-bool getrs_vec_ok(int max_n);
-void launch_getrs_vec(int batch, int max_n, const int *n, const int *nrhs, const double *const *A, const int *lda,
-                      int *const *ipiv, double *const *B, const int *ldb, const int *mask, cudaStream_t s);
+bool getrs_vec_ok(int max_n, int max_nrhs);
+void launch_getrs_vec(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs, const double *const *A,
+                      const int *lda, int *const *ipiv, double *const *B, const int *ldb, const int *mask,
+                      cudaStream_t s);
 void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *const *F11, const int *ld11,
                         double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
                         int *queue, SlotList sl, cudaStream_t s);
@@ -487,8 +488,9 @@ int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *
     if (max_n > 0 && laswp_smem(max_n) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     launch_getrs_validate(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, s);
     if (max_n <= 0 || max_nrhs <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
-    if (max_nrhs == 1 && tuning().getrs_vec && getrs_vec_ok(max_n)) {
-        launch_getrs_vec(batch, max_n, n, nrhs, A, lda, ipiv, B, ldb, info, s);  // one RHS: CTA per system
+    if (tuning().getrs_vec && getrs_vec_ok(max_n, max_nrhs)) {
+        // few right-hand sides (<= GV_MAX_NRHS): CTA per system
+        launch_getrs_vec(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, s);
         return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
     }
     IRR_CUDA_TRY(cudaMemsetAsync(w.counters, 0, CNT_INTS * sizeof(int), s));

@@ -32,7 +32,7 @@ struct Tuning {
     int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
     int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
     int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)
-    int getrs_vec;       // 1: irr_getrs with max_nrhs == 1 by the CTA-per-system kernel (getrs_vec.cu)
+    int getrs_vec;       // 1: irr_getrs with max_nrhs <= 4 by the CTA-per-system kernel (getrs_vec.cu)
 };
 Tuning &tuning();
 

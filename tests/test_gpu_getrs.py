@@ -152,3 +152,24 @@ def test_getrs_single_rhs_exact():
     assert (st == 0).all()
     for X, Xg in zip(Xt, Xs):
         assert np.array_equal(X, Xg)
+
+
+@pytest.mark.parametrize("max_r", [2, 3, 8])
+def test_getrs_few_rhs_vec(max_r):
+    """Few right-hand sides: the CTA-per-system kernel with R = 2 / 4 RHS
+    columns (ragged nrhs_i < R, nrhs_i = 0 skipped; max_r 8 is above
+    GV_MAX_NRHS and takes the strip path) against the oracle."""
+    irr.irr_set_tuning("getrs_vec", 1)
+    rng = np.random.default_rng(31 + max_r)
+    ns = [1, 31, 33, 64, 200, 300] + [int(v) for v in rng.integers(1, 200, 20)]
+    rs = [max_r, 0] + [int(v) for v in rng.integers(1, max_r + 1, len(ns) - 2)]
+    As = [irrgen.uniform_values(12, g, n, n) for g, n in enumerate(ns)]
+    Bs = [irrgen.uniform_values(13, g, n, r) for g, (n, r) in enumerate(zip(ns, rs))]
+    LUs, ipivs, Xs, st = _solve(As, Bs)
+    assert (st == 0).all()
+    for n, r, A, B, LU, ip, X in zip(ns, rs, As, Bs, LUs, ipivs, Xs):
+        if r == 0:
+            continue
+        Xo = oracle.getrs(LU, ip, B)
+        dev = np.abs(X - Xo).max() / max(1e-300, np.abs(Xo).max())
+        assert dev <= 1e-10, f"n={n} r={r}: deviation {dev}"
