@@ -176,8 +176,9 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
  *               max_n / max_nrhs (host) bound them (<= 0: computed, one sync).
  *  A, lda, ipiv, B, ldb   device pointer / int arrays as for irr_getrf.
  *  info         int[batch] (output): 0, or -(argument position) for a bad
- *               n (-5), nrhs (-6), NULL A_i (-7), lda (-8), NULL ipiv_i (-9),
- *               NULL B_i (-10) or ldb (-11); those systems are skipped.  No
+ *               n (-5), nrhs (-6), NULL A_i (-7), lda (-8), NULL ipiv_i or a
+ *               pivot ipiv_i[k] outside [k+1, n_i] (-9), NULL B_i (-10) or
+ *               ldb (-11); those systems are skipped.  No
  *               singularity check (LAPACK dgetrs): a zero U_ii gives IEEE
  *               inf / NaN in X_i.
  *  work         >= irr_getrs_workspace_size(batch) bytes (caller-owned).

@@ -19,6 +19,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "oracle.c")
+_CHECK = os.path.join(_HERE, "check.c")   # batched parity checker (calls the oracle; no method arithmetic)
 _lib = None
 
 CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC", "-std=c11"]
@@ -26,9 +27,10 @@ CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "
 
 def build(force: bool = False) -> str:
     """Compile oracle.c -> liboracle.so (gcc, no FMA contraction, no fast-math)."""
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+    newest = max(os.path.getmtime(_SRC), os.path.getmtime(_CHECK))
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < newest:
         tmp = _SO + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, "-lm"])
+        subprocess.check_call(["gcc", *CFLAGS, "-o", tmp, _SRC, _CHECK, "-lm"])
         os.replace(tmp, _SO)
     return _SO
 
@@ -57,6 +59,11 @@ def lib():
         L.oracle_backward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
         L.oracle_backward_error.restype = C.c_double
         L.oracle_num_threads.restype = C.c_int
+        vp = C.c_void_p
+        L.check_getrf_batch.argtypes = [C.c_int, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_int]
+        L.check_getrf_batch.restype = C.c_int
+        L.check_partial_batch.argtypes = [C.c_int, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_int]
+        L.check_partial_batch.restype = C.c_int
         _lib = L
     return _lib
 
@@ -232,3 +239,49 @@ def backward_error(A0, LU, ipiv):
 
 def num_threads() -> int:
     return lib().oracle_num_threads()
+
+
+# ---------------------------------------------------------------------------
+# Batched parity records (check.c): every matrix of a packed batch against the
+# oracle, without a Python object per matrix.  Field names of one record:
+GETRF_FIELDS = ("info_o", "ipiv_eq", "first_diff", "be", "dl", "du", "rho", "lmax", "exact")
+PARTIAL_FIELDS = GETRF_FIELDS + ("f21_same", "d12", "d22", "front_exact")
+
+
+def _ptrs(flat, offsets, itemsize):
+    """Device-style pointer array (uint64) into a flat host buffer."""
+    base = flat.ctypes.data
+    return (np.uint64(base) + np.asarray(offsets, dtype=np.uint64) * np.uint64(itemsize)).astype(np.uint64)
+
+
+def _i32(x):
+    return np.ascontiguousarray(x, dtype=np.int32)
+
+
+def check_getrf_packed(m, n, A0, ld0, off0, LU, ld, off, ipiv, ipiv_off, info, nthreads: int = 0):
+    """Records (batch x len(GETRF_FIELDS)) comparing the GPU results (LU, ipiv,
+    info in packed host buffers) with oracle_getrf of the originals A0."""
+    m, n, ld0, ld, info = _i32(m), _i32(n), _i32(ld0), _i32(ld), _i32(info)
+    b = len(m)
+    pa, pl = _ptrs(A0, off0, 8), _ptrs(LU, off, 8)
+    pi = _ptrs(ipiv, ipiv_off, 4)
+    out = np.empty((max(1, b), len(GETRF_FIELDS)))
+    nf = lib().check_getrf_batch(b, m.ctypes.data, n.ctypes.data, pa.ctypes.data, ld0.ctypes.data, pl.ctypes.data,
+                                 ld.ctypes.data, pi.ctypes.data, info.ctypes.data, out.ctypes.data, nthreads)
+    assert nf == len(GETRF_FIELDS)
+    return out[:b]
+
+
+def check_partial_packed(n1, n2, F0, ld0, off0, Fg, ld, off, ipiv, ipiv_off, info, nthreads: int = 0):
+    """Records (batch x len(PARTIAL_FIELDS)) for fronts stored as one nf x nf
+    block each (nf = n1 + n2), GPU results against oracle_getrf_partial."""
+    n1, n2, ld0, ld, info = _i32(n1), _i32(n2), _i32(ld0), _i32(ld), _i32(info)
+    b = len(n1)
+    pa, pf = _ptrs(F0, off0, 8), _ptrs(Fg, off, 8)
+    pi = _ptrs(ipiv, ipiv_off, 4)
+    out = np.empty((max(1, b), len(PARTIAL_FIELDS)))
+    nf = lib().check_partial_batch(b, n1.ctypes.data, n2.ctypes.data, pa.ctypes.data, ld0.ctypes.data,
+                                   pf.ctypes.data, ld.ctypes.data, pi.ctypes.data, info.ctypes.data,
+                                   out.ctypes.data, nthreads)
+    assert nf == len(PARTIAL_FIELDS)
+    return out[:b]

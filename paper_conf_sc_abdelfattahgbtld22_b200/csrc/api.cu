@@ -7,6 +7,7 @@
 // (P:L167, L179).
 #include <cstring>
 #include <cstdlib>
+#include <map>
 #include <mutex>
 #include <vector>
 
@@ -102,6 +103,20 @@ static const DeviceInfo *device_info() {
         d.smem_optin = p.sharedMemPerBlockOptin;
     }
     return &d;
+}
+
+cudaError_t smem_optin_fn(const void *func, size_t bytes) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    static std::mutex mu;
+    static std::map<std::pair<const void *, int>, size_t> done;
+    std::lock_guard<std::mutex> lk(mu);
+    size_t &have = done[{func, dev}];
+    if (have >= bytes) return cudaSuccess;
+    e = cudaFuncSetAttribute(func, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e == cudaSuccess) have = bytes;
+    return e;
 }
 
 int num_sms() {

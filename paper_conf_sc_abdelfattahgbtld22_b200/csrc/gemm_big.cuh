@@ -291,12 +291,7 @@ struct SizeFilter {
 
 template <class Prob, int TA, int TB>
 inline void xgemm_launch_t(const Prob &P, int cnt, const int *cnt_ptr, const int *tile_off, cudaStream_t s) {
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(xgemm_sched_kernel<Prob, TA, TB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)BIG_SMEM);
-        attr = true;
-    }
+    smem_optin(xgemm_sched_kernel<Prob, TA, TB>, BIG_SMEM);
     xgemm_sched_kernel<Prob, TA, TB><<<num_sms(), X_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
 }
 

@@ -504,11 +504,7 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_grid_kernel(Prob P, int count, i
 // opt-in to > 48 KB dynamic shared memory once per kernel instantiation
 template <class K>
 inline void gemm_smem_optin(K kernel) {
-    static bool done = false;
-    if (!done) {
-        cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)GEMM_SMEM);
-        done = true;
-    }
+    smem_optin(kernel, GEMM_SMEM);
 }
 
 }  // namespace irr

@@ -350,11 +350,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
                         double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
                         int *queue, SlotList sl, cudaStream_t s) {
     GsArgs g{batch, n1, n2, F11, ld11, F12, ld12, ipiv, info};
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(getrs_strip_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)GS_SMEM);
-        attr = true;
-    }
+    smem_optin(getrs_strip_kernel, GS_SMEM);
     {
         KScope k(K_GEMM_SCAN, s);
         scan_units_kernel<GsUnits><<<1, 1024, 0, s>>>(GsUnits{g}, sl, batch, units_off);

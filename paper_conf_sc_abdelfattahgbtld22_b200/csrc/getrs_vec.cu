@@ -174,8 +174,8 @@ bool getrs_vec_ok(int max_n, int max_nrhs) {
 template <int R>
 static void launch_r(int batch, size_t smem, const int *n, const int *nrhs, const double *const *A, const int *lda,
                      int *const *ipiv, double *const *B, const int *ldb, const int *mask, cudaStream_t s) {
-    if (smem > 48 * 1024)
-        cudaFuncSetAttribute(getrs_vec_kernel<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    // always: the static tri tile counts against the default 48 KB as well
+    smem_optin(getrs_vec_kernel<R>, smem);
     getrs_vec_kernel<R><<<batch, GV_THREADS, smem, s>>>(n, nrhs, A, lda, ipiv, B, ldb, mask);
 }
 

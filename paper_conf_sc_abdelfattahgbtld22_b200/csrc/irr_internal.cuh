@@ -268,6 +268,15 @@ void launch_status_words(int batch, const int *m, const int *n, int *const *ipiv
                          cudaStream_t s);
 
 int num_sms();
+
+// Raise a kernel's dynamic shared-memory limit to >= `bytes` on the CURRENT
+// device (the attribute is per device).  Cached per (kernel, device) under a
+// lock, so repeated launches cost a map lookup; never called on a kernel path.
+cudaError_t smem_optin_fn(const void *func, size_t bytes);
+template <class K>
+inline cudaError_t smem_optin(K *kernel, size_t bytes) {
+    return smem_optin_fn(reinterpret_cast<const void *>(kernel), bytes);
+}
 }  // namespace irr
 
 #define IRR_CUDA_TRY(x)                                  \

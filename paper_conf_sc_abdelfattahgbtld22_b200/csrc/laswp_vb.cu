@@ -165,11 +165,7 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
     LaswpArgs g{max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, mask, (max_n + LS_COLS - 1) / LS_COLS};
     size_t smem = laswp_smem(k2 - k1);
     if (units_off) {
-        static size_t attr = 0;
-        if (smem > 48 * 1024 && smem > attr) {
-            cudaFuncSetAttribute(laswp_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            attr = smem;
-        }
+        smem_optin(laswp_kernel<true>, smem);
         {
             KScope k(K_GEMM_SCAN, s);
             scan_units_kernel<LaswpUnits><<<1, 1024, 0, s>>>(LaswpUnits{g}, sl, batch, units_off);
@@ -178,11 +174,7 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
         laswp_kernel<true><<<num_sms() * 4, LS_NT, smem, s>>>(g, sl, units_off);
         return;
     }
-    static size_t attr = 0;
-    if (smem > 48 * 1024 && smem > attr) {
-        cudaFuncSetAttribute(laswp_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = smem;
-    }
+    smem_optin(laswp_kernel<false>, smem);
     long long total = (long long)batch * g.chunks;
     int grid = num_sms() * 4;
     if (total < grid) grid = (int)total;

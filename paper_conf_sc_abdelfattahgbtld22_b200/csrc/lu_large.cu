@@ -945,14 +945,10 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     const int nb = clamp_nb(tuning().nb);
     const size_t region = l1_region_bytes(nb);
     const size_t smem = region + (size_t)(nb * (nb - 1) / 2 + 2) * sizeof(double);
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaFuncSetAttribute(lu_l1_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaFuncSetAttribute(lu_l1_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaFuncSetAttribute(lu_l1_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        cudaFuncSetAttribute(lu_l1_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = smem;
-    }
+    smem_optin(lu_l1_kernel<true, false>, smem);
+    smem_optin(lu_l1_kernel<false, false>, smem);
+    smem_optin(lu_l1_kernel<true, true>, smem);
+    smem_optin(lu_l1_kernel<false, true>, smem);
     int per_sm = tuning().l1_ctas_per_sm;
     if (per_sm < 1 || per_sm > 3) per_sm = 3;
     int grid = num_sms() * per_sm;
@@ -960,12 +956,8 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     KScope k(K_LU_L1, s);
     if (tuning().l1_rowmap && nb <= 32 && tuning().l1_rows <= L1_MAX_ROWS) {
         const size_t smem_map = smem + (size_t)L1_MAX_ROWS * sizeof(int);
-        static size_t attr_map = 0;
-        if (smem_map > attr_map) {
-            cudaFuncSetAttribute(lu_l1map_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_map);
-            cudaFuncSetAttribute(lu_l1map_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_map);
-            attr_map = smem_map;
-        }
+        smem_optin(lu_l1map_kernel<true>, smem_map);
+        smem_optin(lu_l1map_kernel<false>, smem_map);
         if (tuning().l1_dmma)
             lu_l1map_kernel<true><<<grid, L1_NT, smem_map, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
                                                                 tuning().phase_timing);
@@ -999,20 +991,12 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     if (smem_rows > cap_rows) smem_rows = cap_rows;
     if (smem_rows > a.max_m) smem_rows = a.max_m;
     size_t psmem = (size_t)((smem_rows | 1) + 1) * nb * sizeof(double);
-    static size_t attr_max = 0;
-    if (psmem > attr_max) {
-        cudaFuncSetAttribute(panel_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem);
-        attr_max = psmem;
-    }
+    smem_optin(panel_kernel, psmem);
     const int sms = num_sms();
     int grid_p = sms * 2;
     if (grid_p > a.batch) grid_p = a.batch;
     const size_t pw_smem = sizeof(PanelWinSmem<PW_NT / 32>);
-    static bool pw_attr = false;
-    if (!pw_attr) {
-        cudaFuncSetAttribute(panel_win_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)pw_smem);
-        pw_attr = true;
-    }
+    smem_optin(panel_win_kernel, pw_smem);
     int grid_w = sms * 2;
     if (grid_w > a.batch) grid_w = a.batch;
     const int chunks_per = (a.max_n + SW_COLS - 1) / SW_COLS;
@@ -1020,33 +1004,21 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     int grid_s = sms * 8;
     if (grid_s > sw_items) grid_s = (int)sw_items;
     const size_t sw_smem = (size_t)(nb * (nb + 1) + 2 * nb * (SW_COLS + 1)) * sizeof(double);
-    static size_t sw_attr = 0;
-    if (sw_smem > 48 * 1024 && sw_smem > sw_attr) {
-        cudaFuncSetAttribute(swap_trsm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sw_smem);
-        sw_attr = sw_smem;
-    }
+    smem_optin(swap_trsm_kernel, sw_smem);
     const int *listL = bins + (size_t)BIN_L * a.batch;
     const bool fused = tu.panel_win && tu.strip && a.max_m <= 8 * PW_NT;
     unsigned long long *ph = tu.phase_timing ? reinterpret_cast<unsigned long long *>(counters + CNT_PHASE0) : nullptr;
     const int st_chunks = (a.max_n + ST_COLS - 1) / ST_COLS;
     const size_t st_smem = strip_smem_bytes(nb);
     if (fused) {
-        static size_t st_attr[2] = {0, 0};
-        if (st_smem > st_attr[tu.dmma ? 1 : 0]) {
-            if (tu.dmma) cudaFuncSetAttribute(strip_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)st_smem);
-            else cudaFuncSetAttribute(strip_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)st_smem);
-            st_attr[tu.dmma ? 1 : 0] = st_smem;
-        }
+        if (tu.dmma) smem_optin(strip_kernel<true>, st_smem);
+        else smem_optin(strip_kernel<false>, st_smem);
     }
     // deferred left-block interchanges (strip path only): one pass at the end
     const size_t lsw_smem = (size_t)LSW_BUF * sizeof(double) + 2 * (size_t)a.max_m * sizeof(int);
     const bool defer = fused && tu.defer && lsw_smem <= 200 * 1024;
     if (defer) {
-        static size_t lsw_attr = 0;
-        if (lsw_smem > 48 * 1024 && lsw_smem > lsw_attr) {
-            cudaFuncSetAttribute(left_swaps_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)lsw_smem);
-            lsw_attr = lsw_smem;
-        }
+        smem_optin(left_swaps_kernel, lsw_smem);
     }
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {

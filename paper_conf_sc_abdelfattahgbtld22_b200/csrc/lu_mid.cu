@@ -154,16 +154,13 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
         tuning().phase_timing ? reinterpret_cast<unsigned long long *>(const_cast<int *>(counters) + CNT_PHASE0)
                               : nullptr;
     if (per_sm >= 4) {
-        static size_t attr = 0;
-        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<128, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        smem_optin(lu_mid_kernel<128, 4>, smem);
         lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin, ph);
     } else if (per_sm >= 2) {
-        static size_t attr = 0;
-        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        smem_optin(lu_mid_kernel<256, 2>, smem);
         lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
     } else {
-        static size_t attr = 0;
-        if (smem > attr) { cudaFuncSetAttribute(lu_mid_kernel<256, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem); attr = smem; }
+        smem_optin(lu_mid_kernel<256, 1>, smem);
         lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
     }
 }

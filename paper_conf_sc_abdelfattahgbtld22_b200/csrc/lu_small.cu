@@ -57,7 +57,7 @@ template <int NC>
 struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 stores in every warp's slot
     double L[NC * 32];             // L[k*32 + lane]: multiplier of the row held by `lane` at step k
     double U[s_uoff<NC>(NC) + NC];  // row k of U (n-k values) at s_uoff(k), + overflow pad
-    double rcp[2];                 // reciprocal of the pivot, published with the pivot row (0: divide)
+    double rcp[2];                 // reciprocal of the pivot of step k in rcp[k & 1] (0: divide)
 };
 static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<16>) % 16 == 0 &&
                   sizeof(SmallWarpSmem<8>) % 16 == 0,
@@ -66,7 +66,7 @@ static_assert(s_uoff<32>(32) == 544 && s_uoff<32>(3) == 94, "packed U offsets");
 
 template <int NC, int W>
 __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, bool valid,
-                                       int lane, SmallWarpSmem<NC> &sm) {
+                                       int lane, int n, SmallWarpSmem<NC> &sm) {
     const bool cand = valid && pos >= k;
     // every lane's reciprocal of its own candidate, off the critical path of
     // the pivot search; the winner publishes its one
@@ -86,16 +86,21 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
     const int w = __ffs(wm) - 1;
     const int pmin = __shfl_sync(FULL, pos, w);
     // ---- the pivot row is row k of U: publish it where the output reads it
+    // Row k holds n - k values within its capacity NC - (k & ~1): the pairs
+    // c < n - k are stored (the odd tail's partner slot is still inside the
+    // row), so no step writes into another row's region.
     double *urow = sm.U + s_uoff<NC>(k);
+    const int rem = n - k;
     if (lane == w) {
 #pragma unroll
-        for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
-        sm.rcp[0] = myr;
+        for (int c = 0; c < W; c += 2)
+            if (c < rem) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
+        sm.rcp[k & 1] = myr;
     }
     if (lane == k) my_piv = pmin + 1;
     __syncwarp();
     const double pv = urow[0];
-    const double rc = sm.rcp[0];
+    const double rc = sm.rcp[k & 1];
     // ---- interchange = relabel positions
     if (pos == k) pos = pmin;
     if (lane == w) pos = k;
@@ -115,7 +120,10 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
         double uu[CH];
 #pragma unroll
         for (int q = 0; q < CH; q += 2) {
-            const double2 v = *reinterpret_cast<const double2 *>(urow + e0 + q);
+            // only this row's own slots are read (the pairs past n - k are
+            // padding columns >= n: zeros, never part of the output)
+            const double2 v = (e0 + q < rem) ? *reinterpret_cast<const double2 *>(urow + e0 + q)
+                                             : make_double2(0.0, 0.0);
             uu[q] = v.x;
             uu[q + 1] = v.y;
         }
@@ -124,8 +132,8 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
             if (e0 + q >= 1) a[e0 + q - 1] = fma(-l, uu[q], a[e0 + q]);
     }
     a[W - 1] = 0.0;
-    // no trailing warp barrier: the next step's row k+1 starts past the n-k
-    // values of row k that are still read here, and rcp is read above
+    // no trailing warp barrier: the next step writes row k+1 (past row k's
+    // capacity) and rcp[(k+1) & 1], neither of which this step reads
     ++k;
 }
 
@@ -145,15 +153,15 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     // active width W >= n - k in steps of 32 / 24 / 16 / 12 / 8 / 4 (the
     // FMAs, pivot-row loads and publish stores of a step scale with W)
     if (NC >= 32) {
-        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
-        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
+        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
     }
     if (NC >= 16) {
-        while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
-        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
+        while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
+        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
     }
-    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, sm);
-    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, sm);
+    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
+    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, n, sm);
     __syncwarp();  // L / U rows from every lane are complete
     // ---- write every row once, at its final position p: L(p, c) for c < p,
     //      U(p, c) for c >= p (rows p >= K are pure L rows)
@@ -205,11 +213,7 @@ __global__ void __launch_bounds__(32 * S_WARPS, SmallCfg<NC>::ctas) lu_small_ker
 template <int NC>
 static void launch_class(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
     const size_t smem = (size_t)S_WARPS * sizeof(SmallWarpSmem<NC>);
-    static size_t attr = 0;
-    if (smem > attr) {
-        cudaFuncSetAttribute(lu_small_kernel<NC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = smem;
-    }
+    smem_optin(lu_small_kernel<NC>, smem);
     int grid = num_sms() * SmallCfg<NC>::ctas;
     int need = (a.batch + S_WARPS - 1) / S_WARPS;
     if (grid > need) grid = need;

@@ -40,7 +40,10 @@ void launch_partial_validate(int batch, int max_n1, int max_n2, const int *n1, c
 __global__ void getrs_validate_kernel(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
                                       const double *const *A, const int *lda, int *const *ipiv,
                                       double *const *B, const int *ldb, int *info) {
-    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    // one warp per system: the scalar checks, then every pivot must name a row
+    // in [k+1, n] (the solve kernels index shared memory with them)
+    const int lane = threadIdx.x & 31;
+    const int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (i >= batch) return;
     const int a = n[i], b = nrhs[i];
     int e = 0;
@@ -51,15 +54,24 @@ __global__ void getrs_validate_kernel(int batch, int max_n, int max_nrhs, const 
     else if (a > 0 && ipiv[i] == nullptr) e = -9;
     else if (a > 0 && b > 0 && B[i] == nullptr) e = -10;
     else if (ldb[i] < (a > 1 ? a : 1)) e = -11;
-    info[i] = e;
+    if (e == 0 && a > 0) {
+        const int *p = ipiv[i];
+        bool bad = false;
+        for (int k = lane; k < a; k += 32) {
+            const int v = p[k];
+            bad |= v < k + 1 || v > a;
+        }
+        if (__any_sync(FULL, bad)) e = -9;
+    }
+    if (lane == 0) info[i] = e;
 }
 
 void launch_getrs_validate(int batch, int max_n, int max_nrhs, const int *n, const int *nrhs,
                            const double *const *A, const int *lda, int *const *ipiv, double *const *B,
                            const int *ldb, int *info, cudaStream_t s) {
     KScope k(K_MISC, s);
-    getrs_validate_kernel<<<(batch + 255) / 256, 256, 0, s>>>(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B,
-                                                             ldb, info);
+    getrs_validate_kernel<<<(batch + 7) / 8, 256, 0, s>>>(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb,
+                                                         info);
 }
 
 // a6: per-matrix status words (info, FNV-1a of the pivot bytes), one thread

@@ -10,6 +10,7 @@ if ROOT not in sys.path:
 
 def pytest_configure(config):
     config.addinivalue_line("markers", "gpu: needs a CUDA device (B200, sm_100a)")
+    config.addinivalue_line("markers", "full: parity on every matrix of a full config (also marked gpu)")
 
 
 @pytest.fixture(scope="session")

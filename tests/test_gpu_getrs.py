@@ -173,3 +173,48 @@ def test_getrs_few_rhs_vec(max_r):
         Xo = oracle.getrs(LU, ip, B)
         dev = np.abs(X - Xo).max() / max(1e-300, np.abs(Xo).max())
         assert dev <= 1e-10, f"n={n} r={r}: deviation {dev}"
+
+
+@pytest.mark.parametrize("n,r", [(1200, 4), (1300, 3), (2100, 2), (3500, 1)])
+def test_getrs_vec_static_smem_gap(n, r):
+    """Dynamic shared memory in (48 KB - the static tile, 48 KB] (ADVICE r1:
+    the opt-in was skipped there and the launch failed): solved and matching
+    the oracle."""
+    irr.irr_set_tuning("getrs_vec", 1)
+    As = [irrgen.uniform_values(14, 0, n, n), irrgen.uniform_values(14, 1, 40, 40)]
+    Bs = [irrgen.uniform_values(15, 0, n, r), irrgen.uniform_values(15, 1, 40, r)]
+    LUs, ipivs, Xs, st = _solve(As, Bs)
+    assert (st == 0).all()
+    for A, B, LU, ip, X in zip(As, Bs, LUs, ipivs, Xs):
+        Xo = oracle.getrs(LU, ip, B)
+        dev = np.abs(X - Xo).max() / max(1e-300, np.abs(Xo).max())
+        assert dev <= 1e-10, f"n={A.shape[0]} r={r}: deviation {dev}"
+
+
+@pytest.mark.parametrize("vec", [1, 0])
+def test_getrs_invalid_pivots_flagged(vec):
+    """A pivot outside [k+1, n] (e.g. the zeros of a never-factored batch) is
+    reported as info -9 and that system is left untouched; its neighbours are
+    solved."""
+    irr.irr_set_tuning("getrs_vec", vec)
+    n = [16, 16, 16]
+    FA = MatrixBatch(n, n)
+    RB = MatrixBatch(n, [1, 1, 1])
+    _load(FA, [irrgen.uniform_values(3, g, 16, 16) for g in range(3)])
+    B0 = [irrgen.uniform_values(4, g, 16, 1) for g in range(3)]
+    _load(RB, B0)
+    FA.getrf()
+    torch.cuda.synchronize()
+    ip = FA.ipiv_data.cpu().numpy()
+    FA.ipiv_of(1, ip)[3] = 0          # below k + 1
+    FA.ipiv_of(2, ip)[15] = 17        # above n
+    FA.ipiv_data.copy_(torch.from_numpy(ip))
+    st = FA.getrs(RB).cpu().numpy()
+    torch.cuda.synchronize()
+    assert list(st[:3]) == [0, -9, -9]
+    rb = RB.data.cpu().numpy()
+    for g in (1, 2):
+        assert np.array_equal(np.array(RB.matrix(g, rb)), B0[g])
+    fa = FA.data.cpu().numpy()
+    Xo = oracle.getrs(np.array(FA.matrix(0, fa)), np.array(FA.ipiv_of(0, ip)), B0[0])
+    assert np.abs(np.array(RB.matrix(0, rb)) - Xo).max() <= 1e-10 * np.abs(Xo).max()
