@@ -128,9 +128,15 @@ def tier_of(m, n, tier_m_max=24576, l1=256):
 
 
 def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
-    """Algorithmic (flops, bytes) per kernel class for one getrf step
-    (DESIGN.md 'Roofline accounting'); tiers mirror classify.cu with the
-    library's live tuning."""
+    """Algorithmic (flops, bytes) per kernel class for one getrf step, SURVEY
+    §8(d): flops = FLOPS_DGETRF of the matrices a class works on (the grid-wide
+    tier's flops split by the step of the blocked algorithm each kernel
+    performs: panel, U12 solve, trailing GEMM -- parts of FLOPS_DGETRF, no
+    redundant work); bytes = each matrix read once and written once (16 m n +
+    4 min(m,n) + 32), attributed to the tier that owns the matrix and, inside
+    the grid-wide tier, to its kernel classes in proportion to their flops.
+    Redundant traffic (the blocked algorithm re-streaming the trailing
+    matrix) is never credited.  Tiers mirror classify.cu with the live tuning."""
     m = np.asarray(m, dtype=np.int64)
     n = np.asarray(n, dtype=np.int64)
     t = tier_of(m, n, tier_m_max, l1)
@@ -140,7 +146,9 @@ def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
         out[cls] = (float(F.getrf_flops(m[sel], n[sel]).sum()), float(F.getrf_bytes(m[sel], n[sel]).sum()))
     sel = t == 3
     mL, nL = m[sel], n[sel]
-    g_f = g_b = p_f = p_b = s_f = s_b = 0.0
+    tier_f = float(F.getrf_flops(mL, nL).sum())
+    tier_b = float(F.getrf_bytes(mL, nL).sum())
+    g_f = p_f = s_f = 0.0
     kL = np.minimum(mL, nL)
     for j in range(0, int(kL.max()) if len(kL) else 0, nb):
         act = kL > j
@@ -151,25 +159,26 @@ def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
         Mr = np.maximum(mm - j - ib, 0).astype(np.float64)
         Nr = np.maximum(nn - j - ib, 0).astype(np.float64)
         g_f += float((2 * Mr * Nr * ib).sum())
-        g_b += float((16 * Mr * Nr + 8 * (Mr + Nr) * ib * ((Mr > 0) & (Nr > 0))).sum())
         p_f += float(F.getrf_flops(mm - j, ib).sum())
-        p_b += float((16.0 * (mm - j) * ib).sum())
         s_f += float((ib * ib * Nr).sum())
-        s_b += float((16.0 * ib * (nn - ib)).sum())
-    out["gemm_trailing"] = (g_f, g_b)
-    out["panel"] = (p_f, p_b)
-    out["swap_trsm"] = (s_f, s_b)
-    out["strip"] = (g_f + s_f, g_b + s_b)  # fused interchange + TRSM + GEMM kernel
+    share = (lambda f: tier_b * f / tier_f) if tier_f > 0 else (lambda f: 0.0)
+    out["gemm_trailing"] = (g_f, share(g_f))
+    out["panel"] = (p_f, share(p_f))
+    out["swap_trsm"] = (s_f, share(s_f))
+    out["strip"] = (g_f + s_f, share(g_f + s_f))  # fused interchange + TRSM + GEMM kernel
+    out["grid_tier"] = (tier_f, tier_b)
     return out
 
 
 def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=256):
+    """As class_work for F11, plus the partial-front steps a5.2 (2 n1^2 n2
+    flops; F12 read + written, F11's factors read) and a5.3 (2 n1 n2^2 flops;
+    F22 read + written, F21 and F12 read) with their read-once bytes."""
     n1 = np.asarray(n1, dtype=np.int64)
     n2 = np.asarray(n2, dtype=np.int64)
     out = class_work(n1, n1, nb, tier_m_max, l1)
     out["gemm_dcwi"] = (float((2.0 * n1 * n2 * n2).sum()), float((8.0 * (2 * n2 * n2 + n2 * n1 + n1 * n2)).sum()))
-    out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((32.0 * n1 * n2).sum()))
-    # fused a5.2 (getrs_strip.cu): 2 n1^2 n2 flops; F12 read + written, F11 read once per strip
+    out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((16.0 * n1 * n2 + 8.0 * n1 * n1).sum()))
     out["getrs"] = (float((2.0 * n1 * n1 * n2).sum()), float((16.0 * n1 * n2 + 8.0 * n1 * n1).sum()))
     return out
 
@@ -217,6 +226,17 @@ def time_oracle(cfg, idx, target_s=10.0, threads=None):
     return fl / t / 1e9, threads, desc, t
 
 
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
 # ------------------------------------------------------------------ reference arm
 def run_reference(args, rank, world):
     """--impl reference: the CPU oracle (this tier's reference arm), rank 0 only."""
@@ -234,9 +254,10 @@ def run_reference(args, rank, world):
     v = float(np.mean(vals))
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "Gflop/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": None, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": cfg.name, "description": cfg.description, "batch": int(len(cfg.m))},
-            "cpu_baseline": {"value": v, "unit": "Gflop/s", "cores": threads, "kind": "oracle", "sample": desc},
+            "cpu_baseline": {"value": v, "unit": "Gflop/s", "cores": threads, "kind": "oracle", "sample": desc,
+                             "cpu_model": cpu_model()},
             "e2e": {"value": v, "unit": "Gflop/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -247,7 +268,11 @@ def main():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="C2", choices=irrgen.CONFIG_NAMES)
+    ap.add_argument("--config", default="C5", choices=irrgen.CONFIG_NAMES,
+                    help="workload (default C5: BASELINE.json's headline batch, the largest single-GPU config)")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong: the config's batch split over the N ranks (T1 / TN, SURVEY §8(e)); "
+                         "weak: N x the config")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--e2e-chunks", type=int, default=8, help="chunks of the pipelined end-to-end call")
@@ -286,8 +311,8 @@ def main():
             dist.init_process_group(backend)
     coll_dev = dev if backend == "nccl" else torch.device("cpu")
 
-    # ---- workload: global batch = world x config, LPT-sharded by flops
-    cfg = irrgen.config(args.config, scale=float(world))
+    # ---- workload: the config (strong) or world x the config (weak), LPT-sharded by flops
+    cfg = irrgen.config(args.config, scale=float(world) if args.scaling == "weak" else 1.0)
     kind = cfg.kind
     work = F.getrf_flops(cfg.m, cfg.n) if kind == "getrf" else F.partial_flops(cfg.m, cfg.n)
     owner = lpt_partition(work, world)
@@ -398,44 +423,9 @@ def main():
 
     # ---- e2e: host buffers through the public API, H2D + compute + D2H inside the timed region
     e2e = None
-    if devgen and not args.no_e2e:
-        e2e = {"value": None, "unit": "Gflop/s", "h2d_bytes_per_step": None, "d2h_bytes_per_step": None,
-               "note": "not measured: the batch (68 GB for C5) is generated on the device; no host copy fits"}
-    elif not args.no_e2e:
-        res_host = [torch.empty(o.numel(), dtype=o.dtype, pin_memory=True) for o in outs]
-        h2d = host.numel() * 8
-        d2h = sum(o.numel() * o.element_size() for o in outs)
-        # the public end-to-end entry points stream the batch in chunks: the
-        # H2D of chunk c+1, the factorization of chunk c and the D2H of chunk
-        # c-1 overlap (batch.getrf_host / getrf_partial_host)
-        from paper_conf_sc_abdelfattahgbtld22_b200.batch import getrf_host, getrf_partial_host
-        e2e_fn = getrf_host if kind == "getrf" else getrf_partial_host
-        pipe = None
-        e_ms = []
-        for s in range(args.warmup + args.steps):
-            flush.zero_()
-            torch.cuda.synchronize()
-            if world > 1:
-                dist.barrier()
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            pipe = e2e_fn(B, host, res_host[0], res_host[1], res_host[2], chunks=args.e2e_chunks, pipe=pipe)
-            if world > 1:
-                irr.irr_status_words(B.batch, sm, sn, B.ipiv, B.info, words)
-                if status is not words:
-                    status.copy_(words)
-                dist.all_gather_into_tensor(gathered, status)
-            b.record(stream)
-            torch.cuda.synchronize()
-            if s >= args.warmup:
-                e_ms.append(a.elapsed_time(b))
-        te = torch.tensor([float(np.sum(e_ms))], dtype=torch.float64, device=coll_dev)
-        if world > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        e_step = float(te.item()) / args.steps
-        e2e = {"value": flops_global / (e_step * 1e-3) / 1e9, "unit": "Gflop/s", "ms_per_step": e_step,
-               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "pipeline": f"{args.e2e_chunks} chunks: H2D / getrf / D2H overlapped (pinned host buffers)"}
+    if not args.no_e2e:
+        e2e = run_e2e(args, B, kind, host, flush, stream, world, sm, sn, words, status, gathered, dist, irr,
+                      work, mine, coll_dev)
 
     # ---- roofline of the dominant kernel class (rank-local, per step)
     hbm, hbm_src = peaks()
@@ -477,7 +467,7 @@ def main():
         g, cores, desc, secs = time_oracle(irrgen.config(args.config), np.arange(len(cfg.m)),
                                            target_s=args.cpu_seconds)
         cpu = {"value": g, "unit": "Gflop/s", "cores": cores, "kind": "oracle", "sample": desc,
-               "seconds": secs}
+               "seconds": secs, "cpu_model": cpu_model()}
 
     if args.profile_out and rank == 0:
         with open(args.profile_out, "w") as f:
@@ -488,9 +478,9 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "Gflop/s", "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic (seeded splitmix64 values U[-1,1), sizes per BASELINE config)",
-                "config": {"workload": cfg.name if world == 1 else f"{world}x{args.config}",
+                "config": {"workload": cfg.name if (world == 1 or args.scaling == "strong") else f"{world}x{args.config}",
                            "description": irrgen.config(args.config).description,
                            "batch_per_gpu": int(B.batch), "global_batch": int(len(cfg.m)),
                            "sharding": "LPT by flops" if world > 1 else "none",
@@ -504,6 +494,77 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def run_e2e(args, B, kind, host, flush, stream, world, sm, sn, words, status, gathered, dist, irr, work, mine,
+            coll_dev):
+    """The metric end to end through the public entry points getrf_host /
+    getrf_partial_host: every step copies the inputs from pinned host memory,
+    factors them and copies factors, pivots and info back, chunk-pipelined
+    (H2D of chunk c+1 / compute of chunk c / D2H of chunk c-1 overlap).  For
+    the device-generated C5 the host buffers are filled once (untimed) by a
+    device-to-host copy; when two host copies of the batch do not fit in RAM,
+    the largest prefix of the batch that does is timed and named."""
+    import psutil
+    import torch
+    from paper_conf_sc_abdelfattahgbtld22_b200.batch import (FrontBatch, MatrixBatch, getrf_host,
+                                                             getrf_partial_host)
+    Be, note = B, "whole batch"
+    if host is None:
+        avail = psutil.virtual_memory().available
+        budget = int(avail * 0.70) // 16          # doubles per host copy (two copies: in, out)
+        i1 = B.batch
+        if B.total > budget:
+            ends = B.offsets + (B.ld_h * (B.n_h if kind == "getrf" else B.nf_h))
+            i1 = int(np.searchsorted(ends, budget, side="right"))
+            note = (f"prefix of {i1} of {B.batch} matrices ({ends[i1 - 1] * 8 / 1e9:.1f} GB): two pinned copies of "
+                    f"the whole batch ({B.total * 16 / 1e9:.0f} GB) exceed the host's available RAM "
+                    f"({avail / 1e9:.0f} GB)")
+        if i1 < B.batch:
+            if kind == "getrf":
+                Be = MatrixBatch(B.m_h[:i1], B.n_h[:i1], data=B.data)
+            else:
+                raise RuntimeError("partial e2e prefix not supported")
+        host = torch.empty(Be.total, dtype=torch.float64, pin_memory=True)
+        host.copy_(B.data[: Be.total])          # the device-generated inputs, once (untimed)
+        sel = mine[: Be.batch]
+    else:
+        sel = mine
+    outs = [Be.data, Be.ipiv_data, Be.info]
+    res_host = [torch.empty(o.numel(), dtype=o.dtype, pin_memory=True) for o in outs]
+    h2d = host.numel() * 8
+    d2h = sum(o.numel() * o.element_size() for o in outs)
+    flops = float(work[sel].sum())
+    e2e_fn = getrf_host if kind == "getrf" else getrf_partial_host
+    pipe = None
+    e_ms = []
+    for s in range(args.warmup + args.steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        pipe = e2e_fn(Be, host, res_host[0], res_host[1], res_host[2], chunks=args.e2e_chunks, pipe=pipe)
+        if world > 1:
+            irr.irr_status_words(Be.batch, sm, sn, Be.ipiv, Be.info, words)
+            if status is not words:
+                status.copy_(words)
+            dist.all_gather_into_tensor(gathered, status)
+        b.record(stream)
+        torch.cuda.synchronize()
+        if s >= args.warmup:
+            e_ms.append(a.elapsed_time(b))
+    te = torch.tensor([float(np.sum(e_ms))], dtype=torch.float64, device=coll_dev)
+    if world > 1:
+        ft = torch.tensor([flops], dtype=torch.float64, device=te.device)
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        dist.all_reduce(ft, op=dist.ReduceOp.SUM)
+        flops = float(ft.item())
+    e_step = float(te.item()) / args.steps
+    return {"value": flops / (e_step * 1e-3) / 1e9, "unit": "Gflop/s", "ms_per_step": e_step,
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h), "batch": note,
+            "pipeline": f"{args.e2e_chunks} chunks: H2D / getrf / D2H overlapped (pinned host buffers)"}
 
 
 def _ncu_traffic(config, kname, launches_per_step):

@@ -27,7 +27,8 @@ __all__ = [
     "splitmix64", "matrix_key", "uniform_values", "hash_stream",
     "Config", "config", "CONFIG_NAMES",
     "g1_exact", "g1_singular", "g1_front", "g2_dominant",
-    "front_values",
+    "front_values", "g1_front_lapack", "zuniform_values", "zg1_exact",
+    "Tree", "assembly_tree", "tree_values", "tree_exact",
 ]
 
 _M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
@@ -227,6 +228,77 @@ def g1_front(seed: int, gid: int, n1: int, n2: int):
     return dict(F11=f(F11), F12=f(F12), F21=f(F21), F22=f(F22), X=f(X), S=f(S), L=L, U=U, ipiv=ipiv)
 
 
+def g1_front_lapack(seed: int, gid: int, n1: int, n2: int):
+    """G1'' (LAPACK-style partial, SURVEY §8(f) NEXT 3): F11 = P L U from G1;
+    U12 = X (n1 x n2 small integers), L21 = Y (n2 x n1, entries in
+    {0, +-1/4, +-1/2}), S (n2 x n2 small integers); F12 = P (L X),
+    F21 = Y U, F22 = S + Y X (all exact).  The LAPACK-style partial
+    factorization must return F12 -> X, F21 -> Y, F22 -> S exactly."""
+    F11, L, U, ipiv, _ = g1_exact(seed, gid, n1, n1)
+    h = hash_stream(seed, gid, 4, n1 * n2 * 2 + n2 * n2)
+    X = ((h[: n1 * n2] % np.uint64(9)).astype(np.int64) - 4).astype(np.float64).reshape((n2, n1)).T
+    Y = _L_SET[(h[n1 * n2: 2 * n1 * n2] % np.uint64(len(_L_SET))).astype(np.int64)].reshape((n1, n2)).T
+    S = ((h[2 * n1 * n2:] % np.uint64(9)).astype(np.int64) - 4).astype(np.float64).reshape((n2, n2)).T
+    F12 = _apply_swaps_reverse(L @ X, ipiv - 1) if n1 else np.zeros((0, n2))
+    F21 = Y @ U
+    F22 = S + Y @ X
+    f = np.asfortranarray
+    return dict(F11=f(F11), F12=f(F12), F21=f(F21), F22=f(F22), X=f(X), Y=f(Y), S=f(S), L=L, U=U, ipiv=ipiv)
+
+
+# complex families (ZGETRF, SURVEY §8(f) NEXT 3)
+_ZL_SET = np.array([0, 0.25, -0.25, 0.5, -0.5, 0.25j, -0.25j, 0.5j, -0.5j, 0.25 + 0.25j, 0.25 - 0.25j,
+                    -0.25 + 0.25j, -0.25 - 0.25j])
+_ZUD_SET = np.array([1, -1, 2, -2, 1j, -1j, 2j, -2j])
+
+
+def zuniform_values(seed: int, gid: int, m: int, n: int) -> np.ndarray:
+    """m x n complex128 Fortran matrix: element e = i + j m takes its real part
+    from draw 2e and its imaginary part from draw 2e+1 of the value stream
+    (each an exact dyadic in [-1, 1), as uniform_values)."""
+    key = matrix_key(seed, gid)
+    with np.errstate(over="ignore"):
+        x = splitmix64(key + np.arange(2 * m * n, dtype=np.uint64))
+    u = 2.0 * ((x >> np.uint64(11)).astype(np.float64) * (2.0 ** -53)) - 1.0
+    z = u[0::2] + 1j * u[1::2]
+    return z.reshape((n, m)).T.copy(order="F") if m * n else np.zeros((m, n), dtype=np.complex128, order="F")
+
+
+def zg1_exact(seed: int, gid: int, m: int, n: int, singular_col: int | None = None):
+    """Complex G1: L unit lower with off-diagonals in {0, +-1/4, +-1/2, +-i/4,
+    +-i/2, (+-1 +-i)/4} (|Re| + |Im| <= 1/2), U upper with Gaussian-integer
+    off-diagonals in [-8, 8] + [-8, 8] i and diagonal in {+-1, +-2, +-i, +-2i},
+    ipiv[k] ~ U[k, m).  Every candidate below the chosen pivot has at most
+    half its |Re| + |Im|, every division is by a unit times 1 or 2 and every
+    product is a Gaussian dyadic, so any correct complex GEPP with izamax
+    pivoting returns L, U, ipiv bit-exactly.  Returns (A, L, U, ipiv, info)."""
+    k = min(m, n)
+    h = hash_stream(seed, gid, 5, m * k + 2 * k * n + k + 1)
+    hl = h[: m * k].reshape((k, m)).T
+    hu = h[m * k: m * k + 2 * k * n].reshape((2 * n, k)).T
+    hp = h[m * k + 2 * k * n:]
+    L = np.zeros((m, k), dtype=np.complex128)
+    for j in range(k):
+        L[j, j] = 1.0
+        L[j + 1:, j] = _ZL_SET[(hl[j + 1:, j] % np.uint64(len(_ZL_SET))).astype(np.int64)]
+    U = np.zeros((k, n), dtype=np.complex128)
+    for i in range(k):
+        U[i, i] = _ZUD_SET[int(hu[i, i] % np.uint64(8))]
+        re = (hu[i, i + 1:n] % np.uint64(17)).astype(np.int64) - 8
+        im = (hu[i, n + i + 1:2 * n] % np.uint64(17)).astype(np.int64) - 8
+        U[i, i + 1:] = re + 1j * im
+    ipiv0 = np.array([j + int(hp[j] % np.uint64(m - j)) for j in range(k)], dtype=np.int64)
+    info = 0
+    if singular_col is not None:
+        c = singular_col
+        U[c, c:] = 0.0
+        L[c + 1:, c] = 0.0
+        ipiv0[c] = c
+        info = c + 1
+    A = _apply_swaps_reverse(L @ U, ipiv0)
+    return np.asfortranarray(A), L, U, (ipiv0 + 1).astype(np.int32), info
+
+
 def g2_dominant(seed: int, gid: int, m: int, n: int):
     """G2: permuted column-diagonally-dominant matrix.  Off-diagonals U[-1,1);
     for j < k: a_jj = +-(2*sum_{i!=j}|a_ij| + 1); rows permuted by pi (row r
@@ -336,3 +408,81 @@ def extend_add_level(seed: int, n_parents: int, np_max: int, children_per_parent
             F22.append(uniform_values(seed, gid, k, k))
             gid += 1
     return np_sizes, np.array(parent, dtype=np.int32), np.array(n2, dtype=np.int32), rel, F22, Fp
+
+
+# --------------------------------------------------------------------------
+# Synthetic assembly trees (§III-A):
+# the tree is traversed level by level from the leaves to the root; each
+# front F_r = [F11 F12; F21 F22] is partially factored and its Schur
+# complement F22 is extend-added into the parent front through an index map.
+# --------------------------------------------------------------------------
+@dataclass
+class Tree:
+    n1: np.ndarray          # fully summed variables of each node (its separator)
+    n2: np.ndarray          # contribution-block order (0 at the root)
+    parent: np.ndarray      # parent node, -1 at the root
+    rel: list               # rel[c]: int32[n2[c]], sorted rows / cols of the parent front
+    levels: list            # node ids per level, leaves first (a node's parent is on a later level)
+
+    @property
+    def nf(self):
+        return self.n1 + self.n2
+
+
+def assembly_tree(seed: int, depth: int, s0: float = 8.0, growth: float = 1.41, cfrac=(0.4, 0.9)) -> Tree:
+    """Complete binary tree of `depth` levels shaped like nested dissection of
+    a 2-D grid: a node at height h (leaves h = 0) owns n1 ~ s0 growth^h
+    U[0.75, 1.25] separator variables; a child's contribution block has
+    n2_c ~ U[cfrac] * nf_parent variables, mapped to a sorted random subset of
+    the parent front's nf_p = n1_p + n2_p indices.  Input construction only."""
+    rng = np.random.default_rng(seed)
+    nodes = 2 ** depth - 1
+    # node ids: level by level from the leaves; level h holds 2^(depth-1-h) nodes
+    levels, start = [], 0
+    for h in range(depth):
+        cnt = 2 ** (depth - 1 - h)
+        levels.append(np.arange(start, start + cnt))
+        start += cnt
+    height = np.concatenate([np.full(len(l), h) for h, l in enumerate(levels)])
+    n1 = np.maximum(1, np.rint(s0 * growth ** height * rng.uniform(0.75, 1.25, nodes))).astype(np.int64)
+    parent = np.full(nodes, -1, dtype=np.int64)
+    for h in range(depth - 1):
+        parent[levels[h]] = levels[h + 1][np.arange(len(levels[h])) // 2]
+    n2 = np.zeros(nodes, dtype=np.int64)
+    rel = [np.zeros(0, dtype=np.int32) for _ in range(nodes)]
+    for h in range(depth - 2, -1, -1):        # top down: the parent's front order is known
+        for c in levels[h]:
+            p = parent[c]
+            nfp = int(n1[p] + n2[p])
+            k = int(np.clip(np.rint(rng.uniform(*cfrac) * nfp), 1, nfp))
+            n2[c] = k
+            rel[c] = np.sort(rng.choice(nfp, size=k, replace=False)).astype(np.int32)
+    return Tree(n1, n2, parent, rel, levels)
+
+
+def tree_values(seed: int, tree: Tree):
+    """Original front values (before any extend-add): uniform dyadics, one
+    nf x nf block per node keyed by node id."""
+    return [front_values(seed, int(v), int(tree.n1[v] + tree.n2[v])) for v in range(len(tree.n1))]
+
+
+def tree_exact(seed: int, tree: Tree):
+    """Exact dyadic tree: every node's ASSEMBLED front (original + the
+    children's Schur complements) is a G1' front, so the partial factorization
+    of every node returns its chosen factors bit-exactly: F11 -> L\\U (with the
+    chosen ipiv), F12 -> X, F22 -> S.  The original of node p is the G1' front
+    minus the extend-add of its children's chosen S_c (small integers; exact).
+    Returns (originals, expected) with expected[v] = the g1_front dict."""
+    exp = [g1_front(seed, int(v), int(tree.n1[v]), int(tree.n2[v])) for v in range(len(tree.n1))]
+    orig = []
+    for v in range(len(tree.n1)):
+        e, a = exp[v], int(tree.n1[v])
+        F = np.zeros((a + int(tree.n2[v]),) * 2, order="F")
+        F[:a, :a], F[:a, a:], F[a:, :a], F[a:, a:] = e["F11"], e["F12"], e["F21"], e["F22"]
+        orig.append(F)
+    for c in range(len(tree.n1)):
+        p = tree.parent[c]
+        if p >= 0:
+            r = tree.rel[c]
+            orig[p][np.ix_(r, r)] -= exp[c]["S"]
+    return orig, exp

@@ -59,6 +59,11 @@ def lib():
         L.oracle_backward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
         L.oracle_backward_error.restype = C.c_double
         L.oracle_num_threads.restype = C.c_int
+        L.oracle_getrf_partial_lapack.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, dp, C.c_int,
+                                                  dp, C.c_int, ip, ip]
+        L.oracle_zgetrf.argtypes = [C.c_int, C.c_int, dp, C.c_int, ip, ip, dp]
+        L.oracle_zbackward_error.argtypes = [C.c_int, C.c_int, dp, C.c_int, dp, C.c_int, ip]
+        L.oracle_zbackward_error.restype = C.c_double
         vp = C.c_void_p
         L.check_getrf_batch.argtypes = [C.c_int, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_int]
         L.check_getrf_batch.restype = C.c_int
@@ -138,6 +143,60 @@ def getrf_partial(F11, F12, F21, F22):
     if r < 0:
         raise ValueError(f"oracle_getrf_partial: bad argument {-r}")
     return F11, F12, F22, ipiv[:n1], int(info[0])
+
+
+def getrf_partial_lapack(F11, F12, F21, F22):
+    """LAPACK-style partial front on copies.  Returns
+    (F11 -> L\\U, F12 -> U12 = L^-1 P^T F12, F21 -> L21 = F21 U^-1,
+    F22 -> F22 - L21 U12, ipiv, info)."""
+    F11, F12, F21, F22 = (_fortran(X) for X in (F11, F12, F21, F22))
+    n1, n2 = F11.shape[0], F22.shape[0]
+    ipiv = np.zeros(max(1, n1), dtype=np.int32)
+    info = np.zeros(1, dtype=np.int32)
+    bufs = [X if X.size else np.zeros(1) for X in (F11, F12, F21, F22)]
+    r = lib().oracle_getrf_partial_lapack(n1, n2, _dp(bufs[0]), max(1, n1), _dp(bufs[1]), max(1, n1),
+                                          _dp(bufs[2]), max(1, n2), _dp(bufs[3]), max(1, n2), _ip(ipiv),
+                                          _ip(info))
+    if r < 0:
+        raise ValueError(f"oracle_getrf_partial_lapack: bad argument {-r}")
+    return F11, F12, F21, F22, ipiv[:n1], int(info[0])
+
+
+def _cfortran(A):
+    A = np.asarray(A, dtype=np.complex128)
+    if A.ndim != 2:
+        raise ValueError("matrix must be 2-D")
+    return np.array(A, dtype=np.complex128, order="F", copy=True)
+
+
+def zgetrf(A):
+    """Complex GEPP (LAPACK zgetf2 semantics, izamax pivoting) on a copy of A.
+    Returns (LU complex128 Fortran, ipiv (1-based int32), info, min_sep)."""
+    LU = _cfortran(A)
+    m, n = LU.shape
+    ipiv = np.zeros(max(1, min(m, n)), dtype=np.int32)
+    info = np.zeros(1, dtype=np.int32)
+    sep = np.zeros(1)
+    buf = LU if LU.size else np.zeros((max(1, m), 1), dtype=np.complex128, order="F")
+    r = lib().oracle_zgetrf(m, n, buf.ctypes.data_as(C.POINTER(C.c_double)), max(1, m), _ip(ipiv), _ip(info),
+                            _dp(sep))
+    if r < 0:
+        raise ValueError(f"oracle_zgetrf: bad argument {-r}")
+    return LU, ipiv[: min(m, n)], int(info[0]), float(sep[0])
+
+
+def zbackward_error(A0, LU, ipiv):
+    A0, LU = _cfortran(A0), _cfortran(LU)
+    m, n = A0.shape
+    ipiv = np.ascontiguousarray(ipiv, dtype=np.int32)
+    if ipiv.size == 0:
+        ipiv = np.zeros(1, dtype=np.int32)
+    z = np.zeros((1, 1), dtype=np.complex128, order="F")
+    b0 = A0 if A0.size else z
+    b1 = LU if LU.size else z
+    P = C.POINTER(C.c_double)
+    return lib().oracle_zbackward_error(m, n, b0.ctypes.data_as(P), max(1, m), b1.ctypes.data_as(P), max(1, m),
+                                        _ip(ipiv))
 
 
 def getrf_partial_batch(fronts, nthreads: int = 0):

@@ -32,6 +32,17 @@
  *    as its plain definition Fp[rel_i, rel_j] += F22[i, j].
  *  - oracle_backward_error: ||PA - LU||_F / (||A||_F * k * eps) (north_star;
  *    SURVEY reading Q11), accumulated in long double.
+ *  - oracle_getrf_partial_lapack: the LAPACK-style variant of the partial
+ *    front factorization (reading Q8's alternative; the
+ *    solver's factors L21 = F21 U^-1, U12 = L^-1 P^T F12, L96-97), written
+ *    out as its steps: GEPP of F11, swaps on F12, forward substitution on
+ *    F12, row-by-row substitution x U = f on F21, F22 - L21 U12.
+ *  - oracle_zgetrf / oracle_zbackward_error: LU with partial pivoting of a
+ *    COMPLEX matrix (the solver's A in C^{N x N}, L71 §III-A; SURVEY §8(f)
+ *    NEXT 3) with LAPACK zgetf2 semantics (reading Q20 in DESIGN.md): pivot =
+ *    the smallest row maximising |Re| + |Im| (izamax), the textbook complex
+ *    division (a+bi)/(c+di) = ((ac+bd) + (bc-ad)i) / (c^2+d^2), complex
+ *    multiply (ac-bd) + (ad+bc)i, interleaved (re, im) column-major storage.
  */
 #include <math.h>
 #include <stdint.h>
@@ -402,6 +413,179 @@ double oracle_backward_error(int m, int n, const double *A0, int lda0, const dou
             an += a * a;
         }
     free(PA);
+    if (an == 0.0L) return rn == 0.0L ? 0.0 : INFINITY;
+    return (double)(sqrtl(rn) / (sqrtl(an) * (long double)imax(1, K) * (long double)DBL_EPSILON));
+}
+
+/* ---------------------------------------------------------------------------
+ * LAPACK-style partial front (reading Q8's
+ * alternative): F11 -> L\U (pivots within F11), F12 -> U12 = L^-1 P^T F12,
+ * F21 -> L21 = F21 U^-1, F22 -> F22 - L21 U12.  In exact arithmetic the same
+ * Schur complement as oracle_getrf_partial.
+ * ------------------------------------------------------------------------- */
+int oracle_getrf_partial_lapack(int n1, int n2, double *F11, int ld11, double *F12, int ld12,
+                                double *F21, int ld21, double *F22, int ld22, int *ipiv, int *info)
+{
+    if (n1 < 0) return -1;
+    if (n2 < 0) return -2;
+    if (ld11 < imax(1, n1)) return -4;
+    if (ld12 < imax(1, n1)) return -6;
+    if (ld21 < imax(1, n2)) return -8;
+    if (ld22 < imax(1, n2)) return -10;
+    /* step 1: P L U <- LU(F11), pivot search over F11's n1 rows only */
+    int r = oracle_getrf(n1, n1, F11, ld11, ipiv, info, NULL);
+    if (r < 0) return r;
+#define F11_(i, j) F11[(size_t)(i) + (size_t)(j) * ld11]
+#define F12_(i, j) F12[(size_t)(i) + (size_t)(j) * ld12]
+#define F21_(i, j) F21[(size_t)(i) + (size_t)(j) * ld21]
+#define F22_(i, j) F22[(size_t)(i) + (size_t)(j) * ld22]
+    /* step 2: P^T F12 -- the swaps k = 0..n1-1 in order */
+    for (int k = 0; k < n1; ++k) {
+        int p = ipiv[k] - 1;
+        if (p != k)
+            for (int c = 0; c < n2; ++c) { double t = F12_(k, c); F12_(k, c) = F12_(p, c); F12_(p, c) = t; }
+    }
+    /* step 3: U12 = L^-1 F12 (unit lower): row i -= sum_{j<i} l_ij row j */
+    for (int c = 0; c < n2; ++c)
+        for (int i = 0; i < n1; ++i) {
+            double s = 0.0;
+            for (int j = 0; j < i; ++j) s = s + F11_(i, j) * F12_(j, c);
+            F12_(i, c) = F12_(i, c) - s;
+        }
+    /* step 4: L21 = F21 U^-1: each row x of F21 solves x U = f,
+     * x_j = (f_j - sum_{k<j} x_k u_kj) / u_jj, j ascending */
+    for (int i = 0; i < n2; ++i)
+        for (int j = 0; j < n1; ++j) {
+            double s = 0.0;
+            for (int k = 0; k < j; ++k) s = s + F21_(i, k) * F11_(k, j);
+            F21_(i, j) = (F21_(i, j) - s) / F11_(j, j);
+        }
+    /* step 5: F22 <- F22 - L21 U12, plain triple loop, k ascending */
+    for (int j = 0; j < n2; ++j)
+        for (int i = 0; i < n2; ++i) {
+            double s = 0.0;
+            for (int k = 0; k < n1; ++k) s = s + F21_(i, k) * F12_(k, j);
+            F22_(i, j) = F22_(i, j) - s;
+        }
+#undef F11_
+#undef F12_
+#undef F21_
+#undef F22_
+    return 0;
+}
+
+/* ---------------------------------------------------------------------------
+ * Complex LU with partial pivoting (the solver's
+ * A in C^{N x N}).  Storage: column-major, element (i, j) at A[2 (i + j ld)]
+ * (re) and A[2 (i + j ld) + 1] (im) -- C99 / std::complex<double> layout.
+ * LAPACK zgetf2 semantics (DESIGN reading Q20): k = 0..min(m,n)-1:
+ *   1. p = smallest i >= k maximising cabs1(a_ik) = |Re| + |Im| (izamax);
+ *   2. ipiv[k] = p + 1;
+ *   3. if a_pk != 0: swap rows k, p across all n columns; a_ik <- a_ik / a_kk
+ *      for i > k (textbook complex division); else info <- k + 1 (first);
+ *   4. a_ij <- a_ij - a_ik a_kj for i, j > k (complex multiply, then subtract).
+ * min_sep: rho = min over steps of cabs1(best) / cabs1(second best) (Q13).
+ * ------------------------------------------------------------------------- */
+static double cabs1(double re, double im) { return fabs(re) + fabs(im); }
+
+int oracle_zgetrf(int m, int n, double *A, int ld, int *ipiv, int *info, double *min_sep)
+{
+    if (m < 0) return -1;
+    if (n < 0) return -2;
+    if (ld < imax(1, m)) return -4;
+    *info = 0;
+    double sep = INFINITY;
+#define RE(i, j) A[2 * ((size_t)(i) + (size_t)(j) * (size_t)ld)]
+#define IM(i, j) A[2 * ((size_t)(i) + (size_t)(j) * (size_t)ld) + 1]
+    const int K = imin(m, n);
+    for (int k = 0; k < K; ++k) {
+        int p = k;
+        double best = cabs1(RE(k, k), IM(k, k)), second = -1.0;
+        for (int i = k + 1; i < m; ++i) {
+            double v = cabs1(RE(i, k), IM(i, k));
+            if (v > best) { second = best; best = v; p = i; }
+            else if (v > second) second = v;
+        }
+        if (best > 0.0 && second > 0.0) {
+            double r = best / second;
+            if (r < sep) sep = r;
+        }
+        ipiv[k] = p + 1;
+        if (RE(p, k) != 0.0 || IM(p, k) != 0.0) {
+            if (p != k)
+                for (int j = 0; j < n; ++j) {
+                    double tr = RE(k, j), ti = IM(k, j);
+                    RE(k, j) = RE(p, j); IM(k, j) = IM(p, j);
+                    RE(p, j) = tr; IM(p, j) = ti;
+                }
+            const double c = RE(k, k), d = IM(k, k);
+            const double den = c * c + d * d;
+            for (int i = k + 1; i < m; ++i) {
+                const double a = RE(i, k), b = IM(i, k);
+                RE(i, k) = (a * c + b * d) / den;
+                IM(i, k) = (b * c - a * d) / den;
+            }
+        } else if (*info == 0) {
+            *info = k + 1;
+        }
+        for (int j = k + 1; j < n; ++j) {
+            const double ur = RE(k, j), ui = IM(k, j);
+            for (int i = k + 1; i < m; ++i) {
+                const double lr = RE(i, k), li = IM(i, k);
+                const double pr = lr * ur - li * ui, pi = lr * ui + li * ur;
+                RE(i, j) = RE(i, j) - pr;
+                IM(i, j) = IM(i, j) - pi;
+            }
+        }
+    }
+#undef RE
+#undef IM
+    if (min_sep) *min_sep = sep;
+    return 0;
+}
+
+/* ||PA - LU||_F / (||A||_F * max(1, min(m,n)) * eps) for complex factors
+ * (Q11 with the complex Frobenius norm), long double accumulation. */
+double oracle_zbackward_error(int m, int n, const double *A0, int lda0, const double *LU, int ld,
+                              const int *ipiv)
+{
+    const int K = imin(m, n);
+    const size_t mm = (size_t)(m > 0 ? m : 1), nn = (size_t)(n > 0 ? n : 1);
+    long double *PR = (long double *)malloc(sizeof(long double) * mm * nn);
+    long double *PI = (long double *)malloc(sizeof(long double) * mm * nn);
+    for (int j = 0; j < n; ++j)
+        for (int i = 0; i < m; ++i) {
+            PR[i + (size_t)j * m] = A0[2 * (i + (size_t)j * lda0)];
+            PI[i + (size_t)j * m] = A0[2 * (i + (size_t)j * lda0) + 1];
+        }
+    for (int k = 0; k < K; ++k) {
+        int p = ipiv[k] - 1;
+        if (p != k)
+            for (int j = 0; j < n; ++j) {
+                long double t = PR[k + (size_t)j * m]; PR[k + (size_t)j * m] = PR[p + (size_t)j * m]; PR[p + (size_t)j * m] = t;
+                t = PI[k + (size_t)j * m]; PI[k + (size_t)j * m] = PI[p + (size_t)j * m]; PI[p + (size_t)j * m] = t;
+            }
+    }
+    long double rn = 0.0L, an = 0.0L;
+    for (int j = 0; j < n; ++j)
+        for (int i = 0; i < m; ++i) {
+            long double sr = 0.0L, si = 0.0L;
+            int lim = imin(imin(i, j), K - 1);
+            for (int l = 0; l <= lim; ++l) {
+                long double lr = (l == i) ? 1.0L : (long double)LU[2 * (i + (size_t)l * ld)];
+                long double li = (l == i) ? 0.0L : (long double)LU[2 * (i + (size_t)l * ld) + 1];
+                long double ur = (long double)LU[2 * (l + (size_t)j * ld)];
+                long double ui = (long double)LU[2 * (l + (size_t)j * ld) + 1];
+                sr += lr * ur - li * ui;
+                si += lr * ui + li * ur;
+            }
+            long double dr = PR[i + (size_t)j * m] - sr, di = PI[i + (size_t)j * m] - si;
+            rn += dr * dr + di * di;
+            long double ar = A0[2 * (i + (size_t)j * lda0)], ai = A0[2 * (i + (size_t)j * lda0) + 1];
+            an += ar * ar + ai * ai;
+        }
+    free(PR);
+    free(PI);
     if (an == 0.0L) return rn == 0.0L ? 0.0 : INFINITY;
     return (double)(sqrtl(rn) / (sqrtl(an) * (long double)imax(1, K) * (long double)DBL_EPSILON));
 }

@@ -32,14 +32,20 @@ def _offsets(sizes: np.ndarray, align: int = ALIGN):
 
 
 class MatrixBatch:
-    def __init__(self, m, n, ld=None, device="cuda", with_ipiv=True):
+    def __init__(self, m, n, ld=None, device="cuda", with_ipiv=True, data=None):
+        """data: optional existing float64 buffer (>= total elements) to lay
+        the batch out in (e.g. a prefix of a larger batch), else allocated."""
         self.m_h = np.asarray(m, dtype=np.int64)
         self.n_h = np.asarray(n, dtype=np.int64)
         self.batch = len(self.m_h)
         self.ld_h = np.maximum(1, self.m_h) if ld is None else np.asarray(ld, dtype=np.int64)
-        self.device = torch.device(device)
+        self.device = torch.device(device) if data is None else data.device
         self.offsets, self.total = _offsets(self.ld_h * self.n_h)
-        self.data = torch.empty(self.total, dtype=torch.float64, device=self.device)
+        if data is None:
+            self.data = torch.empty(self.total, dtype=torch.float64, device=self.device)
+        else:
+            assert data.dtype == torch.float64 and data.numel() >= self.total
+            self.data = data[: self.total]
         base = self.data.data_ptr()
         self.ptr = torch.from_numpy(base + 8 * self.offsets).to(self.device)
         self.m = torch.from_numpy(self.m_h.astype(np.int32)).to(self.device)

@@ -39,7 +39,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
 // left-block interchanges (6.80 -> 6.53 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, 0};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -166,6 +166,7 @@ struct Work {
     int *sort;  // size sort (sched.cuh): sorted slots + bucket prefix
     int *keys;  // per-matrix sort keys
     void *plans;  // getrf / partial only: one interchange plan per tier-L slot
+    void *outer_plans;  // getrf / partial only: one outer-block plan per tier-L slot (two-level tier)
 };
 
 static size_t work_bytes_for(int batch) {
@@ -178,7 +179,7 @@ static size_t work_bytes_for(int batch) {
 // grid-wide tier (written by its panel kernel, read by its strip kernel)
 static size_t work_bytes_getrf(int batch) {
     size_t b = (size_t)(batch > 0 ? batch : 1);
-    return work_bytes_for(batch) + align256(b * SWAP_PLAN_BYTES);
+    return work_bytes_for(batch) + align256(b * SWAP_PLAN_BYTES) + align256(b * OUTER_PLAN_BYTES);
 }
 
 static Work carve(void *work, int batch) {
@@ -196,6 +197,8 @@ static Work carve(void *work, int batch) {
     w.keys = (int *)p;
     p += align256(b * sizeof(int));
     w.plans = p;  // valid only in a work_bytes_getrf() workspace
+    p += align256(b * SWAP_PLAN_BYTES);
+    w.outer_plans = p;
     return w;
 }
 
@@ -245,7 +248,7 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
         }
         if (has_large) {
             if (t.l1) launch_lu_l1(a, w.counters, w.bins, w.keys, w.sort, s);
-            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, s);
+            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, w.outer_plans, s);
         }
     }
     if (side != s) {
@@ -326,6 +329,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "getrs_vec")) g_tuning.getrs_vec = value ? 1 : 0;
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
     else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
+    else if (!strcmp(key, "nb_outer")) g_tuning.nb_outer = value < 0 ? 0 : (value > NB_OUTER_MAX ? NB_OUTER_MAX : value);
 }
 
 int irr_get_tuning(const char *key) {
@@ -349,6 +353,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "getrs_vec")) return g_tuning.getrs_vec;
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
     if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) return g_tuning.defer;
+    if (!strcmp(key, "nb_outer")) return g_tuning.nb_outer;
     return -1;
 }
 

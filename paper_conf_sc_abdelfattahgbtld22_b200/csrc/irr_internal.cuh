@@ -33,6 +33,7 @@ struct Tuning {
     int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
     int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)
     int getrs_vec;       // 1: irr_getrs with max_nrhs <= 4 by the CTA-per-system kernel (getrs_vec.cu)
+    int nb_outer;        // grid-wide tier: outer block width of the two-level blocking (0 / <= nb: one level)
 };
 Tuning &tuning();
 
@@ -81,7 +82,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
@@ -224,7 +225,10 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
                    cudaStream_t s);
 // lu_large.cu
 constexpr size_t SWAP_PLAN_BYTES = 1040;  // sizeof(SwapPlan), checked in lu_large.cu
-void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, cudaStream_t s);
+constexpr int NB_OUTER_MAX = 128;          // widest outer block of the two-level grid tier
+constexpr size_t OUTER_PLAN_BYTES = 2064;  // sizeof(OuterPlan), checked in lu_large.cu
+void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, void *outer_plans,
+                     cudaStream_t s);
 void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)

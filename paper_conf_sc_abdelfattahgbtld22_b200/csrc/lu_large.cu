@@ -19,7 +19,7 @@
 //       (DCWI: each kernel infers full / partial / no work per
 //       matrix) with grid-wide kernels per step, so a few huge fronts use the
 //       whole GPU.
-#include "gemm_core.cuh"
+#include "gemm_big.cuh"
 #include "panel.cuh"
 #include "panel_win.cuh"
 #include "sched.cuh"
@@ -36,9 +36,20 @@ static_assert(L1_NT == G_NT && L1_NT == SW_NT, "L1 composes the GEMM and swap pi
 // ------------------------------------------------------------------ swap plan
 // (SwapPlan is defined in panel.cuh: panel_regs can emit it directly.)
 
-// Warp 0 composes the interchanges held in sp.piv[0..ib) (0-based absolute
-// rows).  Caller synchronises the CTA afterwards.
-__device__ __forceinline__ void plan_swaps_core(int j, int ib, SwapPlan &sp) {
+// The plan of one outer block of the two-level grid tier (up to
+// NB_OUTER_MAX interchanges; same fields as SwapPlan).
+struct OuterPlan {
+    int top_src[NB_OUTER_MAX];
+    int piv[NB_OUTER_MAX];
+    int bot_pos[NB_OUTER_MAX], bot_src[NB_OUTER_MAX];
+    int nbot;
+};
+static_assert(sizeof(OuterPlan) <= OUTER_PLAN_BYTES, "outer plan slot");
+
+// One warp composes the interchanges held in sp.piv[0..ib) (0-based absolute
+// rows).  Caller synchronises afterwards.
+template <class Plan>
+__device__ __forceinline__ void plan_swaps_core(int j, int ib, Plan &sp) {
     const int lane = threadIdx.x & 31;
     const int c1 = j + ib;
     for (int t = lane; t < ib; t += 32) sp.top_src[t] = j + t;
@@ -720,7 +731,8 @@ template <bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                         const int *__restrict__ bins,
                                                         const SwapPlan *__restrict__ plans, int *queue, int j,
-                                                        int nb, int chunks_per, unsigned long long *ph, int defer) {
+                                                        int nb, int chunks_per, unsigned long long *ph, int defer,
+                                                        int J, int cmax) {
     extern __shared__ __align__(16) double st_smem[];
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
@@ -759,10 +771,17 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         if (j >= K) continue;
         const int ib = K - j < nb ? K - j : nb;
         const int c1 = j + ib;
-        // virtual columns: the left block [0, jl) (empty when its interchanges
-        // are deferred to left_swaps_kernel) then the right block [c1, n)
-        const int jl = defer ? 0 : j;
-        const int vtot = jl + ni - c1, vb = q * ST_COLS;
+        // virtual columns v in [lb, j + nright): v < j is left-block column v
+        // (interchanges only), v >= j is column v + ib of the right block
+        // [c1, ce) (interchanges + U12 solve + GEMM).  One level: lb = 0 (eager)
+        // or j (left block deferred to left_swaps_kernel), ce = n.  Two-level
+        // (J >= 0): the inner step works inside the outer block [J, cmax):
+        // lb = J, ce = min(n, cmax); columns outside it get the outer block's
+        // interchanges later (outer_swap_trsm_kernel / left_swaps_kernel).
+        const int lb = J >= 0 ? J : (defer ? j : 0);
+        const int ce = imin(ni, cmax);
+        const int nright = ce > c1 ? ce - c1 : 0;
+        const int vtot = (j - lb) + nright, vb = q * ST_COLS;
         if (vb >= vtot) continue;
         double *gA = a.A[i];
         if (slot != last_slot) {
@@ -776,11 +795,12 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         __syncthreads();
         ST_PHASE(0)
         const int W = imin(ST_COLS, vtot - vb);
+        const int v0 = lb + vb;  // first virtual column of the strip
         // row stride GPAD: top doubles as the GEMM's resident B stage
-        swap_chunk<ST_COLS, GPAD>(gA, ld, j, ib, vb, W, jl, c1 - jl, c1, sp, L11, ldl, top, bot, ph);
+        swap_chunk<ST_COLS, GPAD>(gA, ld, j, ib, v0, W, j, ib, c1, sp, L11, ldl, top, bot, ph);
         if (ph && tid == 0) t0 = clock64();
         // trailing GEMM on the strip's right-of-panel columns
-        const int cbeg = (vb > jl ? vb : jl) + (c1 - jl), cend = vb + W + (c1 - jl);
+        const int cbeg = (v0 > j ? v0 : j) + ib, cend = v0 + W + ib;
         if (cbeg < cend && c1 < mi) {
             GemmDesc d0;
             d0.A = gA + c1 + (size_t)j * ld; d0.lda = ld; d0.ta = 0;
@@ -798,7 +818,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
                 ++tt;
                 return true;
             };
-            if (bres && vb >= jl) {  // the GEMM's columns start at top's column 0
+            if (bres && v0 >= j) {  // the GEMM's columns start at top's column 0
                 // B rows >= ib of the resident operand must be zero (A is
                 // zero-filled there, but stale shared memory may hold NaNs)
                 if (ib < 2 * GBK)
@@ -841,6 +861,177 @@ __global__ void __launch_bounds__(LSW_NT) left_swaps_kernel(GetrfArgs a, const i
         if (K > nb) left_swaps_core<LSW_NT>(a.A[i], a.ld[i], mi, K, nb, a.ipiv[i], g, h, buf, LSW_BUF);
     }
 }
+
+
+// ================================================================== two-level grid tier
+// Outer blocks of NBo (<= NB_OUTER_MAX) columns, each factored by NBo / nb
+// inner panel steps confined to the block (panel_win_kernel + strip_kernel
+// with J >= 0), then ONE update of the rest of the matrix per outer block
+// (P:L106's blocked right-looking LU with panel width NBo, the panel itself
+// blocked): the composed interchanges of the NBo pivots + U12 <- L11^-1 A12
+// (outer_swap_trsm_kernel) and A22 -= L21 U12 with K = NBo on the 128 x 128
+// DMMA core (xgemm).  The trailing matrix is streamed once per NBo columns
+// instead of once per nb: arithmetic intensity NBo / 8 flop/B instead of
+// nb / 8 (SURVEY §7 hard part 1).
+
+// one warp per tier-L slot composes the outer block's interchanges
+// ipiv[J .. J + ibo) into a plan (absolute rows); block 0 resets the queue
+// of outer_swap_trsm_kernel (stream-ordered)
+constexpr int OP_NT = 256;
+__global__ void __launch_bounds__(OP_NT) outer_plan_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                           const int *__restrict__ bins, int J, int NBo,
+                                                           OuterPlan *__restrict__ plans, int *queue) {
+    __shared__ OuterPlan sp[OP_NT / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (blockIdx.x == 0 && threadIdx.x == 0) *queue = 0;
+    const int count = counters[CNT_BIN0 + BIN_L];
+    const int *list = bins + (size_t)BIN_L * a.batch;
+    OuterPlan &p = sp[warp];
+    for (int t = blockIdx.x * (OP_NT / 32) + warp; t < count; t += gridDim.x * (OP_NT / 32)) {
+        const int i = list[t];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        if (J >= K || J + NBo >= ni) continue;  // no columns right of the block
+        const int ibo = imin(NBo, K - J);
+        const int *ip = a.ipiv[i];
+        for (int q = lane; q < ibo; q += 32) p.piv[q] = ip[J + q] - 1;
+        __syncwarp();
+        plan_swaps_core(J, ibo, p);
+        __syncwarp();
+        OuterPlan &g = plans[t];
+        for (int q = lane; q < ibo; q += 32) g.top_src[q] = p.top_src[q];
+        const int nbot = p.nbot;
+        for (int q = lane; q < nbot; q += 32) {
+            g.bot_pos[q] = p.bot_pos[q];
+            g.bot_src[q] = p.bot_src[q];
+        }
+        if (lane == 0) g.nbot = nbot;
+        __syncwarp();
+    }
+}
+
+// Right of outer block [J, J + ibo): per (tier-L slot, OS_COLS-column strip),
+// gather the moved rows (the block's interchanges composed), scatter the rows
+// pushed below the block, solve U12 <- L11^-1 U12 in 32-row blocks (diagonal
+// block by the register substitution of the inner steps, the rows below by
+// a rank-32 update with the L column block staged in shared memory), write
+// U12 back.  Dynamic item queue (reset by outer_plan_kernel).
+constexpr int OS_COLS = 32, OS_NT = 128, OS_LD = OS_COLS + 1, OS_LDC = NB_OUTER_MAX + 1;
+constexpr size_t OS_SMEM = (size_t)(2 * NB_OUTER_MAX * OS_LD + 32 * OS_LDC) * sizeof(double);
+__global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                                   const int *__restrict__ bins,
+                                                                   const OuterPlan *__restrict__ plans, int *queue,
+                                                                   int J, int NBo, int chunks_per) {
+    extern __shared__ __align__(16) double os_smem[];
+    double *top = os_smem;                         // [ibo][OS_LD]
+    double *bot = top + NB_OUTER_MAX * OS_LD;      // [nbot][OS_LD]
+    double *Lc = bot + NB_OUTER_MAX * OS_LD;       // L column block: Lc[r + s * OS_LDC]
+    __shared__ OuterPlan sp;
+    __shared__ int item_s;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    constexpr int NWS = OS_NT / 32;
+    const int count = counters[CNT_BIN0 + BIN_L];
+    const int *list = bins + (size_t)BIN_L * a.batch;
+    const long long total = (long long)count * chunks_per;
+    int last_slot = -1;
+    for (;;) {
+        if (tid == 0) item_s = atomicAdd(queue, 1);
+        __syncthreads();
+        const long long w = item_s;
+        __syncthreads();
+        if (w >= total) break;
+        const int slot = (int)(w / chunks_per), q = (int)(w - (long long)slot * chunks_per);
+        const int i = list[slot];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        if (J >= K) continue;
+        const int ibo = imin(NBo, K - J), c1 = J + ibo;
+        const int cb = c1 + q * OS_COLS;
+        if (cb >= ni) continue;
+        const int W = imin(OS_COLS, ni - cb);
+        const long ld = a.ld[i];
+        double *gA = a.A[i];
+        if (slot != last_slot) {
+            const int *src = reinterpret_cast<const int *>(plans + slot);
+            int *dst = reinterpret_cast<int *>(&sp);
+            for (int e = tid; e < (int)(sizeof(OuterPlan) / sizeof(int)); e += OS_NT) dst[e] = src[e];
+            last_slot = slot;
+            __syncthreads();
+        }
+        const int nbot = sp.nbot;
+        // ---- gather (all reads before any write of the strip)
+        for (int c = warp; c < W; c += NWS) {
+            const double *gc = gA + (size_t)(cb + c) * ld;
+            for (int t = lane; t < ibo; t += 32) cp_async8(&top[t * OS_LD + c], gc + sp.top_src[t]);
+            for (int b = lane; b < nbot; b += 32) cp_async8(&bot[b * OS_LD + c], gc + sp.bot_src[b]);
+        }
+        cp_async_commit();
+        cp_async_wait<0>();
+        __syncthreads();
+        // ---- the rows pushed below the block: final for this step
+        for (int c = warp; c < W; c += NWS) {
+            double *gc = gA + (size_t)(cb + c) * ld;
+            for (int b = lane; b < nbot; b += 32) gc[sp.bot_pos[b]] = bot[b * OS_LD + c];
+        }
+        // ---- U12 <- L11^-1 U12, 32-row blocks
+        for (int d0 = 0; d0 < ibo; d0 += 32) {
+            const int bw = imin(32, ibo - d0);
+            // L11 rows [d0, ibo) x cols [d0, d0 + bw) (column block, incl. the diagonal block)
+            for (int sc = warp; sc < bw; sc += NWS) {
+                const double *gl = gA + J + (size_t)(J + d0 + sc) * ld;
+                for (int r = d0 + lane; r < ibo; r += 32) cp_async8(&Lc[(r - d0) + sc * OS_LDC], gl + r);
+            }
+            cp_async_commit();
+            cp_async_wait<0>();
+            __syncthreads();
+            if (tid < W) trsm_col_regs<32>(top + d0 * OS_LD + tid, OS_LD, bw, Lc, OS_LDC);
+            __syncthreads();
+            if (d0 + bw < ibo && lane < W) {
+                double x[32];
+#pragma unroll
+                for (int sc = 0; sc < 32; ++sc) x[sc] = sc < bw ? top[(d0 + sc) * OS_LD + lane] : 0.0;
+                for (int r = d0 + bw + warp; r < ibo; r += NWS) {
+                    double acc = top[r * OS_LD + lane];
+                    const double *lr = Lc + (r - d0);
+#pragma unroll
+                    for (int sc = 0; sc < 32; ++sc) acc = fma(-lr[sc * OS_LDC], x[sc], acc);
+                    top[r * OS_LD + lane] = acc;
+                }
+            }
+            __syncthreads();
+        }
+        // ---- U12 back to rows [J, J + ibo)
+        for (int c = warp; c < W; c += NWS) {
+            double *gc = gA + J + (size_t)(cb + c) * ld;
+            for (int t = lane; t < ibo; t += 32) gc[t] = top[t * OS_LD + c];
+        }
+        __syncthreads();
+    }
+}
+
+// A22 -= L21 U12 of outer block [J, J + ibo) for every tier-L matrix (K = ibo)
+struct OuterTrailProb {
+    GetrfArgs a;
+    const int *list;
+    int J, NBo;
+    __device__ bool get(int slot, GemmDesc &d) const {
+        const int i = list[slot];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        d.m = 0; d.n = 0; d.k = 0;
+        if (J >= K) return false;
+        const int ibo = imin(NBo, K - J), c1 = J + ibo;
+        if (c1 >= mi || c1 >= ni) return false;
+        const long ld = a.ld[i];
+        double *A = a.A[i];
+        d.A = A + c1 + (size_t)J * ld; d.lda = ld; d.ta = 0;
+        d.B = A + J + (size_t)c1 * ld; d.ldb = ld; d.tb = 0;
+        d.C = A + c1 + (size_t)c1 * ld; d.ldc = ld;
+        d.m = mi - c1; d.n = ni - c1; d.k = ibo;
+        d.alpha = -1.0; d.beta = 1.0;
+        return true;
+    }
+};
 
 static size_t strip_smem_bytes(int nb) {
     size_t sw = (size_t)(nb * (nb + 1) + 2 * nb * GPAD) * sizeof(double);
@@ -980,7 +1171,7 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
 }
 
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans_v,
-                     cudaStream_t s) {
+                     void *outer_plans_v, cudaStream_t s) {
     SwapPlan *plans = reinterpret_cast<SwapPlan *>(plans_v);
     const Tuning &tu = tuning();
     const int nb = clamp_nb(tu.nb);
@@ -1016,10 +1207,52 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     }
     // deferred left-block interchanges (strip path only): one pass at the end
     const size_t lsw_smem = (size_t)LSW_BUF * sizeof(double) + 2 * (size_t)a.max_m * sizeof(int);
-    const bool defer = fused && tu.defer && lsw_smem <= 200 * 1024;
+    const int nbo = (tu.nb_outer / nb) * nb;
+    // two-level blocking (outer blocks of nbo columns) on the fused path; it
+    // always defers the interchanges of the columns left of the outer block
+    const bool outer = fused && nbo > nb && nbo <= NB_OUTER_MAX && lsw_smem <= 200 * 1024;
+    const bool defer = fused && (tu.defer || outer) && lsw_smem <= 200 * 1024;
     if (defer) {
         smem_optin(left_swaps_kernel, lsw_smem);
     }
+    if (outer) {
+        OuterPlan *oplans = reinterpret_cast<OuterPlan *>(outer_plans_v);
+        smem_optin(outer_swap_trsm_kernel, OS_SMEM);
+        smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0>, BIG_SMEM);
+        const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
+        const int os_chunks = (a.max_n + OS_COLS - 1) / OS_COLS;
+        const int *cnt_ptr = counters + CNT_BIN0 + BIN_L;
+        for (int J = 0; J < Kmax; J += nbo) {
+            for (int j = J; j < Kmax && j < J + nbo; j += nb) {
+                {
+                    KScope k(K_PANEL, s);
+                    panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb, plans,
+                                                                  counters + CNT_STRIPQ);
+                }
+                KScope k(K_STRIP, s);
+                if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(
+                    a, counters, bins, plans, counters + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
+                else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(
+                    a, counters, bins, plans, counters + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
+            }
+            if (J + nbo >= a.max_n) continue;  // nothing right of the block in any matrix
+            {
+                KScope k(K_SWAP_TRSM, s);
+                int g = (a.batch + OP_NT / 32 - 1) / (OP_NT / 32);
+                if (g > sms * 8) g = sms * 8;
+                outer_plan_kernel<<<g, OP_NT, 0, s>>>(a, counters, bins, J, nbo, oplans, counters + CNT_OUTQ);
+                outer_swap_trsm_kernel<<<sms * 2, OS_NT, OS_SMEM, s>>>(a, counters, bins, oplans,
+                                                                     counters + CNT_OUTQ, J, nbo, os_chunks);
+            }
+            OuterTrailProb P{a, listL, J, nbo};
+            {
+                KScope k(K_GEMM_SCAN, s);
+                xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, s>>>(P, -1, cnt_ptr, tile_off);
+            }
+            KScope k(K_GEMM_TRAIL, s);
+            xgemm_sched_kernel<OuterTrailProb, 0, 0><<<sms, X_NT, BIG_SMEM, s>>>(P, -1, cnt_ptr, tile_off);
+        }
+    } else
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {
             KScope k(K_PANEL, s);
@@ -1032,10 +1265,10 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
             KScope k(K_STRIP, s);
             if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
                                                                              counters + CNT_STRIPQ, j, nb, st_chunks, ph,
-                                                                             defer);
+                                                                             defer, -1, 1 << 30);
             else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(a, counters, bins, plans,
                                                                       counters + CNT_STRIPQ, j, nb, st_chunks, ph,
-                                                                      defer);
+                                                                      defer, -1, 1 << 30);
             continue;
         }
         {
@@ -1060,12 +1293,13 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
             }
         }
     }
-    if (defer && Kmax > nb) {
+    const int lnb = outer ? nbo : nb;  // block width of the deferred left interchanges
+    if (defer && Kmax > lnb) {
         cudaMemsetAsync(counters + CNT_LSWQ, 0, sizeof(int), s);
         KScope k(K_SWAP_TRSM, s);
         int grid = sms * 2;
         if (grid > a.batch) grid = a.batch;
-        left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, nb, a.max_m, counters + CNT_LSWQ);
+        left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, lnb, a.max_m, counters + CNT_LSWQ);
     }
 }
 

@@ -359,3 +359,35 @@ def test_pipelined_host_entry_points(chunks):
     torch.cuda.synchronize()
     assert np.array_equal(fo[0].numpy(), F.data.cpu().numpy())
     assert np.array_equal(fo[2].numpy(), F.info.cpu().numpy())
+
+
+@pytest.mark.parametrize("nb,nbo", [(32, 128), (32, 64), (16, 64), (32, 96), (16, 128)])
+def test_two_level_grid_tier(nb, nbo):
+    """Grid-wide tier with two-level blocking: inner panels of nb confined to
+    outer blocks of nbo, then one interchange + U12 solve + K = nbo GEMM
+    update of the rest per outer block.  Ragged outer / inner tails, tall,
+    wide, K < nbo, widths that end inside an outer block."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("nb", nb)
+    irr.irr_set_tuning("nb_outer", nbo)
+    shapes = [(700, 90), (1024, 64), (1025, 40), (1500, 33), (2048, 70), (513, 513), (90, 700), (600, 600),
+              (300, 17), (257, 257), (1000, 1000), (129, 400), (400, 129), (2000, 1300), (nbo + 1, nbo + 1),
+              (3 * nbo - 1, 3 * nbo + 5)]
+    _run_and_check(_uniform(shapes, seed=77 + nb + nbo))
+
+
+def test_two_level_exact_and_singular():
+    """G1 bit-exact and exact-singular through the two-level grid tier."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("tier_s", 0)
+    irr.irr_set_tuning("tier_m_max", 0)
+    irr.irr_set_tuning("nb_outer", 128)
+    shapes = [(1100, 300), (2000, 260), (600, 600), (140, 1300), (1024, 1024)]
+    mats = [irrgen.g1_exact(15, g, m, n)[0] for g, (m, n) in enumerate(shapes)]
+    _run_and_check(mats, exact=True)
+    cases = [(700, 700, 350), (1200, 300, 129), (520, 520, 0), (900, 900, 127)]
+    mats = [irrgen.g1_singular(16, g, m, n, c)[0] for g, (m, n, c) in enumerate(cases)]
+    LUs, ipivs, info, _ = gpu_getrf(mats)
+    for (m, n, c), A, LU, ip, inf in zip(cases, mats, LUs, ipivs, info):
+        assert inf == c + 1
+        check_getrf(A, LU, ip, int(inf), exact=True, label=f"sing {m}x{n}@{c}")
