@@ -113,6 +113,25 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
                       int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_getrf_partial_lapack -- the LAPACK-style variant of the partial front
+ * factorization (the factors a solver keeps):
+ *      P L U <- LU(F11)              pivoting restricted to F11's rows
+ *      F12   <- U12 = L^-1 P^T F12   (interchanges + unit-lower solve)
+ *      F21   <- L21 = F21 U^-1       (F21 IS overwritten)
+ *      F22   <- F22 - L21 U12        (the same Schur complement as
+ *                                     irr_getrf_partial in exact arithmetic)
+ * Arguments, layouts, ownership, per-front info and host errors exactly as
+ * irr_getrf_partial (F21 is writable here).  Built from the library's own
+ * building blocks (irrLASWP, irrTRSM left-lower-unit and right-upper, irrGEMM).
+ *  work         >= irr_getrf_partial_lapack_workspace_size(batch, ...).
+ * ---------------------------------------------------------------------- */
+size_t irr_getrf_partial_lapack_workspace_size(int batch, int max_n1, int max_n2);
+int irr_getrf_partial_lapack(int batch, int max_n1, int max_n2, const int *n1, const int *n2,
+                             double *const *F11, const int *ld11, double *const *F12, const int *ld12,
+                             double *const *F21, const int *ld21, double *const *F22, const int *ld22,
+                             int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * irr_gemm -- irrGEMM (§IV-C) with the expanded interface:
  *      C_i <- alpha op(A_i) op(B_i) + beta C_i      (beta == 0: C not read)
  * Local dims: C_i is m[i] x n[i]; op(A_i) is m[i] x k[i]; op(B_i) is k[i] x n[i]

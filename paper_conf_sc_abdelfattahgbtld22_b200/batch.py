@@ -154,10 +154,12 @@ class FrontBatch:
             self.work = torch.empty(max(256, nb), dtype=torch.uint8, device=self.device)
         return self.work
 
-    def getrf_partial(self, stream=None):
-        return irr.irr_getrf_partial(self.batch, self.max_n1, self.max_n2, self.n1, self.n2, self.F11, self.ld11,
-                                     self.F12, self.ld12, self.F21, self.ld21, self.F22, self.ld22, self.ipiv,
-                                     self.info, self.workspace(), stream)
+    def getrf_partial(self, stream=None, lapack=False):
+        """irr_getrf_partial (the paper's steps), or with lapack=True
+        irr_getrf_partial_lapack (F12 -> U12, F21 -> L21)."""
+        fn = irr.irr_getrf_partial_lapack if lapack else irr.irr_getrf_partial
+        return fn(self.batch, self.max_n1, self.max_n2, self.n1, self.n2, self.F11, self.ld11, self.F12, self.ld12,
+                  self.F21, self.ld21, self.F22, self.ld22, self.ipiv, self.info, self.workspace(), stream)
 
 
 # ---------------------------------------------------------------------------

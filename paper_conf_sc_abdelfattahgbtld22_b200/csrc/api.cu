@@ -391,10 +391,17 @@ size_t irr_getrf_partial_workspace_size(int batch, int max_n1, int max_n2) {
     return work_bytes_getrf(batch);
 }
 
-int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const int *n2, double *const *F11,
-                      const int *ld11, double *const *F12, const int *ld12, const double *const *F21,
-                      const int *ld21, double *const *F22, const int *ld22, int *const *ipiv, int *info, void *work,
-                      size_t work_bytes, irr_stream_t stream) {
+}  // extern "C"
+
+namespace irr {
+// The partial front factorization, both variants.  lapack == 0: the paper's
+// steps: F12 <- U^-1 L^-1 P^T F12, F22 -= F21 F12, F21 untouched.
+// lapack == 1: U12 = L^-1 P^T F12, L21 = F21 U^-1,
+// F22 -= L21 U12 (F21 overwritten by L21).
+static int partial_core(int lapack, int batch, int max_n1, int max_n2, const int *n1, const int *n2,
+                        double *const *F11, const int *ld11, double *const *F12, const int *ld12,
+                        double *const *F21, const int *ld21, double *const *F22, const int *ld22, int *const *ipiv,
+                        int *info, void *work, size_t work_bytes, irr_stream_t stream) {
     if (batch < 0) return -1;
     if (batch == 0) return IRR_SUCCESS;
     if (!n1) return -4;
@@ -418,7 +425,8 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     rc = resolve_max_dims(batch, max_n1, max_n2, n1, n2, w.counters, s);
     if (rc) return rc;
     if (max_n1 > 0 && laswp_smem(max_n1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
-    launch_partial_validate(batch, max_n1, max_n2, n1, n2, ld11, ld12, ld21, ld22, F11, F12, F21, F22, ipiv, info, s);
+    launch_partial_validate(batch, max_n1, max_n2, n1, n2, ld11, ld12, ld21, ld22, F11, F12,
+                            (const double *const *)F21, F22, ipiv, info, s);
     // step 1: P L U <- LU(F11), pivoting restricted to F11
     GetrfArgs a{batch, max_n1, max_n1, n1, n1, F11, ld11, ipiv, info};
     rc = getrf_core(a, w, 1, s);
@@ -427,32 +435,68 @@ int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const in
     // fronts sorted by n1 (descending buckets): every building-block call
     // below visits only the fronts that still have work at its offset
     launch_size_sort(n1, batch, w.sort, s);
-    // step 2: F12 <- U^-1 L^-1 P^T F12: one fused strip kernel, or
-    // irrLASWP + 2 x irrTRSM (GETRS) as the paper composes it
-    if (tuning().getrs_fused && getrs_strip_ok(max_n1)) {
-        launch_getrs_strip(batch, n1, n2, (const double *const *)F11, ld11, F12, ld12, ipiv, info, w.tile_off,
-                           w.counters + CNT_GSQ, sorted_slots(w.sort, batch, 0), s);
-    } else {
-    launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s, w.tile_off,
-                        sorted_slots(w.sort, batch, 0));
     TrsmArgs t{};
     t.side = IRR_LEFT; t.uplo = IRR_LOWER; t.trans = IRR_NO_TRANS; t.diag = IRR_UNIT;
     t.max_m = max_n1; t.max_n = max_n2; t.m = n1; t.n = n2; t.alpha = 1.0;
     t.T = (const double *const *)F11; t.Ti = 0; t.Tj = 0; t.ldt = ld11;
     t.B = F12; t.Bi = 0; t.Bj = 0; t.ldb = ld12; t.batch = batch;
-    run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
-    t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
-    run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
+    if (!lapack && tuning().getrs_fused && getrs_strip_ok(max_n1)) {
+        // step 2: F12 <- U^-1 L^-1 P^T F12: one fused strip kernel
+        launch_getrs_strip(batch, n1, n2, (const double *const *)F11, ld11, F12, ld12, ipiv, info, w.tile_off,
+                           w.counters + CNT_GSQ, sorted_slots(w.sort, batch, 0), s);
+    } else {
+        // irrLASWP + irrTRSM(L, unit) [+ irrTRSM(U)] as the paper composes GETRS
+        launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s, w.tile_off,
+                            sorted_slots(w.sort, batch, 0));
+        run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
+        if (!lapack) {
+            t.uplo = IRR_UPPER; t.diag = IRR_NON_UNIT;
+            run_trsm_masked(t, info, w.counters, w.tile_off, s, w.sort);
+        }
     }
-    // step 3: F22 <- F22 - F21 F12, F21 untouched
+    if (lapack) {
+        // L21 <- F21 U^-1: right side, upper, non-unit (the sort key n1 is the
+        // triangular dimension here too)
+        TrsmArgs r{};
+        r.side = IRR_RIGHT; r.uplo = IRR_UPPER; r.trans = IRR_NO_TRANS; r.diag = IRR_NON_UNIT;
+        r.max_m = max_n2; r.max_n = max_n1; r.m = n2; r.n = n1; r.alpha = 1.0;
+        r.T = (const double *const *)F11; r.Ti = 0; r.Tj = 0; r.ldt = ld11;
+        r.B = F21; r.Bi = 0; r.Bj = 0; r.ldb = ld21; r.batch = batch;
+        run_trsm_masked(r, info, w.counters, w.tile_off, s, w.sort);
+    }
+    // step 3: F22 <- F22 - F21 F12 / F22 - L21 U12
     GemmArgs g{};
     g.ta = 0; g.tb = 0; g.max_m = max_n2; g.max_n = max_n2; g.max_k = max_n1;
     g.m = n2; g.n = n2; g.k = n1; g.alpha = -1.0; g.beta = 1.0;
-    g.A = F21; g.Ai = 0; g.Aj = 0; g.lda = ld21;
+    g.A = (const double *const *)F21; g.Ai = 0; g.Aj = 0; g.lda = ld21;
     g.B = (const double *const *)F12; g.Bi = 0; g.Bj = 0; g.ldb = ld12;
     g.C = F22; g.Ci = 0; g.Cj = 0; g.ldc = ld22; g.batch = batch;
     launch_gemm_masked(g, info, w.counters, w.tile_off, s, sorted_slots(w.sort, batch, 0));
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+}  // namespace irr
+
+extern "C" {
+
+int irr_getrf_partial(int batch, int max_n1, int max_n2, const int *n1, const int *n2, double *const *F11,
+                      const int *ld11, double *const *F12, const int *ld12, const double *const *F21,
+                      const int *ld21, double *const *F22, const int *ld22, int *const *ipiv, int *info, void *work,
+                      size_t work_bytes, irr_stream_t stream) {
+    return partial_core(0, batch, max_n1, max_n2, n1, n2, F11, ld11, F12, ld12, (double *const *)F21, ld21, F22,
+                        ld22, ipiv, info, work, work_bytes, stream);
+}
+
+size_t irr_getrf_partial_lapack_workspace_size(int batch, int max_n1, int max_n2) {
+    (void)max_n1; (void)max_n2;
+    return work_bytes_getrf(batch);
+}
+
+int irr_getrf_partial_lapack(int batch, int max_n1, int max_n2, const int *n1, const int *n2, double *const *F11,
+                             const int *ld11, double *const *F12, const int *ld12, double *const *F21,
+                             const int *ld21, double *const *F22, const int *ld22, int *const *ipiv, int *info,
+                             void *work, size_t work_bytes, irr_stream_t stream) {
+    return partial_core(1, batch, max_n1, max_n2, n1, n2, F11, ld11, F12, ld12, F21, ld21, F22, ld22, ipiv, info,
+                        work, work_bytes, stream);
 }
 
 // Step a5.2 of the partial front on its own: X <- U^-1 L^-1 P^T B with the

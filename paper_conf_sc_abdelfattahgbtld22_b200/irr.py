@@ -26,6 +26,7 @@ IRR_SUCCESS, IRR_ERR_CUDA, IRR_ERR_WORKSPACE, IRR_ERR_UNSUPPORTED, IRR_ERR_DEVIC
 EXPORTED = (
     "irr_getrf_workspace_size", "irr_getrf", "irr_getrf_partial_workspace_size", "irr_getrf_partial",
     "irr_gemm_workspace_size", "irr_gemm", "irr_trsm_workspace_size", "irr_trsm", "irr_laswp",
+    "irr_getrf_partial_lapack_workspace_size", "irr_getrf_partial_lapack",
     "irr_getrs_workspace_size", "irr_getrs", "irr_status_words", "irr_extend_add",
     "irr_set_tuning", "irr_get_tuning", "irr_reset_tuning", "irr_launch_count", "irr_version",
     "irr_profile_enable", "irr_profile_collect", "irr_profile_num_classes", "irr_profile_class_name",
@@ -57,6 +58,10 @@ def load(path: str | None = None):
     L.irr_getrf_partial_workspace_size.restype = sz
     L.irr_getrf_partial.argtypes = [i, i, i, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
     L.irr_getrf_partial.restype = i
+    L.irr_getrf_partial_lapack_workspace_size.argtypes = [i, i, i]
+    L.irr_getrf_partial_lapack_workspace_size.restype = sz
+    L.irr_getrf_partial_lapack.argtypes = [i, i, i, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
+    L.irr_getrf_partial_lapack.restype = i
     L.irr_gemm_workspace_size.argtypes = [i]
     L.irr_gemm_workspace_size.restype = sz
     L.irr_gemm.argtypes = [i, i, i, i, i, vp, vp, vp, d, vp, i, i, vp, vp, i, i, vp, d, vp, i, i, vp, i, vp, sz, vp]
@@ -144,6 +149,18 @@ def irr_getrf_partial(batch, max_n1, max_n2, n1, n2, F11, ld11, F12, ld12, F21, 
                                   _p(F21), _p(ld21), _p(F22), _p(ld22), _p(ipiv), _p(info), _p(work),
                                   _nbytes(work), _stream(stream))
     return _check(rc, "irr_getrf_partial") if check else rc
+
+
+def irr_getrf_partial_lapack_workspace_size(batch, max_n1, max_n2):
+    return load().irr_getrf_partial_lapack_workspace_size(batch, max_n1, max_n2)
+
+
+def irr_getrf_partial_lapack(batch, max_n1, max_n2, n1, n2, F11, ld11, F12, ld12, F21, ld21, F22, ld22, ipiv,
+                             info, work, stream=None, check=True):
+    rc = load().irr_getrf_partial_lapack(batch, max_n1, max_n2, _p(n1), _p(n2), _p(F11), _p(ld11), _p(F12),
+                                         _p(ld12), _p(F21), _p(ld21), _p(F22), _p(ld22), _p(ipiv), _p(info),
+                                         _p(work), _nbytes(work), _stream(stream))
+    return _check(rc, "irr_getrf_partial_lapack") if check else rc
 
 
 def irr_getrs_workspace_size(batch):

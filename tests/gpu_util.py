@@ -83,9 +83,9 @@ def check_getrf(A0, LU, ipiv, info, exact=False, label=""):
     return "near-tie"
 
 
-def gpu_partial(fronts):
+def gpu_partial(fronts, lapack=False):
     """fronts: list of full nf x nf host arrays with their n1.  Returns the
-    factored fronts, ipivs, info."""
+    factored fronts, ipivs, info (lapack=True: irr_getrf_partial_lapack)."""
     n1 = [f[1] for f in fronts]
     n2 = [f[0].shape[0] - f[1] for f in fronts]
     B = FrontBatch(n1, n2)
@@ -94,7 +94,7 @@ def gpu_partial(fronts):
         if F.size:
             B.front(i, host)[:, :] = F
     B.data.copy_(torch.from_numpy(host))
-    B.getrf_partial()
+    B.getrf_partial(lapack=lapack)
     torch.cuda.synchronize()
     out = B.data.cpu().numpy()
     ip = B.ipiv_data.cpu().numpy()
