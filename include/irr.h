@@ -132,6 +132,25 @@ int irr_getrf_partial_lapack(int batch, int max_n1, int max_n2, const int *n1, c
                              int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_zgetrf -- variable-size batched COMPLEX LU with partial pivoting
+ * (the multifrontal solver's A is in C^{N x N},
+ * P:L71 §III-A), LAPACK zgetrf semantics: P A = L U with the pivot of step
+ * k the smallest row maximising |Re a_ik| + |Im a_ik| (izamax).
+ *  A            double*[batch]: A_i -> m_i x n_i COMPLEX matrix, column-major,
+ *               each element two doubles (re, im) as in C99 double _Complex /
+ *               std::complex<double>; 16-byte aligned; ld[i] in complex
+ *               elements (>= max(1, m_i)).  Overwritten by L (unit, strict
+ *               lower) and U.
+ *  m, n, ipiv, info, max_m, max_n, work, stream: exactly as irr_getrf
+ *               (per-matrix info -1 / -2 / -3 / -4 / -5 for bad m / n / NULL
+ *               A_i / ld / NULL ipiv_i; first exact zero pivot -> info = k).
+ *  work         >= irr_zgetrf_workspace_size(batch, max_m, max_n).
+ * ---------------------------------------------------------------------- */
+size_t irr_zgetrf_workspace_size(int batch, int max_m, int max_n);
+int irr_zgetrf(int batch, int max_m, int max_n, const int *m, const int *n, double *const *A, const int *ld,
+               int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
+
+/* ------------------------------------------------------------------------
  * irr_gemm -- irrGEMM (§IV-C) with the expanded interface:
  *      C_i <- alpha op(A_i) op(B_i) + beta C_i      (beta == 0: C not read)
  * Local dims: C_i is m[i] x n[i]; op(A_i) is m[i] x k[i]; op(B_i) is k[i] x n[i]

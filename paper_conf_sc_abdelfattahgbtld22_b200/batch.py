@@ -275,3 +275,55 @@ def getrf_partial_host(F: "FrontBatch", host_in, host_out, ipiv_out, info_out, c
     pipe.run(cuts, rng, F.data, host_in, host_out, compute,
              [(F.ipiv_data, ipiv_out, prng), (F.info, info_out, lambda a, b: (a, b))])
     return pipe
+
+
+class ZMatrixBatch:
+    """Complex batch for irr_zgetrf: matrix i is m x n complex (interleaved
+    re / im doubles), column-major with ld[i] complex elements, starting on a
+    256-byte boundary; int32 ipiv buffer, info, size and pointer arrays."""
+
+    def __init__(self, m, n, ld=None, device="cuda"):
+        self.m_h = np.asarray(m, dtype=np.int64)
+        self.n_h = np.asarray(n, dtype=np.int64)
+        self.batch = len(self.m_h)
+        self.ld_h = np.maximum(1, self.m_h) if ld is None else np.asarray(ld, dtype=np.int64)
+        self.device = torch.device(device)
+        self.offsets, total = _offsets(2 * self.ld_h * self.n_h)    # in doubles
+        self.total = total
+        self.data = torch.empty(total, dtype=torch.float64, device=self.device)
+        self.ptr = torch.from_numpy(self.data.data_ptr() + 8 * self.offsets).to(self.device)
+        self.m = torch.from_numpy(self.m_h.astype(np.int32)).to(self.device)
+        self.n = torch.from_numpy(self.n_h.astype(np.int32)).to(self.device)
+        self.ld = torch.from_numpy(self.ld_h.astype(np.int32)).to(self.device)
+        self.max_m = int(self.m_h.max()) if self.batch else 0
+        self.max_n = int(self.n_h.max()) if self.batch else 0
+        self.k_h = np.minimum(self.m_h, self.n_h)
+        self.ipiv_off, ipiv_total = _offsets(self.k_h)
+        self.ipiv_data = torch.zeros(ipiv_total, dtype=torch.int32, device=self.device)
+        self.ipiv = torch.from_numpy(self.ipiv_data.data_ptr() + 4 * self.ipiv_off).to(self.device)
+        self.info = torch.zeros(max(1, self.batch), dtype=torch.int32, device=self.device)
+        self.work = None
+
+    def matrix(self, i, flat_host: np.ndarray):
+        """complex128 view of matrix i inside a flat float64 host copy of data."""
+        o, m, n, ld = int(self.offsets[i]), int(self.m_h[i]), int(self.n_h[i]), int(self.ld_h[i])
+        if m * n == 0:
+            return np.zeros((m, n), dtype=np.complex128, order="F")
+        z = flat_host[o: o + 2 * ld * n].view(np.complex128)
+        return np.lib.stride_tricks.as_strided(z, shape=(m, n), strides=(16, 16 * ld))
+
+    def ipiv_of(self, i, ipiv_host: np.ndarray):
+        o, k = int(self.ipiv_off[i]), int(self.k_h[i])
+        return ipiv_host[o:o + k]
+
+    def workspace(self):
+        if self.work is None:
+            nb = irr.irr_zgetrf_workspace_size(self.batch, self.max_m, self.max_n)
+            self.work = torch.empty(max(256, nb), dtype=torch.uint8, device=self.device)
+        return self.work
+
+    def getrf(self, stream=None, max_m=None, max_n=None):
+        """irr_zgetrf on the whole batch (asynchronous on `stream`)."""
+        return irr.irr_zgetrf(self.batch, self.max_m if max_m is None else max_m,
+                              self.max_n if max_n is None else max_n, self.m, self.n, self.ptr, self.ld,
+                              self.ipiv, self.info, self.workspace(), stream)

@@ -79,7 +79,8 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 }
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
-                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs", "extend_add"};
+                                       "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs", "extend_add",
+                                       "zgetrf"};
 
 struct DeviceInfo {
     int sms = 0;
@@ -594,6 +595,34 @@ int irr_extend_add(int batch, int max_n2, const int *n2, const double *const *F2
     int rc = check_device();
     if (rc) return rc;
     launch_extend_add(batch, max_n2, n2, F22, ld22, rel, np, Fp, ldp, info, (cudaStream_t)stream);
+    return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
+}
+
+size_t irr_zgetrf_workspace_size(int batch, int max_m, int max_n) {
+    (void)max_m; (void)max_n;
+    return work_bytes_for(batch);
+}
+
+int irr_zgetrf(int batch, int max_m, int max_n, const int *m, const int *n, double *const *A, const int *ld,
+               int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream) {
+    if (batch < 0) return -1;
+    if (batch == 0) return IRR_SUCCESS;
+    if (!m) return -4;
+    if (!n) return -5;
+    if (!A) return -6;
+    if (!ld) return -7;
+    if (!ipiv) return -8;
+    if (!info) return -9;
+    if (!work) return -10;
+    if (work_bytes < work_bytes_for(batch)) return IRR_ERR_WORKSPACE;
+    int rc = check_device();
+    if (rc) return rc;
+    cudaStream_t s = (cudaStream_t)stream;
+    Work w = carve(work, batch);
+    rc = resolve_max_dims(batch, max_m, max_n, m, n, w.counters, s);
+    if (rc) return rc;
+    ZArgs za{batch, max_m, max_n, m, n, A, ld, ipiv, info};
+    launch_zgetrf(za, w.counters, w.keys, w.sort, s);
     return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
 }
 

@@ -44,7 +44,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, K_EXTEND_ADD, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, K_EXTEND_ADD, K_ZGETRF, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();
@@ -82,7 +82,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15, CNT_ZQ = 16,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
@@ -210,6 +210,17 @@ struct GetrfArgs {
     int *const *ipiv;
     int *info;
 };
+
+// zgetrf.cu: complex LU (interleaved re / im, ld in complex elements)
+struct ZArgs {
+    int batch, max_m, max_n;
+    const int *m, *n;
+    double *const *A;
+    const int *ld;
+    int *const *ipiv;
+    int *info;
+};
+void launch_zgetrf(const ZArgs &a, int *counters, int *keys, int *sort_ws, cudaStream_t s);
 
 // classify.cu
 void launch_extend_add(int batch, int max_n2, const int *n2, const double *const *F22, const int *ld22,

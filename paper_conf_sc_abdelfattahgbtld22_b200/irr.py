@@ -26,7 +26,7 @@ IRR_SUCCESS, IRR_ERR_CUDA, IRR_ERR_WORKSPACE, IRR_ERR_UNSUPPORTED, IRR_ERR_DEVIC
 EXPORTED = (
     "irr_getrf_workspace_size", "irr_getrf", "irr_getrf_partial_workspace_size", "irr_getrf_partial",
     "irr_gemm_workspace_size", "irr_gemm", "irr_trsm_workspace_size", "irr_trsm", "irr_laswp",
-    "irr_getrf_partial_lapack_workspace_size", "irr_getrf_partial_lapack",
+    "irr_getrf_partial_lapack_workspace_size", "irr_getrf_partial_lapack", "irr_zgetrf_workspace_size", "irr_zgetrf",
     "irr_getrs_workspace_size", "irr_getrs", "irr_status_words", "irr_extend_add",
     "irr_set_tuning", "irr_get_tuning", "irr_reset_tuning", "irr_launch_count", "irr_version",
     "irr_profile_enable", "irr_profile_collect", "irr_profile_num_classes", "irr_profile_class_name",
@@ -62,6 +62,10 @@ def load(path: str | None = None):
     L.irr_getrf_partial_lapack_workspace_size.restype = sz
     L.irr_getrf_partial_lapack.argtypes = [i, i, i, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, sz, vp]
     L.irr_getrf_partial_lapack.restype = i
+    L.irr_zgetrf_workspace_size.argtypes = [i, i, i]
+    L.irr_zgetrf_workspace_size.restype = sz
+    L.irr_zgetrf.argtypes = [i, i, i, vp, vp, vp, vp, vp, vp, vp, sz, vp]
+    L.irr_zgetrf.restype = i
     L.irr_gemm_workspace_size.argtypes = [i]
     L.irr_gemm_workspace_size.restype = sz
     L.irr_gemm.argtypes = [i, i, i, i, i, vp, vp, vp, d, vp, i, i, vp, vp, i, i, vp, d, vp, i, i, vp, i, vp, sz, vp]
@@ -161,6 +165,16 @@ def irr_getrf_partial_lapack(batch, max_n1, max_n2, n1, n2, F11, ld11, F12, ld12
                                          _p(ld12), _p(F21), _p(ld21), _p(F22), _p(ld22), _p(ipiv), _p(info),
                                          _p(work), _nbytes(work), _stream(stream))
     return _check(rc, "irr_getrf_partial_lapack") if check else rc
+
+
+def irr_zgetrf_workspace_size(batch, max_m, max_n):
+    return load().irr_zgetrf_workspace_size(batch, max_m, max_n)
+
+
+def irr_zgetrf(batch, max_m, max_n, m, n, A, ld, ipiv, info, work, stream=None, check=True):
+    rc = load().irr_zgetrf(batch, max_m, max_n, _p(m), _p(n), _p(A), _p(ld), _p(ipiv), _p(info), _p(work),
+                           _nbytes(work), _stream(stream))
+    return _check(rc, "irr_zgetrf") if check else rc
 
 
 def irr_getrs_workspace_size(batch):
