@@ -425,7 +425,6 @@ static int partial_core(int lapack, int batch, int max_n1, int max_n2, const int
     Work w = carve(work, batch);
     rc = resolve_max_dims(batch, max_n1, max_n2, n1, n2, w.counters, s);
     if (rc) return rc;
-    if (max_n1 > 0 && laswp_smem(max_n1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     launch_partial_validate(batch, max_n1, max_n2, n1, n2, ld11, ld12, ld21, ld22, F11, F12,
                             (const double *const *)F21, F22, ipiv, info, s);
     // step 1: P L U <- LU(F11), pivoting restricted to F11
@@ -550,7 +549,6 @@ int irr_getrs(irr_trans_t trans, int batch, int max_n, int max_nrhs, const int *
     Work w = carve(work, batch);
     rc = resolve_max_dims(batch, max_n, max_nrhs, n, nrhs, w.counters, s);
     if (rc) return rc;
-    if (max_n > 0 && laswp_smem(max_n) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     launch_getrs_validate(batch, max_n, max_nrhs, n, nrhs, A, lda, ipiv, B, ldb, info, s);
     if (max_n <= 0 || max_nrhs <= 0) return cudaGetLastError() == cudaSuccess ? IRR_SUCCESS : IRR_ERR_CUDA;
     if (tuning().getrs_vec && getrs_vec_ok(max_n, max_nrhs)) {
@@ -724,7 +722,6 @@ int irr_laswp(int max_n, const int *n, double *const *A, int Ai, int Aj, const i
     if (!lda) return -6;
     if (!kcount) return -9;
     if (!ipiv) return -10;
-    if (laswp_smem(k2 - k1) > 227 * 1024) return IRR_ERR_UNSUPPORTED;
     int rc = check_device();
     if (rc) return rc;
     launch_laswp_masked(max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, nullptr, (cudaStream_t)stream,

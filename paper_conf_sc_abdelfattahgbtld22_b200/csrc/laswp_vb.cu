@@ -14,6 +14,7 @@ namespace irr {
 
 constexpr int LS_NT = 256;
 constexpr int LS_COLS = 32;
+constexpr int LS_SPAN_MAX = 4096;  // interchanges per launch (shared-memory plan: 44 B each)
 
 struct LaswpArgs {
     int max_n;
@@ -162,6 +163,14 @@ void launch_laswp_masked(int max_n, const int *n, double *const *A, int Ai, int 
                          const int *kcount, int *const *ipiv, int batch, const int *mask, cudaStream_t s,
                          int *units_off, SlotList sl) {
     if (batch <= 0 || max_n <= 0 || k2 <= k1) return;
+    // long pivot ranges (the few-large regime): applied in consecutive
+    // pieces, which is the same sequence of interchanges (stream-ordered)
+    if (k2 - k1 > LS_SPAN_MAX) {
+        for (int a = k1; a < k2; a += LS_SPAN_MAX)
+            launch_laswp_masked(max_n, n, A, Ai, Aj, lda, a, a + LS_SPAN_MAX < k2 ? a + LS_SPAN_MAX : k2, kcount,
+                                ipiv, batch, mask, s, units_off, sl);
+        return;
+    }
     LaswpArgs g{max_n, n, A, Ai, Aj, lda, k1, k2, kcount, ipiv, batch, mask, (max_n + LS_COLS - 1) / LS_COLS};
     size_t smem = laswp_smem(k2 - k1);
     if (units_off) {

@@ -675,13 +675,18 @@ __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__r
 }
 
 // Windowed register panel straight on global memory (panel_win.cuh): rows
-// <= 2048 in registers (RPT = 2, 4, 8 with window 16, 8, 4), 2 CTAs / SM.
+// <= 2048 in registers (RPT = 2, 4, 8 with window 16, 8, 4), 2 CTAs / SM, by
+// 256 threads; taller panels (the few-large regime) by
+// 512 threads (<= 4096 rows, window 4) or 1024 threads (<= 8192 rows,
+// window 2); beyond that the global-memory panel_getf2.
 constexpr int PW_NT = 256;
-__global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const int *__restrict__ counters,
-                                                             const int *__restrict__ bins, int j, int nb,
-                                                             SwapPlan *__restrict__ plans, int *queue) {
+constexpr int PW_MAX_ROWS = 8192;
+template <int NT>
+__global__ void __launch_bounds__(NT, NT <= 256 ? 2 : 1) panel_win_kernel(GetrfArgs a, const int *__restrict__ counters,
+                                                                         const int *__restrict__ bins, int j, int nb,
+                                                                         SwapPlan *__restrict__ plans, int *queue) {
     extern __shared__ __align__(16) double pw_smem[];
-    PanelWinSmem<PW_NT / 32> &sm = *reinterpret_cast<PanelWinSmem<PW_NT / 32> *>(pw_smem);
+    PanelWinSmem<NT / 32> &sm = *reinterpret_cast<PanelWinSmem<NT / 32> *>(pw_smem);
     __shared__ PanelScratch sc;
     __shared__ int piv_s[NBMAX];
     const int tid = threadIdx.x;
@@ -697,11 +702,16 @@ __global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const 
         const int rows = mi - j;
         double *gP = a.A[i] + j + (size_t)j * ld;
         int z;
-        if (rows <= 2 * PW_NT) z = panel_win<PW_NT, 2, 16>(gP, ld, rows, ib, piv_s, sm);
-        else if (rows <= 4 * PW_NT) z = panel_win<PW_NT, 4, 8>(gP, ld, rows, ib, piv_s, sm);
-        else if (rows <= 8 * PW_NT) z = panel_win<PW_NT, 8, 4>(gP, ld, rows, ib, piv_s, sm);
-        else z = panel_getf2<PW_NT>(gP, ld, 0, rows, 0, ib, 0, ib, piv_s, sc);
-        if (rows <= 8 * PW_NT) {
+        bool planned = true;
+        if (NT == 256 && rows <= 2 * NT) z = panel_win<NT, 2, 16>(gP, ld, rows, ib, piv_s, sm);
+        else if (NT == 256 && rows <= 4 * NT) z = panel_win<NT, 4, 8>(gP, ld, rows, ib, piv_s, sm);
+        else if (NT <= 512 && rows <= 8 * NT) z = panel_win<NT, 8, 4>(gP, ld, rows, ib, piv_s, sm);
+        else if (NT == 1024 && rows <= 8 * NT) z = panel_win<NT, 8, 2>(gP, ld, rows, ib, piv_s, sm);
+        else {
+            z = panel_getf2<NT>(gP, ld, 0, rows, 0, ib, 0, ib, piv_s, sc);
+            planned = false;
+        }
+        if (planned) {
             // the interchange plan for the strip kernel (absolute rows)
             SwapPlan &g = plans[t];
             if (tid < ib) g.top_src[tid] = j + sm.plan.top_src[tid];
@@ -714,6 +724,20 @@ __global__ void __launch_bounds__(PW_NT, 2) panel_win_kernel(GetrfArgs a, const 
         if (tid < ib) a.ipiv[i][j + tid] = j + piv_s[tid] + 1;
         if (tid == 0 && z && a.info[i] == 0) a.info[i] = j + z;
         __syncthreads();
+    }
+}
+
+// the windowed panel for the tallest panel of the launch
+static void launch_panel_win(int max_rows, int grid, const GetrfArgs &a, int *counters, const int *bins, int j,
+                             int nb, SwapPlan *plans, int *queue, cudaStream_t s) {
+    if (max_rows <= 8 * 256) {
+        panel_win_kernel<256><<<grid, 256, sizeof(PanelWinSmem<8>), s>>>(a, counters, bins, j, nb, plans, queue);
+    } else if (max_rows <= 8 * 512) {
+        const int g = grid < num_sms() ? grid : num_sms();
+        panel_win_kernel<512><<<g, 512, sizeof(PanelWinSmem<16>), s>>>(a, counters, bins, j, nb, plans, queue);
+    } else {
+        const int g = grid < num_sms() ? grid : num_sms();
+        panel_win_kernel<1024><<<g, 1024, sizeof(PanelWinSmem<32>), s>>>(a, counters, bins, j, nb, plans, queue);
     }
 }
 
@@ -1186,8 +1210,9 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     const int sms = num_sms();
     int grid_p = sms * 2;
     if (grid_p > a.batch) grid_p = a.batch;
-    const size_t pw_smem = sizeof(PanelWinSmem<PW_NT / 32>);
-    smem_optin(panel_win_kernel, pw_smem);
+    smem_optin(panel_win_kernel<256>, sizeof(PanelWinSmem<8>));
+    smem_optin(panel_win_kernel<512>, sizeof(PanelWinSmem<16>));
+    smem_optin(panel_win_kernel<1024>, sizeof(PanelWinSmem<32>));
     int grid_w = sms * 2;
     if (grid_w > a.batch) grid_w = a.batch;
     const int chunks_per = (a.max_n + SW_COLS - 1) / SW_COLS;
@@ -1197,7 +1222,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     const size_t sw_smem = (size_t)(nb * (nb + 1) + 2 * nb * (SW_COLS + 1)) * sizeof(double);
     smem_optin(swap_trsm_kernel, sw_smem);
     const int *listL = bins + (size_t)BIN_L * a.batch;
-    const bool fused = tu.panel_win && tu.strip && a.max_m <= 8 * PW_NT;
+    const bool fused = tu.panel_win && tu.strip && a.max_m <= PW_MAX_ROWS;
     unsigned long long *ph = tu.phase_timing ? reinterpret_cast<unsigned long long *>(counters + CNT_PHASE0) : nullptr;
     const int st_chunks = (a.max_n + ST_COLS - 1) / ST_COLS;
     const size_t st_smem = strip_smem_bytes(nb);
@@ -1226,8 +1251,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
             for (int j = J; j < Kmax && j < J + nbo; j += nb) {
                 {
                     KScope k(K_PANEL, s);
-                    panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb, plans,
-                                                                  counters + CNT_STRIPQ);
+                    launch_panel_win(a.max_m - j, grid_w, a, counters, bins, j, nb, plans, counters + CNT_STRIPQ, s);
                 }
                 KScope k(K_STRIP, s);
                 if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(
@@ -1256,7 +1280,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {
             KScope k(K_PANEL, s);
-            panel_win_kernel<<<grid_w, PW_NT, pw_smem, s>>>(a, counters, bins, j, nb, plans, counters + CNT_STRIPQ);
+            launch_panel_win(a.max_m - j, grid_w, a, counters, bins, j, nb, plans, counters + CNT_STRIPQ, s);
         } else {
             KScope k(K_PANEL, s);
             panel_kernel<<<grid_p, P_NT, psmem, s>>>(a, counters, bins, j, nb, smem_rows);
