@@ -174,17 +174,27 @@ int oracle_getrf_partial(int n1, int n2, double *F11, int ld11, double *F12, int
         if (p != k)
             for (int c = 0; c < n2; ++c) { double t = F12_(k, c); F12_(k, c) = F12_(p, c); F12_(p, c) = t; }
     }
+    /* The dot products of steps 3-5 run along ROWS of F11 and F21; they read
+     * them from row-major copies (T11[i][j] = F11(i, j), T21[i][k] = F21(i, k)),
+     * which changes only where the same values are read from: every sum has
+     * the same terms in the same order. */
+    double *T11 = (double *)malloc(sizeof(double) * (size_t)(n1 > 0 ? n1 : 1) * (size_t)(n1 > 0 ? n1 : 1));
+    double *T21 = (double *)malloc(sizeof(double) * (size_t)(n1 > 0 ? n1 : 1) * (size_t)(n2 > 0 ? n2 : 1));
+    for (int j = 0; j < n1; ++j)
+        for (int i = 0; i < n1; ++i) T11[(size_t)i * n1 + j] = F11_(i, j);
+    for (int k = 0; k < n1; ++k)
+        for (int i = 0; i < n2; ++i) T21[(size_t)i * n1 + k] = F21_(i, k);
     for (int c = 0; c < n2; ++c) {
         /* step 3: L^-1 (unit lower): row i -= sum_{j<i} l_ij row j */
         for (int i = 0; i < n1; ++i) {
             double s = 0.0;
-            for (int j = 0; j < i; ++j) s = s + F11_(i, j) * F12_(j, c);
+            for (int j = 0; j < i; ++j) s = s + T11[(size_t)i * n1 + j] * F12_(j, c);
             F12_(i, c) = F12_(i, c) - s;
         }
         /* step 4: U^-1: row i = (row i - sum_{j>i} u_ij row j) / u_ii */
         for (int i = n1 - 1; i >= 0; --i) {
             double s = 0.0;
-            for (int j = i + 1; j < n1; ++j) s = s + F11_(i, j) * F12_(j, c);
+            for (int j = i + 1; j < n1; ++j) s = s + T11[(size_t)i * n1 + j] * F12_(j, c);
             F12_(i, c) = (F12_(i, c) - s) / F11_(i, i);
         }
     }
@@ -192,9 +202,11 @@ int oracle_getrf_partial(int n1, int n2, double *F11, int ld11, double *F12, int
     for (int j = 0; j < n2; ++j)
         for (int i = 0; i < n2; ++i) {
             double s = 0.0;
-            for (int k = 0; k < n1; ++k) s = s + F21_(i, k) * F12_(k, j);
+            for (int k = 0; k < n1; ++k) s = s + T21[(size_t)i * n1 + k] * F12_(k, j);
             F22_(i, j) = F22_(i, j) - s;
         }
+    free(T11);
+    free(T21);
 #undef F11_
 #undef F12_
 #undef F21_
