@@ -127,7 +127,7 @@ def tier_of(m, n, tier_m_max=24576, l1=256):
     return t
 
 
-def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
+def class_work(m, n, nb=32, tier_m_max=24576, l1=256, nbo=0):
     """Algorithmic (flops, bytes) per kernel class for one getrf step, SURVEY
     §8(d): flops = FLOPS_DGETRF of the matrices a class works on (the grid-wide
     tier's flops split by the step of the blocked algorithm each kernel
@@ -148,35 +148,51 @@ def class_work(m, n, nb=32, tier_m_max=24576, l1=256):
     mL, nL = m[sel], n[sel]
     tier_f = float(F.getrf_flops(mL, nL).sum())
     tier_b = float(F.getrf_bytes(mL, nL).sum())
-    g_f = p_f = s_f = 0.0
+    g_f = p_f = s_f = og_f = os_f = 0.0
     kL = np.minimum(mL, nL)
+    two = nbo > nb
     for j in range(0, int(kL.max()) if len(kL) else 0, nb):
         act = kL > j
         if not act.any():
             break
         mm, nn, kk = mL[act], nL[act], kL[act]
         ib = np.minimum(nb, kk - j)
+        # inner steps of the two-level tier stop at their outer block's edge
+        ce = np.minimum(kk, (j // nbo + 1) * nbo) if two else nn
         Mr = np.maximum(mm - j - ib, 0).astype(np.float64)
-        Nr = np.maximum(nn - j - ib, 0).astype(np.float64)
+        Nr = np.maximum(ce - j - ib, 0).astype(np.float64)
         g_f += float((2 * Mr * Nr * ib).sum())
         p_f += float(F.getrf_flops(mm - j, ib).sum())
         s_f += float((ib * ib * Nr).sum())
+        if two and (j + nb) % nbo == 0 or (two and np.any(kk - j <= nb)):
+            # end of an outer block [J, J + ibo) for the matrices whose block ends here
+            J = (j // nbo) * nbo
+            end = (kk <= j + nb) | ((j + nb) % nbo == 0)
+            ibo = np.minimum(nbo, kk - J)[end].astype(np.float64)
+            Mo = np.maximum(mm[end] - J - ibo, 0)
+            No = np.maximum(nn[end] - J - ibo, 0)
+            og_f += float((2 * Mo * No * ibo).sum())
+            os_f += float((ibo * ibo * No).sum())
     share = (lambda f: tier_b * f / tier_f) if tier_f > 0 else (lambda f: 0.0)
-    out["gemm_trailing"] = (g_f, share(g_f))
+    if two:
+        out["gemm_trailing"] = (og_f, share(og_f))     # xgemm, K = nbo
+        out["outer_trsm"] = (os_f, share(os_f))        # outer interchanges + U12 solve
+    else:
+        out["gemm_trailing"] = (g_f, share(g_f))
+        out["swap_trsm"] = (s_f, share(s_f))
     out["panel"] = (p_f, share(p_f))
-    out["swap_trsm"] = (s_f, share(s_f))
-    out["strip"] = (g_f + s_f, share(g_f + s_f))  # fused interchange + TRSM + GEMM kernel
+    out["strip"] = (g_f + s_f, share(g_f + s_f))  # fused interchange + TRSM + GEMM kernel (inner steps)
     out["grid_tier"] = (tier_f, tier_b)
     return out
 
 
-def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=256):
+def class_work_partial(n1, n2, nb=32, tier_m_max=24576, l1=256, nbo=0):
     """As class_work for F11, plus the partial-front steps a5.2 (2 n1^2 n2
     flops; F12 read + written, F11's factors read) and a5.3 (2 n1 n2^2 flops;
     F22 read + written, F21 and F12 read) with their read-once bytes."""
     n1 = np.asarray(n1, dtype=np.int64)
     n2 = np.asarray(n2, dtype=np.int64)
-    out = class_work(n1, n1, nb, tier_m_max, l1)
+    out = class_work(n1, n1, nb, tier_m_max, l1, nbo)
     out["gemm_dcwi"] = (float((2.0 * n1 * n2 * n2).sum()), float((8.0 * (2 * n2 * n2 + n2 * n1 + n1 * n2)).sum()))
     out["trsm_leaf"] = (float((2.0 * n1 * n1 * n2).sum()), float((16.0 * n1 * n2 + 8.0 * n1 * n1).sum()))
     out["getrs"] = (float((2.0 * n1 * n1 * n2).sum()), float((16.0 * n1 * n2 + 8.0 * n1 * n1).sum()))
@@ -331,14 +347,16 @@ def main():
         ld_loc = B.ld_h
         call = lambda: B.getrf()  # noqa: E731
         cw = class_work(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
-                        irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
+                        irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0,
+                        irr.irr_get_tuning("nb_outer"))
         bytes_local = float(F.getrf_bytes(m_loc, n_loc).sum())
         gm, gn = m_loc, n_loc
     else:
         B = FrontBatch(m_loc, n_loc, device=dev)
         call = lambda: B.getrf_partial()  # noqa: E731
         cw = class_work_partial(m_loc, n_loc, irr.irr_get_tuning("nb"), irr.irr_get_tuning("tier_m_max"),
-                                irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0)
+                                irr.irr_get_tuning("l1_rows") if irr.irr_get_tuning("l1") else 0,
+                                irr.irr_get_tuning("nb_outer"))
         bytes_local = float(F.partial_bytes(m_loc, n_loc).sum())
         gm = gn = B.nf_h
     outs = [B.data, B.ipiv_data, B.info]

@@ -80,7 +80,7 @@ void prof_record(int cls, cudaStream_t s, bool begin) {
 
 static const char *k_names[NKCLASS] = {"classify", "lu_small", "lu_mid", "panel", "swap_trsm", "gemm_scan",
                                        "gemm_trailing", "trsm_leaf", "gemm_dcwi", "laswp", "misc", "lu_l1", "strip", "getrs", "extend_add",
-                                       "zgetrf"};
+                                       "zgetrf", "outer_trsm", "left_swaps"};
 
 struct DeviceInfo {
     int sms = 0;

@@ -44,7 +44,7 @@ inline void count_launch(int k = 1) { launch_counter() += k; }
 // kernel classes for the optional per-class device timing (irr_profile_*)
 enum KClass {
     K_CLASSIFY = 0, K_LU_SMALL, K_LU_MID, K_PANEL, K_SWAP_TRSM, K_GEMM_SCAN, K_GEMM_TRAIL,
-    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, K_EXTEND_ADD, K_ZGETRF, NKCLASS
+    K_TRSM_LEAF, K_GEMM_DCWI, K_LASWP, K_MISC, K_LU_L1, K_STRIP, K_GETRS, K_EXTEND_ADD, K_ZGETRF, K_OUTER_TRSM, K_LEFT_SWAPS, NKCLASS
 };
 void prof_record(int cls, cudaStream_t s, bool begin);
 bool prof_on();

@@ -803,7 +803,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
         // lb = J, ce = min(n, cmax); columns outside it get the outer block's
         // interchanges later (outer_swap_trsm_kernel / left_swaps_kernel).
         const int lb = J >= 0 ? J : (defer ? j : 0);
-        const int ce = imin(ni, cmax);
+        const int ce = J >= 0 ? imin(imin(ni, cmax), K) : ni;  // an outer block ends at min(J + nbo, K)
         const int nright = ce > c1 ? ce - c1 : 0;
         const int vtot = (j - lb) + nright, vb = q * ST_COLS;
         if (vb >= vtot) continue;
@@ -915,8 +915,9 @@ __global__ void __launch_bounds__(OP_NT) outer_plan_kernel(GetrfArgs a, const in
         const int i = list[t];
         const int mi = a.m[i], ni = a.n[i];
         const int K = mi < ni ? mi : ni;
-        if (J >= K || J + NBo >= ni) continue;  // no columns right of the block
+        if (J >= K) continue;
         const int ibo = imin(NBo, K - J);
+        if (J + ibo >= ni) continue;  // no columns right of the block
         const int *ip = a.ipiv[i];
         for (int q = lane; q < ibo; q += 32) p.piv[q] = ip[J + q] - 1;
         __syncwarp();
@@ -934,25 +935,33 @@ __global__ void __launch_bounds__(OP_NT) outer_plan_kernel(GetrfArgs a, const in
     }
 }
 
-// Right of outer block [J, J + ibo): per (tier-L slot, OS_COLS-column strip),
-// gather the moved rows (the block's interchanges composed), scatter the rows
-// pushed below the block, solve U12 <- L11^-1 U12 in 32-row blocks (diagonal
-// block by the register substitution of the inner steps, the rows below by
-// a rank-32 update with the L column block staged in shared memory), write
-// U12 back.  Dynamic item queue (reset by outer_plan_kernel).
-constexpr int OS_COLS = 32, OS_NT = 128, OS_LD = OS_COLS + 1, OS_LDC = NB_OUTER_MAX + 1;
-constexpr size_t OS_SMEM = (size_t)(2 * NB_OUTER_MAX * OS_LD + 32 * OS_LDC) * sizeof(double);
+// Right of outer block [J, J + ibo): per (tier-L slot, OS_COLS-column strip):
+//   1. the block's interchanges composed (outer_plan_kernel): the ibo rows that
+//      end in [J, J + ibo) are gathered into shared memory (cp.async; each
+//      column's top rows are one contiguous 1 KB range), the <= ibo rows pushed
+//      below the block are read into registers and, after every read of the
+//      strip, written to their new rows;
+//   2. U12 <- L11^-1 U12 in 32-row blocks d: the diagonal block by a warp-wide
+//      substitution (lane = row, 8 columns per warp, the solved entry
+//      broadcast by shuffle), the rows below it by a rank-32 DMMA update
+//      (m8n8k4, operands in shared memory: the L column block staged once per
+//      d, U12 rows in place);
+//   3. U12 back to rows [J, J + ibo) (coalesced).
+// Dynamic item queue (reset by outer_plan_kernel).
+constexpr int OS_COLS = 64, OS_NT = 256, OS_TLD = OS_COLS + 1, OS_LDC = 136;
+constexpr int OS_BOTQ = NB_OUTER_MAX / (OS_NT / 32);  // bot rows per warp (registers)
+constexpr size_t OS_SMEM = (size_t)(NB_OUTER_MAX * OS_TLD + 32 * OS_LDC) * sizeof(double);
 __global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                                    const int *__restrict__ bins,
                                                                    const OuterPlan *__restrict__ plans, int *queue,
                                                                    int J, int NBo, int chunks_per) {
     extern __shared__ __align__(16) double os_smem[];
-    double *top = os_smem;                         // [ibo][OS_LD]
-    double *bot = top + NB_OUTER_MAX * OS_LD;      // [nbot][OS_LD]
-    double *Lc = bot + NB_OUTER_MAX * OS_LD;       // L column block: Lc[r + s * OS_LDC]
+    double *top = os_smem;                       // U12 rows: top[t * OS_TLD + c]
+    double *Lc = top + NB_OUTER_MAX * OS_TLD;    // L column block: Lc[s * OS_LDC + r]
     __shared__ OuterPlan sp;
     __shared__ int item_s;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int g = lane >> 2, t4 = lane & 3;
     constexpr int NWS = OS_NT / 32;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
@@ -983,51 +992,110 @@ __global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, 
             __syncthreads();
         }
         const int nbot = sp.nbot;
-        // ---- gather (all reads before any write of the strip)
+        // ---- 1. gather (every read of the strip before any write)
         for (int c = warp; c < W; c += NWS) {
             const double *gc = gA + (size_t)(cb + c) * ld;
-            for (int t = lane; t < ibo; t += 32) cp_async8(&top[t * OS_LD + c], gc + sp.top_src[t]);
-            for (int b = lane; b < nbot; b += 32) cp_async8(&bot[b * OS_LD + c], gc + sp.bot_src[b]);
+            for (int r = lane; r < ibo; r += 32) cp_async8(&top[r * OS_TLD + c], gc + sp.top_src[r]);
         }
         cp_async_commit();
+        double bv[OS_BOTQ][2];
+#pragma unroll
+        for (int u = 0; u < OS_BOTQ; ++u) {
+            const int b = warp + NWS * u;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int c = lane + 32 * h;
+                bv[u][h] = (b < nbot && c < W) ? gA[sp.bot_src[b] + (size_t)(cb + c) * ld] : 0.0;
+            }
+        }
         cp_async_wait<0>();
         __syncthreads();
-        // ---- the rows pushed below the block: final for this step
-        for (int c = warp; c < W; c += NWS) {
-            double *gc = gA + (size_t)(cb + c) * ld;
-            for (int b = lane; b < nbot; b += 32) gc[sp.bot_pos[b]] = bot[b * OS_LD + c];
+#pragma unroll
+        for (int u = 0; u < OS_BOTQ; ++u) {
+            const int b = warp + NWS * u;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int c = lane + 32 * h;
+                if (b < nbot && c < W) gA[sp.bot_pos[b] + (size_t)(cb + c) * ld] = bv[u][h];
+            }
         }
-        // ---- U12 <- L11^-1 U12, 32-row blocks
+        // ---- 2. U12 <- L11^-1 U12, 32-row blocks
         for (int d0 = 0; d0 < ibo; d0 += 32) {
             const int bw = imin(32, ibo - d0);
-            // L11 rows [d0, ibo) x cols [d0, d0 + bw) (column block, incl. the diagonal block)
+            const int below = ibo - d0 - bw;   // rows under the diagonal block
             for (int sc = warp; sc < bw; sc += NWS) {
-                const double *gl = gA + J + (size_t)(J + d0 + sc) * ld;
-                for (int r = d0 + lane; r < ibo; r += 32) cp_async8(&Lc[(r - d0) + sc * OS_LDC], gl + r);
+                const double *gl = gA + J + d0 + (size_t)(J + d0 + sc) * ld;
+                for (int r = lane; r < ibo - d0; r += 32) cp_async8(&Lc[sc * OS_LDC + r], gl + r);
             }
             cp_async_commit();
             cp_async_wait<0>();
             __syncthreads();
-            if (tid < W) trsm_col_regs<32>(top + d0 * OS_LD + tid, OS_LD, bw, Lc, OS_LDC);
+            // diagonal block: warp w solves columns [8w, 8w + 8), lane = row
+            {
+                const int c0 = warp * 8;
+                double x[8];
+#pragma unroll
+                for (int c = 0; c < 8; ++c) x[c] = (lane < bw && c0 + c < W) ? top[(d0 + lane) * OS_TLD + c0 + c] : 0.0;
+                for (int s = 0; s < bw - 1; ++s) {
+                    const double l = (lane > s && lane < bw) ? Lc[s * OS_LDC + lane] : 0.0;
+#pragma unroll
+                    for (int c = 0; c < 8; ++c) x[c] = fma(-l, __shfl_sync(FULL, x[c], s), x[c]);
+                }
+                if (lane < bw)
+#pragma unroll
+                    for (int c = 0; c < 8; ++c)
+                        if (c0 + c < W) top[(d0 + lane) * OS_TLD + c0 + c] = x[c];
+            }
             __syncthreads();
-            if (d0 + bw < ibo && lane < W) {
-                double x[32];
+            // rows below: C[r][c] -= sum_s Lc[s][bw + r] * X[s][c], 32 x 32 output tiles per warp (DMMA)
+            if (below > 0) {
+                const int tiles_m = (below + 31) / 32, tiles = tiles_m * 2;
+                for (int tt = warp; tt < tiles; tt += NWS) {
+                    const int rb = (tt % tiles_m) * 32, cbt = (tt / tiles_m) * 32;
+                    double acc[4][4][2];
 #pragma unroll
-                for (int sc = 0; sc < 32; ++sc) x[sc] = sc < bw ? top[(d0 + sc) * OS_LD + lane] : 0.0;
-                for (int r = d0 + bw + warp; r < ibo; r += NWS) {
-                    double acc = top[r * OS_LD + lane];
-                    const double *lr = Lc + (r - d0);
+                    for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-                    for (int sc = 0; sc < 32; ++sc) acc = fma(-lr[sc * OS_LDC], x[sc], acc);
-                    top[r * OS_LD + lane] = acc;
+                        for (int n8 = 0; n8 < 4; ++n8) { acc[mi][n8][0] = 0.0; acc[mi][n8][1] = 0.0; }
+#pragma unroll
+                    for (int ks = 0; ks < 32; ks += 4) {
+                        const int s = ks + t4;
+                        double av[4], bvv[4];
+#pragma unroll
+                        for (int mi = 0; mi < 4; ++mi) {
+                            const int r = rb + 8 * mi + g;   // row under the block
+                            av[mi] = (s < bw && r < below) ? Lc[s * OS_LDC + bw + r] : 0.0;
+                        }
+#pragma unroll
+                        for (int n8 = 0; n8 < 4; ++n8) {
+                            const int c = cbt + 8 * n8 + g;
+                            bvv[n8] = (s < bw && c < W) ? top[(d0 + s) * OS_TLD + c] : 0.0;
+                        }
+#pragma unroll
+                        for (int mi = 0; mi < 4; ++mi)
+#pragma unroll
+                            for (int n8 = 0; n8 < 4; ++n8) dmma_8x8x4(acc[mi][n8][0], acc[mi][n8][1], av[mi], bvv[n8]);
+                    }
+#pragma unroll
+                    for (int mi = 0; mi < 4; ++mi) {
+                        const int r = rb + 8 * mi + g;
+                        if (r >= below) continue;
+                        double *row = top + (size_t)(d0 + bw + r) * OS_TLD;
+#pragma unroll
+                        for (int n8 = 0; n8 < 4; ++n8) {
+                            const int c = cbt + 8 * n8 + 2 * t4;
+                            if (c < W) row[c] -= acc[mi][n8][0];
+                            if (c + 1 < W) row[c + 1] -= acc[mi][n8][1];
+                        }
+                    }
                 }
             }
             __syncthreads();
         }
-        // ---- U12 back to rows [J, J + ibo)
+        // ---- 3. U12 back to rows [J, J + ibo)
         for (int c = warp; c < W; c += NWS) {
             double *gc = gA + J + (size_t)(cb + c) * ld;
-            for (int t = lane; t < ibo; t += 32) gc[t] = top[t * OS_LD + c];
+            for (int r = lane; r < ibo; r += 32) gc[r] = top[r * OS_TLD + c];
         }
         __syncthreads();
     }
@@ -1259,12 +1327,14 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                 else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(
                     a, counters, bins, plans, counters + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
             }
-            if (J + nbo >= a.max_n) continue;  // nothing right of the block in any matrix
             {
-                KScope k(K_SWAP_TRSM, s);
+                KScope k(K_MISC, s);
                 int g = (a.batch + OP_NT / 32 - 1) / (OP_NT / 32);
                 if (g > sms * 8) g = sms * 8;
                 outer_plan_kernel<<<g, OP_NT, 0, s>>>(a, counters, bins, J, nbo, oplans, counters + CNT_OUTQ);
+            }
+            {
+                KScope k(K_OUTER_TRSM, s);
                 outer_swap_trsm_kernel<<<sms * 2, OS_NT, OS_SMEM, s>>>(a, counters, bins, oplans,
                                                                      counters + CNT_OUTQ, J, nbo, os_chunks);
             }
@@ -1320,7 +1390,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     const int lnb = outer ? nbo : nb;  // block width of the deferred left interchanges
     if (defer && Kmax > lnb) {
         cudaMemsetAsync(counters + CNT_LSWQ, 0, sizeof(int), s);
-        KScope k(K_SWAP_TRSM, s);
+        KScope k(K_LEFT_SWAPS, s);
         int grid = sms * 2;
         if (grid > a.batch) grid = a.batch;
         left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, lnb, a.max_m, counters + CNT_LSWQ);

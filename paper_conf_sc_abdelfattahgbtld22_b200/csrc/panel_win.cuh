@@ -218,7 +218,7 @@ __device__ int panel_win(double *gP, long ld, int rows, int ib, int *piv, PanelW
         if (WB >= 8)
             for (; c < bend && bend - c > 4; ++c)
                 pwin_step<NT, RPT, WB, (WB >= 8 ? 8 : WB), NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
-        for (; c < bend; ++c) pwin_step<NT, RPT, WB, 4, NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
+        for (; c < bend; ++c) pwin_step<NT, RPT, WB, (WB >= 4 ? 4 : WB), NBX>(a, pos, c, bend, gP, ld, rows, piv, sm, zero_at);
         __syncthreads();
     }
     // ---- the permutation: L of the last window's pivots, and of the rows
