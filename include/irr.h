@@ -151,6 +151,20 @@ int irr_zgetrf(int batch, int max_m, int max_n, const int *m, const int *n, doub
                int *const *ipiv, int *info, void *work, size_t work_bytes, irr_stream_t stream);
 
 /* ------------------------------------------------------------------------
+ * irr_shard_lpt / irr_shard_lpt_work -- flop-balanced partition of a batch
+ * over `parts` GPUs of one box (north_star: "fronts are
+ * partitioned flop-balanced across the GPUs").  HOST arrays, host code, no
+ * CUDA.  Longest-processing-time first: items by work descending (index
+ * ascending on ties), each to the least-loaded part (lowest id on ties);
+ * deterministic.  irr_shard_lpt weighs matrix i by FLOPS_DGETRF(m[i], n[i])
+ * (reading Q1); irr_shard_lpt_work takes the weights (e.g. partial-front
+ * flops, reading Q2).  owner[i] in [0, parts).  Returns 0 or -(position) of
+ * a bad argument.
+ * ---------------------------------------------------------------------- */
+int irr_shard_lpt(int batch, const int *m, const int *n, int parts, int *owner);
+int irr_shard_lpt_work(int batch, const double *work, int parts, int *owner);
+
+/* ------------------------------------------------------------------------
  * irr_gemm -- irrGEMM (§IV-C) with the expanded interface:
  *      C_i <- alpha op(A_i) op(B_i) + beta C_i      (beta == 0: C not read)
  * Local dims: C_i is m[i] x n[i]; op(A_i) is m[i] x k[i]; op(B_i) is k[i] x n[i]

@@ -325,7 +325,6 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "panel_win")) g_tuning.panel_win = value ? 1 : 0;
     else if (!strcmp(key, "strip")) g_tuning.strip = value ? 1 : 0;
     else if (!strcmp(key, "gemm_big")) g_tuning.gemm_big = value ? 1 : 0;
-    else if (!strcmp(key, "l1_rowmap")) g_tuning.l1_rowmap = value ? 1 : 0;
     else if (!strcmp(key, "getrs_fused")) g_tuning.getrs_fused = value ? 1 : 0;
     else if (!strcmp(key, "getrs_vec")) g_tuning.getrs_vec = value ? 1 : 0;
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
@@ -349,7 +348,6 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "panel_win")) return g_tuning.panel_win;
     if (!strcmp(key, "strip")) return g_tuning.strip;
     if (!strcmp(key, "gemm_big")) return g_tuning.gemm_big;
-    if (!strcmp(key, "l1_rowmap")) return g_tuning.l1_rowmap;
     if (!strcmp(key, "getrs_fused")) return g_tuning.getrs_fused;
     if (!strcmp(key, "getrs_vec")) return g_tuning.getrs_vec;
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;

@@ -23,7 +23,13 @@
 
 namespace irr {
 
-constexpr int XBM = 128, XBN = 128, XBK = 16, X_NT = 256, XST = 4;
+#ifndef XGEMM_ST
+#define XGEMM_ST 4      // cp.async ring depth (K chunks in flight)
+#endif
+#ifndef XGEMM_MINB
+#define XGEMM_MINB 1    // resident CTAs per SM
+#endif
+constexpr int XBM = 128, XBN = 128, XBK = 16, X_NT = 256, XST = XGEMM_ST;
 constexpr int XLD_KM = 132;  // [k][m] layout: XBK rows of XBM (+4)
 constexpr int XLD_MK = 20;   // [m][k] layout: XBM rows of XBK (+4)
 constexpr int XSTAGE = 2560; // doubles per operand stage: max(16 * 132, 128 * 20)
@@ -235,7 +241,7 @@ __global__ void __launch_bounds__(1024) xgemm_scan_kernel(Prob P, int count, con
 
 // Persistent: CTA b owns the tiles whose weighted start lies in its 1/G share.
 template <class Prob, int TA, int TB>
-__global__ void __launch_bounds__(X_NT, 1) xgemm_sched_kernel(Prob P, int count, const int *count_ptr,
+__global__ void __launch_bounds__(X_NT, XGEMM_MINB) xgemm_sched_kernel(Prob P, int count, const int *count_ptr,
                                                              const int *__restrict__ tile_off) {
     extern __shared__ __align__(16) unsigned char x_smem[];
     BigSmem &sm = *reinterpret_cast<BigSmem *>(x_smem);
@@ -292,7 +298,7 @@ struct SizeFilter {
 template <class Prob, int TA, int TB>
 inline void xgemm_launch_t(const Prob &P, int cnt, const int *cnt_ptr, const int *tile_off, cudaStream_t s) {
     smem_optin(xgemm_sched_kernel<Prob, TA, TB>, BIG_SMEM);
-    xgemm_sched_kernel<Prob, TA, TB><<<num_sms(), X_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+    xgemm_sched_kernel<Prob, TA, TB><<<num_sms() * XGEMM_MINB, X_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
 }
 
 // one persistent CTA per SM; the transposes select the shared layouts

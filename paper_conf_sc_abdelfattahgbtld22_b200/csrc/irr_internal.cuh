@@ -28,7 +28,7 @@ struct Tuning {
     int panel_win;       // 1: grid-wide panels by the windowed register panel (rows <= 2048)
     int strip;           // 1: fused interchange + TRSM + GEMM per 64-column strip (needs panel_win)
     int gemm_big;        // 1: long-K DCWI GEMMs on the 128x128 DMMA core (gemm_big.cuh)
-    int l1_rowmap;       // 1: L1 kernel in row-map form (no interchanges until one final permutation)
+    int unused_;         // (was: row-map L1 variant, measured slower in round 1, removed)
     int getrs_fused;     // 1: partial-front step a5.2 by the fused strip kernel (getrs_strip.cu)
     int l1_rows;         // max rows of the CTA-per-matrix tier (<= L1_TALL_ROWS)
     int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)

@@ -437,197 +437,6 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
     }
 }
 
-// ================================================================== L1, row-map form
-// Same CTA-per-matrix schedule as lu_l1_kernel, but rows never move while the
-// matrix is factored: rowid[r] (shared memory) is the storage row that holds
-// LAPACK row r after the interchanges so far.  A panel interchange is a
-// relabelling of rowid (P:L192's "rehearsal" becomes the only bookkeeping);
-// the panel is gathered through rowid, written back through the new rowid,
-// U12 is solved in place on the pivot rows, and the trailing GEMM reads /
-// writes its rows through rowid.  One permutation per column at the very end
-// puts every row in LAPACK order.  Compared with swapping eagerly this drops
-// the interchanges of the left block and of the rows pushed below the panel
-// (a gather + scatter of up to 2 ib rows over n - ib columns per panel, one
-// 32-byte sector per 8-byte element) in favour of one read + one write of
-// each column from L2.
-__device__ __forceinline__ void u12_chunk(double *__restrict__ gA, long ld, int cb, int W, const int *__restrict__ prow,
-                                          int ib, const double *L11p, double *top) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    constexpr int LT = SW_COLS + 1;
-    // lane = pivot row (ib <= 32): its storage row is read once
-    const bool on = lane < ib;
-    const int pr = on ? prow[lane] : 0;
-    if (on)
-        for (int c = warp; c < W; c += L1_NT / 32) cp_async8(&top[lane * LT + c], gA + pr + (size_t)(cb + c) * ld);
-    cp_async_commit();
-    cp_async_wait<0>();
-    __syncthreads();
-    if (tid < W) trsm_col_regs<32>(top + tid, LT, ib, L11p, 0);
-    __syncthreads();
-    if (on)
-        for (int c = warp; c < W; c += L1_NT / 32) gA[pr + (size_t)(cb + c) * ld] = top[lane * LT + c];
-}
-
-template <bool DMMA>
-__global__ void __launch_bounds__(L1_NT, 3) lu_l1map_kernel(GetrfArgs a, int *__restrict__ counters,
-                                                            const int *__restrict__ bins, int nb,
-                                                            int l1_region_doubles, int phase_timing) {
-    extern __shared__ __align__(16) unsigned char l1_smem[];
-    __shared__ __align__(16) PanelRegScratch<L1_NT / 32, 32> prs;
-    __shared__ SwapPlan sp;
-    __shared__ int piv_s[NBMAX];
-    __shared__ int next_s;
-    double *smd = reinterpret_cast<double *>(l1_smem);
-    GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(l1_smem);
-    double *L11p = smd + l1_region_doubles;
-    int *rowid = reinterpret_cast<int *>(L11p + (nb * (nb - 1)) / 2 + 2);
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int count = counters[CNT_BIN0 + BIN_L1];
-    const int *list = bins + (size_t)BIN_L1 * a.batch;
-    unsigned long long *ph = reinterpret_cast<unsigned long long *>(counters + CNT_PHASE0);
-#define L1_PHASE(k)                                                                   \
-    if (phase_timing && tid == 0) {                                                   \
-        long long t1 = clock64();                                                     \
-        atomicAdd(ph + (k), (unsigned long long)(t1 - t0));                           \
-        t0 = t1;                                                                      \
-    }
-    while (true) {
-        if (tid == 0) next_s = atomicAdd(&counters[CNT_L1_NEXT], 1);
-        __syncthreads();
-        const int t = next_s;
-        if (t >= count) break;
-        const int i = list[t];
-        const int mi = a.m[i], ni = a.n[i];
-        const long ld = a.ld[i];
-        double *gA = a.A[i];
-        int *gip = a.ipiv[i];
-        const int K = mi < ni ? mi : ni;
-        int info = 0;
-        long long t0 = phase_timing ? clock64() : 0;
-        for (int r = tid; r < mi; r += L1_NT) rowid[r] = r;
-        __syncthreads();
-        for (int j = 0; j < K; j += nb) {
-            const int ib = K - j < nb ? K - j : nb;
-            const int rows = mi - j, c1 = j + ib;
-            // ---- a4.1 panel: gather LAPACK rows j.. through rowid
-            double *P = smd;
-            const int ldp = rows | 1;
-            {
-                // lanes over rows, each lane's <= 8 storage rows read once
-                int sr[L1_MAX_ROWS / 32];
-#pragma unroll
-                for (int q = 0; q < L1_MAX_ROWS / 32; ++q) sr[q] = (lane + 32 * q < rows) ? rowid[j + lane + 32 * q] : -1;
-                for (int c = warp; c < ib; c += L1_NT / 32) {
-                    const double *gc = gA + (size_t)(j + c) * ld;
-#pragma unroll
-                    for (int q = 0; q < L1_MAX_ROWS / 32; ++q)
-                        if (sr[q] >= 0) cp_async8(&P[lane + 32 * q + c * ldp], gc + sr[q]);
-                }
-            }
-            cp_async_commit();
-            cp_async_wait<0>();
-            __syncthreads();
-            L1_PHASE(3)
-            const int z = panel_regs<L1_NT, 2, 32>(P, ldp, rows, ib, piv_s, prs, &sp, j);
-            L1_PHASE(4)
-            if (z && !info) info = j + z;
-            // ---- the interchanges as a relabelling of rowid (plan in LAPACK rows)
-            {
-                const int nbot = sp.nbot;
-                int vt = 0, vb = 0;
-                if (tid < ib) vt = rowid[sp.top_src[tid]];
-                if (tid >= 64 && tid - 64 < nbot) vb = rowid[sp.bot_src[tid - 64]];
-                __syncthreads();
-                if (tid < ib) rowid[j + tid] = vt;
-                if (tid >= 64 && tid - 64 < nbot) rowid[sp.bot_pos[tid - 64]] = vb;
-                __syncthreads();
-            }
-            // ---- panel back to its storage rows; strict lower L11 packed by columns
-            {
-                int sr[L1_MAX_ROWS / 32];
-#pragma unroll
-                for (int q = 0; q < L1_MAX_ROWS / 32; ++q) sr[q] = (lane + 32 * q < rows) ? rowid[j + lane + 32 * q] : -1;
-                for (int c = warp; c < ib; c += L1_NT / 32) {
-                    double *gc = gA + (size_t)(j + c) * ld;
-                    const double *pc = P + c * ldp;
-#pragma unroll
-                    for (int q = 0; q < L1_MAX_ROWS / 32; ++q)
-                        if (sr[q] >= 0) gc[sr[q]] = pc[lane + 32 * q];
-                    double *lc = L11p + (c * (2 * ib - c - 1)) / 2 - (c + 1);
-                    for (int r = c + 1 + lane; r < ib; r += 32) lc[r] = pc[r];
-                }
-            }
-            if (tid < ib) gip[j + tid] = piv_s[tid] + j + 1;
-            __syncthreads();
-            L1_PHASE(0)
-            // ---- a4.3 U12 <- L11^-1 A12 in place on the pivot rows
-            for (int cb = c1; cb < ni; cb += SW_COLS) {
-                u12_chunk(gA, ld, cb, imin(SW_COLS, ni - cb), rowid + j, ib, L11p, smd);
-                __syncthreads();
-            }
-            L1_PHASE(5)
-            // ---- a4.4 trailing update through rowid
-            if (c1 < mi && c1 < ni) {
-                GemmDesc d0;
-                d0.A = gA + (size_t)j * ld; d0.lda = ld; d0.ta = 0;
-                d0.B = gA + (size_t)c1 * ld; d0.ldb = ld; d0.tb = 0;
-                d0.C = gA + (size_t)c1 * ld; d0.ldc = ld;
-                d0.m = mi - c1; d0.n = ni - c1; d0.k = ib;
-                d0.alpha = -1.0; d0.beta = 1.0;
-                d0.rmap = rowid + c1; d0.kmap = rowid + j;
-                const int ntm = (d0.m + GBM - 1) / GBM, ntiles = ntm * ((d0.n + GBN - 1) / GBN);
-                int tt = 0;
-                auto next = [&](GemmDesc &d, int &r0, int &cc0) -> bool {
-                    if (tt >= ntiles) return false;
-                    d = d0;
-                    r0 = (tt % ntm) * GBM;
-                    cc0 = (tt / ntm) * GBN;
-                    ++tt;
-                    return true;
-                };
-                gemm_tile_stream<DMMA, decltype(next), true>(next, gsm);
-            }
-            __syncthreads();
-            L1_PHASE(2)
-        }
-        // ---- LAPACK row order: column block by column block through shared memory
-        {
-            bool moved = false;
-            for (int r = tid; r < mi; r += L1_NT) moved |= rowid[r] != r;
-            if (__syncthreads_or(moved)) {
-                int CB = l1_region_doubles / mi;
-                if (CB > ni) CB = ni;
-                for (int c0 = 0; c0 < ni; c0 += CB) {
-                    const int W = imin(CB, ni - c0);
-                    for (int c = warp; c < W; c += L1_NT / 32) {
-                        const double *gc = gA + (size_t)(c0 + c) * ld;
-                        for (int r = lane; r < mi; r += 32) cp_async8(&smd[c * mi + r], gc + r);
-                    }
-                    cp_async_commit();
-                    cp_async_wait<0>();
-                    __syncthreads();
-                    int sr[L1_MAX_ROWS / 32];
-#pragma unroll
-                    for (int q = 0; q < L1_MAX_ROWS / 32; ++q) {
-                        const int r = lane + 32 * q;
-                        sr[q] = (r < mi && rowid[r] != r) ? rowid[r] : -1;
-                    }
-                    for (int c = warp; c < W; c += L1_NT / 32) {
-                        double *gc = gA + (size_t)(c0 + c) * ld;
-#pragma unroll
-                        for (int q = 0; q < L1_MAX_ROWS / 32; ++q)
-                            if (sr[q] >= 0) gc[lane + 32 * q] = smd[c * mi + sr[q]];
-                    }
-                    __syncthreads();
-                }
-            }
-        }
-        L1_PHASE(6)
-        if (tid == 0) a.info[i] = info;
-    }
-#undef L1_PHASE
-}
-
 // ================================================================== L2
 __global__ void __launch_bounds__(P_NT) panel_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                      const int *__restrict__ bins, int j, int nb, int smem_rows) {
@@ -1237,18 +1046,6 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     KScope k(K_LU_L1, s);
-    if (tuning().l1_rowmap && nb <= 32 && tuning().l1_rows <= L1_MAX_ROWS) {
-        const size_t smem_map = smem + (size_t)L1_MAX_ROWS * sizeof(int);
-        smem_optin(lu_l1map_kernel<true>, smem_map);
-        smem_optin(lu_l1map_kernel<false>, smem_map);
-        if (tuning().l1_dmma)
-            lu_l1map_kernel<true><<<grid, L1_NT, smem_map, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
-                                                                tuning().phase_timing);
-        else
-            lu_l1map_kernel<false><<<grid, L1_NT, smem_map, s>>>(a, counters, bins, nb, (int)(region / sizeof(double)),
-                                                                 tuning().phase_timing);
-        return;
-    }
     // the tall-panel variant only when the bin can hold > 256 rows (it needs
     // more registers: the default variant keeps the lower spill count)
     const bool tall = tuning().l1_rows > L1_MAX_ROWS;
@@ -1344,7 +1141,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                 xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, s>>>(P, -1, cnt_ptr, tile_off);
             }
             KScope k(K_GEMM_TRAIL, s);
-            xgemm_sched_kernel<OuterTrailProb, 0, 0><<<sms, X_NT, BIG_SMEM, s>>>(P, -1, cnt_ptr, tile_off);
+            xgemm_sched_kernel<OuterTrailProb, 0, 0><<<sms * XGEMM_MINB, X_NT, BIG_SMEM, s>>>(P, -1, cnt_ptr, tile_off);
         }
     } else
     for (int j = 0; j < Kmax; j += nb) {

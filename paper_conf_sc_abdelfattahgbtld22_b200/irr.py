@@ -27,6 +27,7 @@ EXPORTED = (
     "irr_getrf_workspace_size", "irr_getrf", "irr_getrf_partial_workspace_size", "irr_getrf_partial",
     "irr_gemm_workspace_size", "irr_gemm", "irr_trsm_workspace_size", "irr_trsm", "irr_laswp",
     "irr_getrf_partial_lapack_workspace_size", "irr_getrf_partial_lapack", "irr_zgetrf_workspace_size", "irr_zgetrf",
+    "irr_shard_lpt", "irr_shard_lpt_work",
     "irr_getrs_workspace_size", "irr_getrs", "irr_status_words", "irr_extend_add",
     "irr_set_tuning", "irr_get_tuning", "irr_reset_tuning", "irr_launch_count", "irr_version",
     "irr_profile_enable", "irr_profile_collect", "irr_profile_num_classes", "irr_profile_class_name",
@@ -66,6 +67,10 @@ def load(path: str | None = None):
     L.irr_zgetrf_workspace_size.restype = sz
     L.irr_zgetrf.argtypes = [i, i, i, vp, vp, vp, vp, vp, vp, vp, sz, vp]
     L.irr_zgetrf.restype = i
+    L.irr_shard_lpt.argtypes = [i, vp, vp, i, vp]
+    L.irr_shard_lpt.restype = i
+    L.irr_shard_lpt_work.argtypes = [i, vp, i, vp]
+    L.irr_shard_lpt_work.restype = i
     L.irr_gemm_workspace_size.argtypes = [i]
     L.irr_gemm_workspace_size.restype = sz
     L.irr_gemm.argtypes = [i, i, i, i, i, vp, vp, vp, d, vp, i, i, vp, vp, i, i, vp, d, vp, i, i, vp, i, vp, sz, vp]
@@ -175,6 +180,16 @@ def irr_zgetrf(batch, max_m, max_n, m, n, A, ld, ipiv, info, work, stream=None, 
     rc = load().irr_zgetrf(batch, max_m, max_n, _p(m), _p(n), _p(A), _p(ld), _p(ipiv), _p(info), _p(work),
                            _nbytes(work), _stream(stream))
     return _check(rc, "irr_zgetrf") if check else rc
+
+
+def irr_shard_lpt_work(work, parts: int):
+    """Host LPT partition through the C ABI: owner (int32 numpy array)."""
+    import numpy as np
+    w = np.ascontiguousarray(work, dtype=np.float64)
+    owner = np.zeros(max(1, len(w)), dtype=np.int32)
+    rc = load().irr_shard_lpt_work(len(w), w.ctypes.data, int(parts), owner.ctypes.data)
+    _check(rc, "irr_shard_lpt_work")
+    return owner[: len(w)]
 
 
 def irr_getrs_workspace_size(batch):

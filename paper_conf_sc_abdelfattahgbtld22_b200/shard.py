@@ -15,7 +15,17 @@ import numpy as np
 def lpt_partition(work, parts: int) -> np.ndarray:
     """Longest-processing-time-first greedy: items sorted by decreasing work,
     each given to the currently least-loaded part (ties -> lowest part id).
-    Returns owner[i] in [0, parts).  Deterministic."""
+    Returns owner[i] in [0, parts).  Deterministic.  Computed by the C ABI's
+    irr_shard_lpt_work (host code in libirr.so)."""
+    from . import irr
+    work = np.asarray(work, dtype=np.float64)
+    if parts <= 1 or len(work) == 0:
+        return np.zeros(len(work), dtype=np.int64)
+    return irr.irr_shard_lpt_work(work, parts).astype(np.int64)
+
+
+def lpt_partition_reference(work, parts: int) -> np.ndarray:
+    """The same greedy in Python (tests compare the C ABI against it)."""
     work = np.asarray(work, dtype=np.float64)
     owner = np.zeros(len(work), dtype=np.int64)
     if parts <= 1 or len(work) == 0:

@@ -69,16 +69,11 @@ def test_tier_m_boundary_and_extreme_shapes(tier_m_max):
     _run_and_check(_uniform(shapes, seed=5))
 
 
-@pytest.mark.parametrize("l1", [1, 0, "rowmap"])
+@pytest.mark.parametrize("l1", [1, 0])
 @pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
 def test_tier_l_forced_small_nb(nb, l1):
     """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256,
-    "rowmap": the same in row-map form (interchanges as a relabelling, one
-    final permutation), l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1
-    sizes."""
-    if l1 == "rowmap":
-        irr.irr_set_tuning("l1_rowmap", 1)
-        l1 = 1
+    l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
     irr.irr_set_tuning("tier_s", 0)
     irr.irr_set_tuning("tier_m_max", 0)
     irr.irr_set_tuning("nb", nb)
@@ -109,19 +104,19 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "M", "L", "L2", "Lswap", "Ltall"])
+@pytest.mark.parametrize("tier", ["default", "M", "L", "L2", "L2two", "Ltall"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
     if tier == "M":
         irr.irr_set_tuning("tier_m_max", 24576)
-    if tier == "Lswap":
-        irr.irr_set_tuning("l1_rowmap", 1)
     if tier == "Ltall":
         irr.irr_set_tuning("l1_rows", 1024)
-    if tier in ("L", "L2", "Lswap", "Ltall"):
+    if tier == "L2two":
+        irr.irr_set_tuning("nb_outer", 128)
+    if tier in ("L", "L2", "L2two", "Ltall"):
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
-    if tier == "L2":
+    if tier in ("L2", "L2two"):
         irr.irr_set_tuning("l1", 0)
     shapes = [(1, 1), (5, 5), (32, 32), (32, 17), (17, 32), (33, 33), (64, 20), (20, 64), (130, 130),
               (150, 160), (257, 100), (100, 257), (300, 300)]
@@ -391,3 +386,37 @@ def test_two_level_exact_and_singular():
     for (m, n, c), A, LU, ip, inf in zip(cases, mats, LUs, ipivs, info):
         assert inf == c + 1
         check_getrf(A, LU, ip, int(inf), exact=True, label=f"sing {m}x{n}@{c}")
+
+
+def test_results_bitwise_identical_across_shard_counts():
+    """a C5-shaped batch factored as G = 1, 2, 4, 8 LPT
+    shards (one irr_getrf per shard, inputs keyed by global id) gives
+    bitwise the same factors, pivots and status words per global matrix."""
+    from paper_conf_sc_abdelfattahgbtld22_b200 import flops as F
+    from paper_conf_sc_abdelfattahgbtld22_b200.batch import MatrixBatch
+    from paper_conf_sc_abdelfattahgbtld22_b200.shard import lpt_partition
+    cfg = irrgen.config("C5", scale=0.01)
+    w = F.getrf_flops(cfg.m, cfg.n)
+    ref = None
+    for G in (1, 2, 4, 8):
+        owner = lpt_partition(w, G)
+        got = {}
+        for r in range(G):
+            mine = np.nonzero(owner == r)[0]
+            B = MatrixBatch(cfg.m[mine], cfg.n[mine])
+            host = np.zeros(B.total)
+            irrgen.fill_packed(cfg.seed, cfg.m[mine], cfg.n[mine], B.ld_h, B.offsets, host, gids=mine)
+            B.data.copy_(torch.from_numpy(host))
+            B.getrf()
+            words = torch.zeros(2 * B.batch, dtype=torch.int32, device="cuda")
+            irr.irr_status_words(B.batch, B.m, B.n, B.ipiv, B.info, words)
+            torch.cuda.synchronize()
+            out, ip = B.data.cpu().numpy(), B.ipiv_data.cpu().numpy()
+            wd = words.cpu().numpy().reshape(-1, 2)
+            for q, g in enumerate(mine):
+                got[int(g)] = (np.array(B.matrix(q, out)).tobytes(), np.array(B.ipiv_of(q, ip)).tobytes(),
+                               tuple(wd[q]))
+        if ref is None:
+            ref = got
+        else:
+            assert got == ref, f"G = {G} differs from G = 1"

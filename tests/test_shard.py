@@ -42,41 +42,81 @@ def _free_port():
     return p
 
 
+def _status_words(cfg, gids):
+    """(info, FNV-1a of ipiv) per matrix -- the record irr_status_words
+    writes on the GPU (include/irr.h; GPU test_status_words pins the GPU words
+    to this host definition) -- here from the oracle's factorization."""
+    import oracle
+    from gpu_util import fnv1a_ipiv
+    out = np.zeros((len(gids), 2), dtype=np.int64)
+    for q, g in enumerate(gids):
+        A = irrgen.uniform_values(cfg.seed, int(g), int(cfg.m[g]), int(cfg.n[g]))
+        _, ip, info, _ = oracle.getrf(A)
+        out[q] = (info, fnv1a_ipiv(ip))
+    return out
+
+
 def _worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    cfg = irrgen.config("C2", scale=0.2 * world)
+    cfg = irrgen.config("C2", scale=0.02)          # the same 200 matrices at every world size (strong)
     w = F.getrf_flops(cfg.m, cfg.n)
     owner = lpt_partition(w, world)
     mine = np.nonzero(owner == rank)[0]
     pad = int(np.bincount(owner, minlength=world).max())
-    # per-matrix status word of this rank (here a deterministic stand-in: the global id)
-    status = torch.full((pad,), -7, dtype=torch.int64)
-    status[: len(mine)] = torch.from_numpy(mine)
-    gathered = torch.zeros(world * pad, dtype=torch.int64)
+    # this rank's real status words (info, ipiv hash) of its own matrices, padded
+    status = torch.full((pad, 2), -7, dtype=torch.int64)
+    status[: len(mine)] = torch.from_numpy(_status_words(cfg, mine))
+    gathered = torch.zeros(world * pad, 2, dtype=torch.int64)
     dist.all_gather_into_tensor(gathered, status)
     t = torch.tensor([float(rank + 1)], dtype=torch.float64)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)       # max-over-ranks timing reduction
     if rank == 0:
         shards = [np.nonzero(owner == r)[0] for r in range(world)]
-        merged = merge_status(gathered.view(world, pad).numpy(), shards)
+        g = gathered.view(world, pad, 2).numpy()
+        merged = np.stack([merge_status(g[:, :, f], shards) for f in range(2)], axis=1)
         q.put((merged.tolist(), float(t.item()), len(w)))
     dist.destroy_process_group()
 
 
 def test_gloo_two_ranks_gather_and_merge():
+    """world_size 2 over gloo: every matrix's status word lands at its global
+    id after the gather, and the gathered words equal the single-process
+    (G = 1) words bitwise (results independent of G)."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
     procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
     for p in procs:
         p.start()
-    merged, tmax, total = q.get(timeout=120)
+    merged, tmax, total = q.get(timeout=300)
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    assert merged == list(range(total))           # every matrix's word lands at its global id
+    cfg = irrgen.config("C2", scale=0.02)
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    single = _status_words(cfg, np.arange(total))
+    assert np.array_equal(np.array(merged), single)
     assert tmax == 2.0
+
+
+def test_lpt_c_abi_equals_reference():
+    """irr_shard_lpt_work (C ABI, host) == the Python LPT greedy, and
+    irr_shard_lpt (flops from m, n) == irr_shard_lpt_work on FLOPS_DGETRF."""
+    from paper_conf_sc_abdelfattahgbtld22_b200 import irr
+    from paper_conf_sc_abdelfattahgbtld22_b200.shard import lpt_partition_reference
+    cfg = irrgen.config("C5", scale=0.05)
+    w = F.getrf_flops(cfg.m, cfg.n)
+    for parts in (2, 3, 8):
+        assert np.array_equal(lpt_partition(w, parts), lpt_partition_reference(w, parts))
+        m32 = np.ascontiguousarray(cfg.m, dtype=np.int32)
+        n32 = np.ascontiguousarray(cfg.n, dtype=np.int32)
+        owner = np.zeros(len(w), dtype=np.int32)
+        assert irr.load().irr_shard_lpt(len(w), m32.ctypes.data, n32.ctypes.data, parts, owner.ctypes.data) == 0
+        assert np.array_equal(owner, lpt_partition(w, parts))
 
 
 def test_sibling_rounds_and_level_shard():
