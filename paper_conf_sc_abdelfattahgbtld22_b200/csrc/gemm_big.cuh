@@ -137,30 +137,55 @@ __device__ __forceinline__ void xgemm_epilogue(const GemmDesc &d, int r0, int c0
     const int g = lane >> 2, t = lane & 3;
     const int wm = (warp & 1) * 64, wn = (warp >> 1) * 32;
     const bool rd = d.beta != 0.0;
+    // two 8-row groups per round: 16 loads of C in flight before the stores
+    // (the compiler cannot move later loads above the stores: same array)
 #pragma unroll
-    for (int mi = 0; mi < 8; ++mi) {
-        const int r = r0 + wm + 8 * mi + g;
-        if (r >= d.m) continue;
-        double cv[8];
+    for (int m2 = 0; m2 < 8; m2 += 2) {
+        double cv[2][8];
         if (rd) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int r = r0 + wm + 8 * (m2 + h) + g;
+#pragma unroll
+                for (int ni = 0; ni < 4; ++ni)
+#pragma unroll
+                    for (int i = 0; i < 2; ++i) {
+                        const int c = c0 + wn + 8 * ni + 2 * t + i;
+                        cv[h][ni * 2 + i] = (r < d.m && c < d.n) ? d.C[r + (size_t)c * d.ldc] : 0.0;
+                    }
+            }
+        }
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int mi = m2 + h;
+            const int r = r0 + wm + 8 * mi + g;
+            if (r >= d.m) continue;
 #pragma unroll
             for (int ni = 0; ni < 4; ++ni)
 #pragma unroll
                 for (int i = 0; i < 2; ++i) {
                     const int c = c0 + wn + 8 * ni + 2 * t + i;
-                    cv[ni * 2 + i] = c < d.n ? d.C[r + (size_t)c * d.ldc] : 0.0;
+                    if (c >= d.n) continue;
+                    double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
+                    if (rd) v = fma(d.beta, cv[h][ni * 2 + i], v);
+                    d.C[r + (size_t)c * d.ldc] = v;
                 }
         }
+    }
+}
+
+// C tile -> L2 at the start of the tile (one 128-byte line = 16 rows of a
+// column per prefetch, 4 per thread), so the epilogue's loads hit L2 instead
+// of HBM; the DMMA pipe idles during the epilogue of this 1-CTA/SM core.
+__device__ __forceinline__ void xgemm_prefetch_c(const GemmDesc &d, int r0, int c0) {
+    if (d.beta == 0.0) return;
+    const int tid = threadIdx.x;
+    const int c = c0 + (tid & 127);
+    if (c >= d.n) return;
 #pragma unroll
-        for (int ni = 0; ni < 4; ++ni)
-#pragma unroll
-            for (int i = 0; i < 2; ++i) {
-                const int c = c0 + wn + 8 * ni + 2 * t + i;
-                if (c >= d.n) continue;
-                double v = d.alpha * acc[(mi * 4 + ni) * 2 + i];
-                if (rd) v = fma(d.beta, cv[ni * 2 + i], v);
-                d.C[r + (size_t)c * d.ldc] = v;
-            }
+    for (int q = 0; q < 4; ++q) {
+        const int r = r0 + (tid >> 7) * 64 + 16 * q;
+        if (r < d.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(d.C + r + (size_t)c * d.ldc));
     }
 }
 
@@ -171,6 +196,7 @@ __device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, Bi
 #pragma unroll
     for (int q = 0; q < 64; ++q) acc[q] = 0.0;
     const int nk = (d.k + XBK - 1) / XBK;
+    xgemm_prefetch_c(d, r0, c0);
 #pragma unroll
     for (int s = 0; s < XST - 1; ++s) {
         if (s < nk) xgemm_issue<TA, TB>(d, r0, c0, s * XBK, sm, s);

@@ -671,14 +671,15 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
 // The deferred left-block interchanges of the grid-wide tier: one CTA per
 // tier-L matrix (dynamic queue), after the last panel (left_swaps_core).
 constexpr int LSW_NT = 256;
-constexpr int LSW_BUF = 6144;  // doubles of column buffer (48 KB)
+constexpr int LSW_BUF = 6144;  // doubles of column buffer (48 KB), at least one full column (max_m)
+static int lsw_buf_doubles(int max_m) { return max_m > LSW_BUF ? ((max_m + 1) & ~1) : LSW_BUF; }
 __global__ void __launch_bounds__(LSW_NT) left_swaps_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                             const int *__restrict__ bins, int nb, int maps,
-                                                            int *queue) {
+                                                            int bufd, int *queue) {
     extern __shared__ __align__(16) double lsw_smem[];
     __shared__ int item_s;
     double *buf = lsw_smem;
-    int *g = reinterpret_cast<int *>(lsw_smem + LSW_BUF);
+    int *g = reinterpret_cast<int *>(lsw_smem + bufd);
     int *h = g + maps;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
@@ -691,7 +692,7 @@ __global__ void __launch_bounds__(LSW_NT) left_swaps_kernel(GetrfArgs a, const i
         const int i = list[t];
         const int mi = a.m[i], ni = a.n[i];
         const int K = mi < ni ? mi : ni;
-        if (K > nb) left_swaps_core<LSW_NT>(a.A[i], a.ld[i], mi, K, nb, a.ipiv[i], g, h, buf, LSW_BUF);
+        if (K > nb) left_swaps_core<LSW_NT>(a.A[i], a.ld[i], mi, K, nb, a.ipiv[i], g, h, buf, bufd);
     }
 }
 
@@ -744,111 +745,118 @@ __global__ void __launch_bounds__(OP_NT) outer_plan_kernel(GetrfArgs a, const in
     }
 }
 
-// Right of outer block [J, J + ibo): per (tier-L slot, OS_COLS-column strip):
-//   1. the block's interchanges composed (outer_plan_kernel): the ibo rows that
-//      end in [J, J + ibo) are gathered into shared memory (cp.async; each
-//      column's top rows are one contiguous 1 KB range), the <= ibo rows pushed
-//      below the block are read into registers and, after every read of the
-//      strip, written to their new rows;
-//   2. U12 <- L11^-1 U12 in 32-row blocks d: the diagonal block by a warp-wide
+// Right of outer block [J, J + ibo): per (tier-L matrix, OS_COLS-column
+// strip), over a DENSE item space (per-matrix strip counts prefix-summed on
+// the device; each persistent CTA walks a contiguous range, so consecutive
+// strips of one matrix share the CTA and its L11):
+//   0. on a new matrix: the unit-lower L11 (ibo x ibo) staged in shared memory
+//      once, and the block's composed interchange plan (outer_plan_kernel);
+//   1. one thread per moved row: the ibo rows that end in [J, J + ibo) are
+//      gathered into shared memory (cp.async), the <= ibo rows pushed below
+//      the block are read into registers and -- after every read of the
+//      strip -- written to their new rows;
+//   2. U12 <- L11^-1 U12 in 32-row blocks: the diagonal block by a warp-wide
 //      substitution (lane = row, 8 columns per warp, the solved entry
 //      broadcast by shuffle), the rows below it by a rank-32 DMMA update
-//      (m8n8k4, operands in shared memory: the L column block staged once per
-//      d, U12 rows in place);
-//   3. U12 back to rows [J, J + ibo) (coalesced).
-// Dynamic item queue (reset by outer_plan_kernel).
-constexpr int OS_COLS = 64, OS_NT = 256, OS_TLD = OS_COLS + 1, OS_LDC = 136;
-constexpr int OS_BOTQ = NB_OUTER_MAX / (OS_NT / 32);  // bot rows per warp (registers)
-constexpr size_t OS_SMEM = (size_t)(NB_OUTER_MAX * OS_TLD + 32 * OS_LDC) * sizeof(double);
-__global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
+//      (m8n8k4, both operands in shared memory);
+//   3. U12 back to rows [J, J + ibo), one thread per row (coalesced).
+constexpr int OS_COLS = 64, OS_NT = 256, OS_TLD = OS_COLS + 1, OS_LDL = 136;
+constexpr size_t OS_SMEM = (size_t)(NB_OUTER_MAX * OS_TLD + NB_OUTER_MAX * OS_LDL) * sizeof(double);
+
+struct OuterStrips {
+    GetrfArgs a;
+    const int *list;
+    int J, NBo;
+    __device__ int units(int slot) const {
+        const int i = list[slot];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        if (J >= K) return 0;
+        const int c1 = J + imin(NBo, K - J);
+        return c1 < ni ? (ni - c1 + OS_COLS - 1) / OS_COLS : 0;
+    }
+};
+
+__global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                                    const int *__restrict__ bins,
-                                                                   const OuterPlan *__restrict__ plans, int *queue,
-                                                                   int J, int NBo, int chunks_per) {
+                                                                   const OuterPlan *__restrict__ plans,
+                                                                   const int *__restrict__ off, int J, int NBo) {
     extern __shared__ __align__(16) double os_smem[];
     double *top = os_smem;                       // U12 rows: top[t * OS_TLD + c]
-    double *Lc = top + NB_OUTER_MAX * OS_TLD;    // L column block: Lc[s * OS_LDC + r]
+    double *Ls = top + NB_OUTER_MAX * OS_TLD;    // L11: Ls[s * OS_LDL + r] (column s, row r)
     __shared__ OuterPlan sp;
-    __shared__ int item_s;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int g = lane >> 2, t4 = lane & 3;
     constexpr int NWS = OS_NT / 32;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
-    const long long total = (long long)count * chunks_per;
     int last_slot = -1;
-    for (;;) {
-        if (tid == 0) item_s = atomicAdd(queue, 1);
-        __syncthreads();
-        const long long w = item_s;
-        __syncthreads();
-        if (w >= total) break;
-        const int slot = (int)(w / chunks_per), q = (int)(w - (long long)slot * chunks_per);
+    auto strip = [&](int slot, int q) {
         const int i = list[slot];
         const int mi = a.m[i], ni = a.n[i];
         const int K = mi < ni ? mi : ni;
-        if (J >= K) continue;
         const int ibo = imin(NBo, K - J), c1 = J + ibo;
         const int cb = c1 + q * OS_COLS;
-        if (cb >= ni) continue;
         const int W = imin(OS_COLS, ni - cb);
         const long ld = a.ld[i];
         double *gA = a.A[i];
         if (slot != last_slot) {
+            __syncthreads();
             const int *src = reinterpret_cast<const int *>(plans + slot);
             int *dst = reinterpret_cast<int *>(&sp);
             for (int e = tid; e < (int)(sizeof(OuterPlan) / sizeof(int)); e += OS_NT) dst[e] = src[e];
+            // strict lower part of L11, column by column (lanes over rows)
+            for (int sc = warp; sc < ibo - 1; sc += NWS) {
+                const double *gl = gA + J + (size_t)(J + sc) * ld;
+                for (int r = sc + 1 + lane; r < ibo; r += 32) cp_async8(&Ls[sc * OS_LDL + r], gl + r);
+            }
             last_slot = slot;
-            __syncthreads();
         }
+        __syncthreads();
         const int nbot = sp.nbot;
-        // ---- 1. gather (every read of the strip before any write)
-        for (int c = warp; c < W; c += NWS) {
-            const double *gc = gA + (size_t)(cb + c) * ld;
-            for (int r = lane; r < ibo; r += 32) cp_async8(&top[r * OS_TLD + c], gc + sp.top_src[r]);
-        }
-        cp_async_commit();
-        double bv[OS_BOTQ][2];
+        // ---- 1. gather: threads [0, 128) the top rows, [128, 256) the rows pushed down
+        const double *gcb = gA + (size_t)cb * ld;
+        double bv[OS_COLS];
+        if (tid < NB_OUTER_MAX) {
+            if (tid < ibo) {
+                const double *src = gcb + sp.top_src[tid];
+                double *dst = top + tid * OS_TLD;
+#pragma unroll 8
+                for (int c = 0; c < W; ++c) cp_async8(dst + c, src + (size_t)c * ld);
+            }
+        } else {
+            const int b = tid - NB_OUTER_MAX;
+            if (b < nbot) {
+                const double *src = gcb + sp.bot_src[b];
 #pragma unroll
-        for (int u = 0; u < OS_BOTQ; ++u) {
-            const int b = warp + NWS * u;
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int c = lane + 32 * h;
-                bv[u][h] = (b < nbot && c < W) ? gA[sp.bot_src[b] + (size_t)(cb + c) * ld] : 0.0;
+                for (int c = 0; c < OS_COLS; ++c) bv[c] = c < W ? src[(size_t)c * ld] : 0.0;
             }
         }
+        cp_async_commit();
         cp_async_wait<0>();
         __syncthreads();
+        if (tid >= NB_OUTER_MAX) {
+            const int b = tid - NB_OUTER_MAX;
+            if (b < nbot) {
+                double *dst = gA + (size_t)cb * ld + sp.bot_pos[b];
 #pragma unroll
-        for (int u = 0; u < OS_BOTQ; ++u) {
-            const int b = warp + NWS * u;
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int c = lane + 32 * h;
-                if (b < nbot && c < W) gA[sp.bot_pos[b] + (size_t)(cb + c) * ld] = bv[u][h];
+                for (int c = 0; c < OS_COLS; ++c)
+                    if (c < W) dst[(size_t)c * ld] = bv[c];
             }
         }
         // ---- 2. U12 <- L11^-1 U12, 32-row blocks
         for (int d0 = 0; d0 < ibo; d0 += 32) {
             const int bw = imin(32, ibo - d0);
-            const int below = ibo - d0 - bw;   // rows under the diagonal block
-            for (int sc = warp; sc < bw; sc += NWS) {
-                const double *gl = gA + J + d0 + (size_t)(J + d0 + sc) * ld;
-                for (int r = lane; r < ibo - d0; r += 32) cp_async8(&Lc[sc * OS_LDC + r], gl + r);
-            }
-            cp_async_commit();
-            cp_async_wait<0>();
-            __syncthreads();
-            // diagonal block: warp w solves columns [8w, 8w + 8), lane = row
-            {
+            const int below = ibo - d0 - bw;
+            {   // diagonal block: warp w solves columns [8w, 8w + 8), lane = row
                 const int c0 = warp * 8;
                 double x[8];
 #pragma unroll
                 for (int c = 0; c < 8; ++c) x[c] = (lane < bw && c0 + c < W) ? top[(d0 + lane) * OS_TLD + c0 + c] : 0.0;
-                for (int s = 0; s < bw - 1; ++s) {
-                    const double l = (lane > s && lane < bw) ? Lc[s * OS_LDC + lane] : 0.0;
+                for (int sc = 0; sc < bw - 1; ++sc) {
+                    const double l = (lane > sc && lane < bw) ? Ls[(d0 + sc) * OS_LDL + d0 + lane] : 0.0;
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) x[c] = fma(-l, __shfl_sync(FULL, x[c], s), x[c]);
+                    for (int c = 0; c < 8; ++c) x[c] = fma(-l, __shfl_sync(FULL, x[c], sc), x[c]);
                 }
                 if (lane < bw)
 #pragma unroll
@@ -856,8 +864,7 @@ __global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, 
                         if (c0 + c < W) top[(d0 + lane) * OS_TLD + c0 + c] = x[c];
             }
             __syncthreads();
-            // rows below: C[r][c] -= sum_s Lc[s][bw + r] * X[s][c], 32 x 32 output tiles per warp (DMMA)
-            if (below > 0) {
+            if (below > 0) {   // rows below: 32 x 32 output tiles per warp (DMMA)
                 const int tiles_m = (below + 31) / 32, tiles = tiles_m * 2;
                 for (int tt = warp; tt < tiles; tt += NWS) {
                     const int rb = (tt % tiles_m) * 32, cbt = (tt / tiles_m) * 32;
@@ -868,22 +875,22 @@ __global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, 
                         for (int n8 = 0; n8 < 4; ++n8) { acc[mi][n8][0] = 0.0; acc[mi][n8][1] = 0.0; }
 #pragma unroll
                     for (int ks = 0; ks < 32; ks += 4) {
-                        const int s = ks + t4;
-                        double av[4], bvv[4];
+                        const int sc = ks + t4;
+                        double av[4], bb[4];
 #pragma unroll
                         for (int mi = 0; mi < 4; ++mi) {
-                            const int r = rb + 8 * mi + g;   // row under the block
-                            av[mi] = (s < bw && r < below) ? Lc[s * OS_LDC + bw + r] : 0.0;
+                            const int r = rb + 8 * mi + g;   // row under the diagonal block
+                            av[mi] = (sc < bw && r < below) ? Ls[(d0 + sc) * OS_LDL + d0 + bw + r] : 0.0;
                         }
 #pragma unroll
                         for (int n8 = 0; n8 < 4; ++n8) {
                             const int c = cbt + 8 * n8 + g;
-                            bvv[n8] = (s < bw && c < W) ? top[(d0 + s) * OS_TLD + c] : 0.0;
+                            bb[n8] = (sc < bw && c < W) ? top[(d0 + sc) * OS_TLD + c] : 0.0;
                         }
 #pragma unroll
                         for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-                            for (int n8 = 0; n8 < 4; ++n8) dmma_8x8x4(acc[mi][n8][0], acc[mi][n8][1], av[mi], bvv[n8]);
+                            for (int n8 = 0; n8 < 4; ++n8) dmma_8x8x4(acc[mi][n8][0], acc[mi][n8][1], av[mi], bb[n8]);
                     }
 #pragma unroll
                     for (int mi = 0; mi < 4; ++mi) {
@@ -901,13 +908,15 @@ __global__ void __launch_bounds__(OS_NT, 2) outer_swap_trsm_kernel(GetrfArgs a, 
             }
             __syncthreads();
         }
-        // ---- 3. U12 back to rows [J, J + ibo)
-        for (int c = warp; c < W; c += NWS) {
-            double *gc = gA + J + (size_t)(cb + c) * ld;
-            for (int r = lane; r < ibo; r += 32) gc[r] = top[r * OS_TLD + c];
+        // ---- 3. U12 back to rows [J, J + ibo), one thread per row
+        if (tid < ibo) {
+            double *dst = gA + J + tid + (size_t)cb * ld;
+            const double *src = top + tid * OS_TLD;
+#pragma unroll 8
+            for (int c = 0; c < W; ++c) dst[(size_t)c * ld] = src[c];
         }
-        __syncthreads();
-    }
+    };
+    walk_units(SlotList{nullptr, nullptr, 0}, count, off, strip);
 }
 
 // A22 -= L21 U12 of outer block [J, J + ibo) for every tier-L matrix (K = ibo)
@@ -1096,7 +1105,8 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         else smem_optin(strip_kernel<false>, st_smem);
     }
     // deferred left-block interchanges (strip path only): one pass at the end
-    const size_t lsw_smem = (size_t)LSW_BUF * sizeof(double) + 2 * (size_t)a.max_m * sizeof(int);
+    const int lsw_bufd = lsw_buf_doubles(a.max_m);
+    const size_t lsw_smem = (size_t)lsw_bufd * sizeof(double) + 2 * (size_t)a.max_m * sizeof(int);
     const int nbo = (tu.nb_outer / nb) * nb;
     // two-level blocking (outer blocks of nbo columns) on the fused path; it
     // always defers the interchanges of the columns left of the outer block
@@ -1110,7 +1120,6 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         smem_optin(outer_swap_trsm_kernel, OS_SMEM);
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0>, BIG_SMEM);
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
-        const int os_chunks = (a.max_n + OS_COLS - 1) / OS_COLS;
         const int *cnt_ptr = counters + CNT_BIN0 + BIN_L;
         for (int J = 0; J < Kmax; J += nbo) {
             for (int j = J; j < Kmax && j < J + nbo; j += nb) {
@@ -1131,9 +1140,13 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                 outer_plan_kernel<<<g, OP_NT, 0, s>>>(a, counters, bins, J, nbo, oplans, counters + CNT_OUTQ);
             }
             {
+                KScope k(K_GEMM_SCAN, s);
+                scan_units_kernel<OuterStrips><<<1, 1024, 0, s>>>(OuterStrips{a, listL, J, nbo},
+                                                                  SlotList{nullptr, cnt_ptr, 0}, a.batch, tile_off);
+            }
+            {
                 KScope k(K_OUTER_TRSM, s);
-                outer_swap_trsm_kernel<<<sms * 2, OS_NT, OS_SMEM, s>>>(a, counters, bins, oplans,
-                                                                     counters + CNT_OUTQ, J, nbo, os_chunks);
+                outer_swap_trsm_kernel<<<sms, OS_NT, OS_SMEM, s>>>(a, counters, bins, oplans, tile_off, J, nbo);
             }
             OuterTrailProb P{a, listL, J, nbo};
             {
@@ -1190,7 +1203,8 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
         KScope k(K_LEFT_SWAPS, s);
         int grid = sms * 2;
         if (grid > a.batch) grid = a.batch;
-        left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, lnb, a.max_m, counters + CNT_LSWQ);
+        left_swaps_kernel<<<grid, LSW_NT, lsw_smem, s>>>(a, counters, bins, lnb, a.max_m, lsw_bufd,
+                                                        counters + CNT_LSWQ);
     }
 }
 

@@ -19,9 +19,16 @@ METRICS = {
     "grid": "launch__grid_size",
     "block": "launch__block_size",
     "smem_dyn": "launch__shared_mem_per_block_dynamic",
-    "dfma_pipe_pct": "sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active",
+    "fp64_pipe_pct": "sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active",
+    "dmma_pipe_pct": "sm__inst_executed_pipe_tensor_subpipe_dmma.avg.pct_of_peak_sustained_active",
+    "tensor_pipe_pct": "TPC.TriageCompute.sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+    "fp64_pipe_realtime_pct": "TPC.TriageCompute.sm__pipe_fp64_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+    "dfma_thread_inst_x2": "derived__sm__sass_thread_inst_executed_op_dfma_pred_on_x2",
+    "inst_executed": "inst_executed",
     "l2_hit": "lts__t_sector_hit_rate.pct",
 }
+_TIME = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3, "ms": 1e3, "second": 1e6, "s": 1e6}
+_BYTES = {"byte": 1, "B": 1, "Kbyte": 1e3, "KB": 1e3, "Mbyte": 1e6, "MB": 1e6, "Gbyte": 1e9, "GB": 1e9}
 
 
 def load(path):
@@ -40,11 +47,10 @@ def load(path):
             except ValueError:
                 continue
             unit = u.get(m, "")
-            if k == "dur_us":
-                x = x / 1000.0 if unit == "nsecond" else (x * 1000.0 if unit == "msecond" else x)
+            if k == "dur_us":        # always microseconds, whatever unit ncu printed
+                x = x * _TIME.get(unit, 1.0)
             if k.startswith("dram_"):
-                scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
-                x = x * scale
+                x = x * _BYTES.get(unit, 1)
             rec[k] = x
         st = [(k.replace("smsp__pcsamp_warps_issue_stalled_", ""), float(v.replace(",", "")))
               for k, v in d.items()
