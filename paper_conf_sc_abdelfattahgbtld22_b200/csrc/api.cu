@@ -38,8 +38,9 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // 100.4; 0 = no tier M is 6.00 on C2 but slower on C5), S/M concurrent with L1, DMMA for the
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
-// left-block interchanges (6.80 -> 6.53 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, 0};
+// left-block interchanges (6.80 -> 6.53 ms), two-level grid tier with outer
+// blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower).
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, NB_OUTER_MAX};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 

@@ -45,28 +45,37 @@ struct SmallCfg<16> { static constexpr int ctas = 6, bin = BIN_S16; };  // 80 re
 template <>
 struct SmallCfg<8> { static constexpr int ctas = 8, bin = BIN_S8; };    // 64 regs, 32 warps / SM
 
-// offset of packed U row k; row k's capacity is NC - (k & ~1) (even, so every
-// row starts 16-byte aligned for the pair stores)
+// U rows are packed in step order, row k taking exactly its step width W(k)
+// (the class of n - k: 32 / 24 / 16 / 12 / 8 / 4), so a step publishes and
+// reads its full W-wide pair stores / loads without predicates and no step
+// touches another row's slots.  Capacity = the widths summed at n = NC.
 template <int NC>
-__host__ __device__ constexpr int s_uoff(int k) {
-    return (k & 1) ? 2 * (k >> 1) * (NC + 1 - (k >> 1)) + NC - 2 * (k >> 1)
-                   : 2 * (k >> 1) * (NC + 1 - (k >> 1));
+__host__ __device__ constexpr int s_width(int rem) {
+    return (NC >= 32 && rem > 24) ? 32 : (NC >= 32 && rem > 16) ? 24 : (NC >= 16 && rem > 12) ? 16
+         : (NC >= 16 && rem > 8) ? 12 : (rem > 4) ? (NC >= 8 ? 8 : NC) : 4;
+}
+template <int NC>
+__host__ __device__ constexpr int s_ucap() {
+    int t = 0;
+    for (int k = 0; k < NC; ++k) t += s_width<NC>(NC - k);
+    return t;
 }
 
 template <int NC>
 struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 stores in every warp's slot
     double L[NC * 32];             // L[k*32 + lane]: multiplier of the row held by `lane` at step k
-    double U[s_uoff<NC>(NC) + NC];  // row k of U (n-k values) at s_uoff(k), + overflow pad
+    double U[s_ucap<NC>()];        // row k of U at urow[k], W(k) slots
     double rcp[2];                 // reciprocal of the pivot of step k in rcp[k & 1] (0: divide)
+    int urow[NC];                  // offset of U row k
 };
 static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<16>) % 16 == 0 &&
                   sizeof(SmallWarpSmem<8>) % 16 == 0,
               "per-warp slots must stay 16-byte aligned");
-static_assert(s_uoff<32>(32) == 544 && s_uoff<32>(3) == 94, "packed U offsets");
+static_assert(s_ucap<32>() == 608 && s_ucap<16>() == 160 && s_ucap<8>() == 48, "packed U capacity");
 
 template <int NC, int W>
 __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, bool valid,
-                                       int lane, int n, SmallWarpSmem<NC> &sm) {
+                                       int lane, int &uo, SmallWarpSmem<NC> &sm) {
     const bool cand = valid && pos >= k;
     // every lane's reciprocal of its own candidate, off the critical path of
     // the pivot search; the winner publishes its one
@@ -86,17 +95,14 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
     const int w = __ffs(wm) - 1;
     const int pmin = __shfl_sync(FULL, pos, w);
     // ---- the pivot row is row k of U: publish it where the output reads it
-    // Row k holds n - k values within its capacity NC - (k & ~1): the pairs
-    // c < n - k are stored (the odd tail's partner slot is still inside the
-    // row), so no step writes into another row's region.
-    double *urow = sm.U + s_uoff<NC>(k);
-    const int rem = n - k;
+    double *urow = sm.U + uo;
     if (lane == w) {
 #pragma unroll
-        for (int c = 0; c < W; c += 2)
-            if (c < rem) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
+        for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
         sm.rcp[k & 1] = myr;
     }
+    if (lane == 0) sm.urow[k] = uo;
+    uo += W;
     if (lane == k) my_piv = pmin + 1;
     __syncwarp();
     const double pv = urow[0];
@@ -120,10 +126,7 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
         double uu[CH];
 #pragma unroll
         for (int q = 0; q < CH; q += 2) {
-            // only this row's own slots are read (the pairs past n - k are
-            // padding columns >= n: zeros, never part of the output)
-            const double2 v = (e0 + q < rem) ? *reinterpret_cast<const double2 *>(urow + e0 + q)
-                                             : make_double2(0.0, 0.0);
+            const double2 v = *reinterpret_cast<const double2 *>(urow + e0 + q);
             uu[q] = v.x;
             uu[q + 1] = v.y;
         }
@@ -132,8 +135,8 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
             if (e0 + q >= 1) a[e0 + q - 1] = fma(-l, uu[q], a[e0 + q]);
     }
     a[W - 1] = 0.0;
-    // no trailing warp barrier: the next step writes row k+1 (past row k's
-    // capacity) and rcp[(k+1) & 1], neither of which this step reads
+    // no trailing warp barrier: the next step writes row k+1 (its own W
+    // slots after row k's) and rcp[(k+1) & 1], neither of which this step reads
     ++k;
 }
 
@@ -148,26 +151,26 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
         a[c] = (valid && c < n) ? *gr : 0.0;
         gr += ld;
     }
-    int pos = lane, my_piv = 0, info = 0, k = 0;
+    int pos = lane, my_piv = 0, info = 0, k = 0, uo = 0;
     const int K = m < n ? m : n;
     // active width W >= n - k in steps of 32 / 24 / 16 / 12 / 8 / 4 (the
     // FMAs, pivot-row loads and publish stores of a step scale with W)
     if (NC >= 32) {
-        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
-        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
+        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
     }
     if (NC >= 16) {
-        while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
-        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
+        while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+        while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
     }
-    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, n, sm);
-    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, n, sm);
+    while (k < K && n - k > 4) s_step<NC, (NC >= 8 ? 8 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+    while (k < K) s_step<NC, 4>(a, k, pos, my_piv, info, valid, lane, uo, sm);
     __syncwarp();  // L / U rows from every lane are complete
     // ---- write every row once, at its final position p: L(p, c) for c < p,
     //      U(p, c) for c >= p (rows p >= K are pure L rows)
     if (valid) {
         double *go = gA + pos;
-        const double *ur = sm.U + s_uoff<NC>(pos < K ? pos : 0) - pos;
+        const double *ur = sm.U + sm.urow[pos < K ? pos : 0] - pos;
         for (int c = 0; c < n; ++c) {
             double v;
             if (c < pos) v = sm.L[c * 32 + lane];

@@ -69,11 +69,13 @@ def test_tier_m_boundary_and_extreme_shapes(tier_m_max):
     _run_and_check(_uniform(shapes, seed=5))
 
 
-@pytest.mark.parametrize("l1", [1, 0])
+@pytest.mark.parametrize("l1,nbo", [(1, 128), (0, 0), (0, 128)])
 @pytest.mark.parametrize("nb", [5, 8, 16, 32, 64])
-def test_tier_l_forced_small_nb(nb, l1):
+def test_tier_l_forced_small_nb(nb, l1, nbo):
     """Force everything through tier L (l1=1: CTA-per-matrix for m <= 256,
-    l1=0: grid-wide kernel chain): nb-1, nb, nb+1, 2nb+-1 sizes."""
+    l1=0: grid-wide kernel chain, one level (nbo 0) or two-level blocking):
+    nb-1, nb, nb+1, 2nb+-1 sizes."""
+    irr.irr_set_tuning("nb_outer", nbo)
     irr.irr_set_tuning("tier_s", 0)
     irr.irr_set_tuning("tier_m_max", 0)
     irr.irr_set_tuning("nb", nb)
@@ -215,6 +217,7 @@ def test_windowed_panel_grid_tier(nb):
     tall, wide and square, window boundaries inside and at the panel edge."""
     irr.irr_set_tuning("l1", 0)
     irr.irr_set_tuning("nb", nb)
+    irr.irr_set_tuning("nb_outer", 0)      # the one-level chain (two-level: test_two_level_grid_tier)
     shapes = [(700, 90), (1024, 64), (1025, 40), (1500, 33), (2048, 70), (2100, 40), (513, 513),
               (90, 700), (600, 600), (300, 17), (257, 257)]
     _run_and_check(_uniform(shapes, seed=31 + nb))
@@ -270,6 +273,7 @@ def test_deferred_left_interchanges(defer, l1):
     tier (l1=0): both match the oracle and agree bitwise (interchanges only
     move values)."""
     irr.irr_set_tuning("l1", l1)
+    irr.irr_set_tuning("nb_outer", 0)      # eager vs deferred exists on the one-level chain
     irr.irr_set_tuning("defer", defer)
     shapes = [(256, 256), (200, 240), (256, 70), (180, 256), (129, 200), (250, 33)]
     if not l1:
