@@ -465,15 +465,18 @@ def main():
         roof = {"bound": "hbm", "achieved": ach, "peak": hbm, "unit": "GB/s", "frac": ach / hbm}
     else:
         ach = fl / (dms_step * 1e-3) / 1e12
-        roof = {"bound": "alu", "achieved": ach, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
-                "frac": ach / FP64_PEAK_TFLOPS}
+        # classes whose flops run on the FP64 tensor core (mma.sync DMMA) vs the DFMA pipe
+        dmma = {"gemm_trailing", "strip", "lu_l1", "gemm_dcwi", "getrs", "outer_trsm"}
+        roof = {"bound": "tensor" if dname in dmma else "alu", "achieved": ach, "peak": FP64_PEAK_TFLOPS,
+                "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS}
     roof["kernel"] = dname
     roof["share_of_step"] = dms_step / (total_ms / args.steps)
     roof["launches_per_step"] = dcnt / args.steps
     roof["peak_source"] = ("measured: MEASURED_PEAKS.json hbm_gbs" if hbm_src == "measured" else
                            "fallback 6,650 GB/s (B200_PROFILING.md; MEASURED_PEAKS.json absent)") \
         if roof["bound"] == "hbm" else \
-        "derived: 148 SM x 64 DFMA/clk x 2 flop x 1.965 GHz"
+        ("measured FP64 tensor (DMMA m8n8k4) and DFMA rate 64 FMA/clk/SM (tools/microbench.cu, "
+         "profiles/r01/microbench.txt) x 148 SM x 2 flop x 1.965 GHz = the FP64 nominal peak")
     roof["traffic"] = _ncu_traffic(args.config, dname, dcnt / args.steps)
     whole = {"flops": flops_local, "bytes": bytes_local,
              "fp64_frac": flops_local / (ms_per_step * 1e-3) / (FP64_PEAK_TFLOPS * 1e12),

@@ -40,7 +40,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
 // left-block interchanges (6.80 -> 6.53 ms), two-level grid tier with outer
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, NB_OUTER_MAX};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, NB_OUTER_MAX, 8};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -331,6 +331,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
     else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
     else if (!strcmp(key, "nb_outer")) g_tuning.nb_outer = value < 0 ? 0 : (value > NB_OUTER_MAX ? NB_OUTER_MAX : value);
+    else if (!strcmp(key, "xgemm_warps")) g_tuning.xgemm_warps = value >= 16 ? 16 : 8;
 }
 
 int irr_get_tuning(const char *key) {
@@ -354,6 +355,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "l1_rows")) return g_tuning.l1_rows;
     if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) return g_tuning.defer;
     if (!strcmp(key, "nb_outer")) return g_tuning.nb_outer;
+    if (!strcmp(key, "xgemm_warps")) return g_tuning.xgemm_warps;
     return -1;
 }
 

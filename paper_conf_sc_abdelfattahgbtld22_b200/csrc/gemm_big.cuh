@@ -63,14 +63,14 @@ __device__ __forceinline__ void x_pair(double *dst, const double *src, bool ok0,
 // Element pairs along each operand's contiguous dimension (m for A, k for
 // A^T, k for B, n for B^T): both shared layouts keep such pairs 16-byte
 // aligned (even leading dimensions 132 / 20).
-template <int TA, int TB>
+template <int TA, int TB, int NT = X_NT>
 __device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st) {
     const int tid = threadIdx.x;
     double *As = sm.A[st];
     double *Bs = sm.B[st];
 #pragma unroll
-    for (int q = 0; q < (XBM * XBK) / (2 * X_NT); ++q) {
-        const int e = tid + X_NT * q;
+    for (int q = 0; q < (XBM * XBK) / (2 * NT); ++q) {
+        const int e = tid + NT * q;
         if (!TA) {  // A(m, k) at A + m + k lda: pairs along m
             const int m = 2 * (e & (XBM / 2 - 1)), kk = e / (XBM / 2);
             const int gm = r0 + m, gk = k0 + kk;
@@ -86,8 +86,8 @@ __device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, i
         }
     }
 #pragma unroll
-    for (int q = 0; q < (XBN * XBK) / (2 * X_NT); ++q) {
-        const int e = tid + X_NT * q;
+    for (int q = 0; q < (XBN * XBK) / (2 * NT); ++q) {
+        const int e = tid + NT * q;
         if (!TB) {  // B(k, n) at B + k + n ldb: pairs along k
             const int kk = 2 * (e & (XBK / 2 - 1)), n = e / (XBK / 2);
             const int gn = c0 + n, gk = k0 + kk;
@@ -104,18 +104,29 @@ __device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, i
     }
 }
 
-template <int TA, int TB>
-__device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double (&acc)[64]) {
+// NWG warps: 8 -> a 2 x 4 warp grid of 64 x 32 warp tiles (MI = 8 mma rows),
+// 16 -> 4 x 4 warps of 32 x 32 (MI = 4): more warps to hide the DMMA /
+// fragment-load latencies at half the accumulators per thread.
+template <int NWG>
+struct XWarp {
+    static constexpr int MI = NWG == 16 ? 4 : 8;
+    static constexpr int WGM = NWG == 16 ? 4 : 2;   // warps along m
+    static constexpr int ACC = MI * 4 * 2;
+};
+
+template <int TA, int TB, int NWG = 8>
+__device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double (&acc)[XWarp<NWG>::ACC]) {
+    constexpr int MI = XWarp<NWG>::MI, WGM = XWarp<NWG>::WGM;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int g = lane >> 2, t = lane & 3;
-    const int wm = (warp & 1) * 64, wn = (warp >> 1) * 32;
+    const int wm = (warp % WGM) * (8 * MI), wn = (warp / WGM) * 32;
     const double *As = sm.A[st];
     const double *Bs = sm.B[st];
 #pragma unroll
     for (int ks = 0; ks < XBK; ks += 4) {
-        double a[8], b[4];
+        double a[MI], b[4];
 #pragma unroll
-        for (int mi = 0; mi < 8; ++mi) {
+        for (int mi = 0; mi < MI; ++mi) {
             const int m = wm + 8 * mi + g, k = ks + t;
             a[mi] = TA ? As[m * XLD_MK + k] : As[k * XLD_KM + m];
         }
@@ -125,22 +136,25 @@ __device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double 
             b[ni] = TB ? Bs[k * XLD_KM + n] : Bs[n * XLD_MK + k];
         }
 #pragma unroll
-        for (int mi = 0; mi < 8; ++mi)
+        for (int mi = 0; mi < MI; ++mi)
 #pragma unroll
             for (int ni = 0; ni < 4; ++ni)
                 dmma_8x8x4(acc[(mi * 4 + ni) * 2], acc[(mi * 4 + ni) * 2 + 1], a[mi], b[ni]);
     }
 }
 
-__device__ __forceinline__ void xgemm_epilogue(const GemmDesc &d, int r0, int c0, const double (&acc)[64]) {
+template <int NWG = 8>
+__device__ __forceinline__ void xgemm_epilogue(const GemmDesc &d, int r0, int c0,
+                                               const double (&acc)[XWarp<NWG>::ACC]) {
+    constexpr int MI = XWarp<NWG>::MI, WGM = XWarp<NWG>::WGM;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int g = lane >> 2, t = lane & 3;
-    const int wm = (warp & 1) * 64, wn = (warp >> 1) * 32;
+    const int wm = (warp % WGM) * (8 * MI), wn = (warp / WGM) * 32;
     const bool rd = d.beta != 0.0;
     // two 8-row groups per round: 16 loads of C in flight before the stores
     // (the compiler cannot move later loads above the stores: same array)
 #pragma unroll
-    for (int m2 = 0; m2 < 8; m2 += 2) {
+    for (int m2 = 0; m2 < MI; m2 += 2) {
         double cv[2][8];
         if (rd) {
 #pragma unroll
@@ -177,42 +191,45 @@ __device__ __forceinline__ void xgemm_epilogue(const GemmDesc &d, int r0, int c0
 // C tile -> L2 at the start of the tile (one 128-byte line = 16 rows of a
 // column per prefetch, 4 per thread), so the epilogue's loads hit L2 instead
 // of HBM; the DMMA pipe idles during the epilogue of this 1-CTA/SM core.
+template <int NT = X_NT>
 __device__ __forceinline__ void xgemm_prefetch_c(const GemmDesc &d, int r0, int c0) {
     if (d.beta == 0.0) return;
+    constexpr int GR = XBM / (NT / 128);   // rows per thread group
     const int tid = threadIdx.x;
     const int c = c0 + (tid & 127);
     if (c >= d.n) return;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const int r = r0 + (tid >> 7) * 64 + 16 * q;
+    for (int q = 0; q < GR / 16; ++q) {
+        const int r = r0 + (tid >> 7) * GR + 16 * q;
         if (r < d.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(d.C + r + (size_t)c * d.ldc));
     }
 }
 
 // One tile: the whole K loop through the 4-deep ring, then the epilogue.
-template <int TA, int TB>
+template <int TA, int TB, int NWG = 8>
 __device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, BigSmem &sm) {
-    double acc[64];
+    constexpr int NT = 32 * NWG, ACC = XWarp<NWG>::ACC;
+    double acc[ACC];
 #pragma unroll
-    for (int q = 0; q < 64; ++q) acc[q] = 0.0;
+    for (int q = 0; q < ACC; ++q) acc[q] = 0.0;
     const int nk = (d.k + XBK - 1) / XBK;
-    xgemm_prefetch_c(d, r0, c0);
+    xgemm_prefetch_c<NT>(d, r0, c0);
 #pragma unroll
     for (int s = 0; s < XST - 1; ++s) {
-        if (s < nk) xgemm_issue<TA, TB>(d, r0, c0, s * XBK, sm, s);
+        if (s < nk) xgemm_issue<TA, TB, NT>(d, r0, c0, s * XBK, sm, s);
         cp_async_commit();
     }
     for (int kc = 0; kc < nk; ++kc) {
         cp_async_wait<XST - 2>();
         __syncthreads();
         const int nx = kc + XST - 1;
-        if (nx < nk) xgemm_issue<TA, TB>(d, r0, c0, nx * XBK, sm, nx % XST);
+        if (nx < nk) xgemm_issue<TA, TB, NT>(d, r0, c0, nx * XBK, sm, nx % XST);
         cp_async_commit();
-        xgemm_compute<TA, TB>(sm, kc % XST, acc);
+        xgemm_compute<TA, TB, NWG>(sm, kc % XST, acc);
     }
     cp_async_wait<0>();
     __syncthreads();  // the ring is refilled by the next tile's prologue
-    xgemm_epilogue(d, r0, c0, acc);
+    xgemm_epilogue<NWG>(d, r0, c0, acc);
 }
 
 __device__ __forceinline__ int xgemm_tiles_of(const GemmDesc &d) {
@@ -266,8 +283,8 @@ __global__ void __launch_bounds__(1024) xgemm_scan_kernel(Prob P, int count, con
 }
 
 // Persistent: CTA b owns the tiles whose weighted start lies in its 1/G share.
-template <class Prob, int TA, int TB>
-__global__ void __launch_bounds__(X_NT, XGEMM_MINB) xgemm_sched_kernel(Prob P, int count, const int *count_ptr,
+template <class Prob, int TA, int TB, int NWG = 8>
+__global__ void __launch_bounds__(32 * NWG, XGEMM_MINB) xgemm_sched_kernel(Prob P, int count, const int *count_ptr,
                                                              const int *__restrict__ tile_off) {
     extern __shared__ __align__(16) unsigned char x_smem[];
     BigSmem &sm = *reinterpret_cast<BigSmem *>(x_smem);
@@ -301,7 +318,7 @@ __global__ void __launch_bounds__(X_NT, XGEMM_MINB) xgemm_sched_kernel(Prob P, i
         }
         if (off_b + local * w >= u_end) return;
         const int ntm = (cur.m + XBM - 1) / XBM;
-        xgemm_tile<TA, TB>(cur, (local % ntm) * XBM, (local / ntm) * XBN, sm);
+        xgemm_tile<TA, TB, NWG>(cur, (local % ntm) * XBM, (local / ntm) * XBN, sm);
         ++local;
     }
 }

@@ -34,6 +34,7 @@ struct Tuning {
     int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)
     int getrs_vec;       // 1: irr_getrs with max_nrhs <= 4 by the CTA-per-system kernel (getrs_vec.cu)
     int nb_outer;        // grid-wide tier: outer block width of the two-level blocking (0 / <= nb: one level)
+    int xgemm_warps;     // 8 or 16 warps per 128 x 128 DMMA tile CTA (the two-level trailing GEMM)
 };
 Tuning &tuning();
 

@@ -1118,7 +1118,8 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
     if (outer) {
         OuterPlan *oplans = reinterpret_cast<OuterPlan *>(outer_plans_v);
         smem_optin(outer_swap_trsm_kernel, OS_SMEM);
-        smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0>, BIG_SMEM);
+        smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 8>, BIG_SMEM);
+        smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 16>, BIG_SMEM);
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
         const int *cnt_ptr = counters + CNT_BIN0 + BIN_L;
         for (int J = 0; J < Kmax; J += nbo) {
@@ -1154,7 +1155,12 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                 xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, s>>>(P, -1, cnt_ptr, tile_off);
             }
             KScope k(K_GEMM_TRAIL, s);
-            xgemm_sched_kernel<OuterTrailProb, 0, 0><<<sms * XGEMM_MINB, X_NT, BIG_SMEM, s>>>(P, -1, cnt_ptr, tile_off);
+            if (tu.xgemm_warps == 16)
+                xgemm_sched_kernel<OuterTrailProb, 0, 0, 16><<<sms * XGEMM_MINB, 512, BIG_SMEM, s>>>(P, -1, cnt_ptr,
+                                                                                                 tile_off);
+            else
+                xgemm_sched_kernel<OuterTrailProb, 0, 0, 8><<<sms * XGEMM_MINB, 256, BIG_SMEM, s>>>(P, -1, cnt_ptr,
+                                                                                                tile_off);
         }
     } else
     for (int j = 0; j < Kmax; j += nb) {
