@@ -39,8 +39,10 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // grid-wide GEMMs (22.1 vs 17.5 TFLOP/s) and inside L1 (C2 6.53 -> 6.44 ms once
 // the deferred interchanges took the L1 kernel off its spills), deferred L1
 // left-block interchanges (6.80 -> 6.53 ms), two-level grid tier with outer
-// blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, L1_MAX_ROWS, 1, 1, NB_OUTER_MAX, 8};
+// blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
+// CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
+// rows: C3 61.7), 8-warp xgemm CTAs (16 warps: C3 58.3, C5 651 ms).
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -250,7 +252,7 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
         }
         if (has_large) {
             if (t.l1) launch_lu_l1(a, w.counters, w.bins, w.keys, w.sort, s);
-            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, w.outer_plans, s);
+            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, w.outer_plans, s, w.keys, w.sort);
         }
     }
     if (side != s) {

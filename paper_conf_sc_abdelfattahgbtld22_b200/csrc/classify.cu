@@ -33,7 +33,7 @@ __global__ void __launch_bounds__(256) classify_kernel(GetrfArgs a, int *counter
             else if (el <= M1_ELEMS && el <= tier_m_max) bin = BIN_M1;
             else if (el <= M2_ELEMS && el <= tier_m_max) bin = BIN_M2;
             else if (el <= tier_m_max) bin = BIN_M3;
-            else if (l1 && mi <= l1) bin = BIN_L1;  // l1 = max rows of the CTA-per-matrix tier
+            else if (l1 && mi <= l1) bin = mi <= L1_MAX_ROWS ? BIN_L1 : BIN_L1T;  // l1 = max rows of the CTA-per-matrix tier
             else bin = BIN_L;
         }
     }

@@ -70,7 +70,8 @@ struct KScope {
 // L = blocked right-looking LU with one kernel chain per panel iteration.
 // L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
 // kernels per panel iteration.
-enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, BIN_S16 = 6, BIN_S8 = 7, NBINS = 8 };
+enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, BIN_S16 = 6, BIN_S8 = 7, BIN_L1T = 8,
+           NBINS = 9 };  // L1T: CTA-per-matrix tier, 257..l1_rows rows (tall-panel kernel variant)
 constexpr int L1_MAX_ROWS = 256;    // panels up to this many rows are staged in shared memory
 constexpr int L1_TALL_ROWS = 1024;  // taller L1 panels: panel_win in global memory (128 threads x 8 rows)
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
@@ -83,7 +84,7 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15, CNT_ZQ = 16,
+enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15, CNT_ZQ = 16, CNT_PANELQ = 17,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
@@ -240,7 +241,7 @@ constexpr size_t SWAP_PLAN_BYTES = 1040;  // sizeof(SwapPlan), checked in lu_lar
 constexpr int NB_OUTER_MAX = 128;          // widest outer block of the two-level grid tier
 constexpr size_t OUTER_PLAN_BYTES = 2064;  // sizeof(OuterPlan), checked in lu_large.cu
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, void *outer_plans,
-                     cudaStream_t s);
+                     cudaStream_t s, int *keys = nullptr, int *sort_ws = nullptr);
 void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)

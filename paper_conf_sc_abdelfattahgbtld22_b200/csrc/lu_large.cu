@@ -493,16 +493,24 @@ constexpr int PW_MAX_ROWS = 8192;
 template <int NT>
 __global__ void __launch_bounds__(NT, NT <= 256 ? 2 : 1) panel_win_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                                          const int *__restrict__ bins, int j, int nb,
-                                                                         SwapPlan *__restrict__ plans, int *queue) {
+                                                                         SwapPlan *__restrict__ plans, int *queue,
+                                                                         int *pqueue) {
     extern __shared__ __align__(16) double pw_smem[];
     PanelWinSmem<NT / 32> &sm = *reinterpret_cast<PanelWinSmem<NT / 32> *>(pw_smem);
     __shared__ PanelScratch sc;
     __shared__ int piv_s[NBMAX];
     const int tid = threadIdx.x;
+    __shared__ int item_s;
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
     if (blockIdx.x == 0 && tid == 0) *queue = 0;  // the strip kernel's work queue (stream-ordered)
-    for (int t = blockIdx.x; t < count; t += gridDim.x) {
+    for (;;) {
+        // dynamic queue over the LPT-ordered list (reset by the kernel that follows)
+        if (tid == 0) item_s = atomicAdd(pqueue, 1);
+        __syncthreads();
+        const int t = item_s;
+        __syncthreads();
+        if (t >= count) break;
         const int i = list[t];
         const int mi = a.m[i], ni = a.n[i], ld = a.ld[i];
         const int K = mi < ni ? mi : ni;
@@ -539,14 +547,15 @@ __global__ void __launch_bounds__(NT, NT <= 256 ? 2 : 1) panel_win_kernel(GetrfA
 // the windowed panel for the tallest panel of the launch
 static void launch_panel_win(int max_rows, int grid, const GetrfArgs &a, int *counters, const int *bins, int j,
                              int nb, SwapPlan *plans, int *queue, cudaStream_t s) {
+    int *pq = counters + CNT_PANELQ;
     if (max_rows <= 8 * 256) {
-        panel_win_kernel<256><<<grid, 256, sizeof(PanelWinSmem<8>), s>>>(a, counters, bins, j, nb, plans, queue);
+        panel_win_kernel<256><<<grid, 256, sizeof(PanelWinSmem<8>), s>>>(a, counters, bins, j, nb, plans, queue, pq);
     } else if (max_rows <= 8 * 512) {
         const int g = grid < num_sms() ? grid : num_sms();
-        panel_win_kernel<512><<<g, 512, sizeof(PanelWinSmem<16>), s>>>(a, counters, bins, j, nb, plans, queue);
+        panel_win_kernel<512><<<g, 512, sizeof(PanelWinSmem<16>), s>>>(a, counters, bins, j, nb, plans, queue, pq);
     } else {
         const int g = grid < num_sms() ? grid : num_sms();
-        panel_win_kernel<1024><<<g, 1024, sizeof(PanelWinSmem<32>), s>>>(a, counters, bins, j, nb, plans, queue);
+        panel_win_kernel<1024><<<g, 1024, sizeof(PanelWinSmem<32>), s>>>(a, counters, bins, j, nb, plans, queue, pq);
     }
 }
 
@@ -561,7 +570,7 @@ static void launch_panel_win(int max_rows, int grid, const GetrfArgs &a, int *co
 constexpr int ST_COLS = GBN;
 static_assert(sizeof(SwapPlan) <= SWAP_PLAN_BYTES, "plan slot");
 template <bool DMMA>
-__global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *__restrict__ counters,
+__global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, int *__restrict__ counters,
                                                         const int *__restrict__ bins,
                                                         const SwapPlan *__restrict__ plans, int *queue, int j,
                                                         int nb, int chunks_per, unsigned long long *ph, int defer,
@@ -585,6 +594,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, const int *
     const long long total = (long long)count * chunks_per;
     int last_slot = -1;
     long long t0 = (ph && tid == 0) ? clock64() : 0;
+    if (blockIdx.x == 0 && tid == 0) counters[CNT_PANELQ] = 0;  // the next panel launch's queue (stream-ordered)
 #define ST_PHASE(k)                                                           \
     if (ph && tid == 0) {                                                     \
         long long t1 = clock64();                                             \
@@ -1016,12 +1026,13 @@ static size_t l1_region_bytes(int nb) {
     return (m + 15) & ~size_t(15);
 }
 
-// LPT key of an L1 matrix: 32 + cube root of its m n min(m,n) (>= 32, so the
-// bucketed size sort puts every L1 matrix before the zero keys of the rest)
+// LPT key of a matrix of bin `bin`: 32 + cube root of its m n min(m,n) (>= 32,
+// so the bucketed size sort puts every matrix of the bin before the zero keys
+// of the rest)
 __global__ void l1_key_kernel(GetrfArgs a, const int *__restrict__ counters, const int *__restrict__ bins,
-                              int *__restrict__ key) {
-    const int count = counters[CNT_BIN0 + BIN_L1];
-    const int *list = bins + (size_t)BIN_L1 * a.batch;
+                              int *__restrict__ key, int bin = BIN_L1) {
+    const int count = counters[CNT_BIN0 + bin];
+    const int *list = bins + (size_t)bin * a.batch;
     for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < count; t += gridDim.x * blockDim.x) {
         const int i = list[t];
         const double m = a.m[i], n = a.n[i];
@@ -1030,19 +1041,6 @@ __global__ void l1_key_kernel(GetrfArgs a, const int *__restrict__ counters, con
 }
 
 void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s) {
-    const int *order = nullptr, *order_count = nullptr;
-    if (keys && sort_ws) {
-        cudaMemsetAsync(keys, 0, (size_t)a.batch * sizeof(int), s);
-        {
-            KScope k(K_MISC, s);
-            int g = (a.batch + 255) / 256;
-            l1_key_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(a, counters, bins, keys);
-        }
-        launch_size_sort(keys, a.batch, sort_ws, s);
-        SlotList sl = sorted_slots(sort_ws, a.batch, 31);
-        order = sl.idx;
-        order_count = sl.prefix + sl.bucket0;
-    }
     const int nb = clamp_nb(tuning().nb);
     const size_t region = l1_region_bytes(nb);
     const size_t smem = region + (size_t)(nb * (nb - 1) / 2 + 2) * sizeof(double);
@@ -1054,22 +1052,64 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
     if (per_sm < 1 || per_sm > 3) per_sm = 3;
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
-    KScope k(K_LU_L1, s);
-    // the tall-panel variant only when the bin can hold > 256 rows (it needs
-    // more registers: the default variant keeps the lower spill count)
-    const bool tall = tuning().l1_rows > L1_MAX_ROWS;
     const int rd = (int)(region / sizeof(double)), pt = tuning().phase_timing, df = tuning().defer;
-    if (tuning().l1_dmma) {  // default: DMMA (measured faster once the variant stopped spilling)
-        if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
-        else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
-    } else {
-        if (tall) lu_l1_kernel<false, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
-        else lu_l1_kernel<false, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
-    }
+    const bool dm = tuning().l1_dmma;  // default: DMMA (measured faster once the variant stopped spilling)
+    // one launch per bin: matrices of 257..l1_rows rows (BIN_L1T) by the
+    // tall-panel variant (windowed panels in place), the rest by the staged-
+    // panel variant, which needs fewer registers; each walks its bin LPT first
+    auto one = [&](int bin, bool tall) {
+        const int *order = nullptr, *order_count = nullptr;
+        if (keys && sort_ws) {
+            cudaMemsetAsync(keys, 0, (size_t)a.batch * sizeof(int), s);
+            {
+                KScope k(K_MISC, s);
+                int g = (a.batch + 255) / 256;
+                l1_key_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(a, counters, bins, keys, bin);
+            }
+            launch_size_sort(keys, a.batch, sort_ws, s);
+            SlotList sl = sorted_slots(sort_ws, a.batch, 31);
+            order = sl.idx;
+            order_count = sl.prefix + sl.bucket0;
+        }
+        cudaMemsetAsync(counters + CNT_L1_NEXT, 0, sizeof(int), s);
+        KScope k(K_LU_L1, s);
+        if (dm) {
+            if (tall) lu_l1_kernel<true, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+            else lu_l1_kernel<true, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+        } else {
+            if (tall) lu_l1_kernel<false, true><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+            else lu_l1_kernel<false, false><<<grid, L1_NT, smem, s>>>(a, counters, bins, nb, rd, pt, order, order_count, df);
+        }
+    };
+    if (tuning().l1_rows > L1_MAX_ROWS) one(BIN_L1T, true);
+    one(BIN_L1, false);
 }
 
-void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans_v,
-                     void *outer_plans_v, cudaStream_t s) {
+// the grid-wide tier's list in LPT order (largest first, buckets of 32 in
+// the cube-root key): every kernel of the tier walks slots in this order, so
+// the dynamic queues hand out the biggest panels / strips first
+__global__ void set_bin_list_kernel(const int *__restrict__ sorted, const int *__restrict__ count_ptr,
+                                    int *__restrict__ dst) {
+    const int count = *count_ptr;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < count; t += gridDim.x * blockDim.x) dst[t] = sorted[t];
+}
+
+void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *tile_off, void *plans_v,
+                     void *outer_plans_v, cudaStream_t s, int *keys, int *sort_ws) {
+    int *bins = const_cast<int *>(bins_c);
+    if (keys && sort_ws) {
+        cudaMemsetAsync(keys, 0, (size_t)a.batch * sizeof(int), s);
+        const int g = (a.batch + 255) / 256;
+        {
+            KScope k(K_MISC, s);
+            l1_key_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(a, counters, bins, keys, BIN_L);
+        }
+        launch_size_sort(keys, a.batch, sort_ws, s);
+        SlotList sl = sorted_slots(sort_ws, a.batch, 31);
+        KScope k(K_MISC, s);
+        set_bin_list_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(sl.idx, sl.prefix + sl.bucket0,
+                                                                bins + (size_t)BIN_L * a.batch);
+    }
     SwapPlan *plans = reinterpret_cast<SwapPlan *>(plans_v);
     const Tuning &tu = tuning();
     const int nb = clamp_nb(tu.nb);
@@ -1181,6 +1221,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *ti
                                                                       defer, -1, 1 << 30);
             continue;
         }
+        cudaMemsetAsync(counters + CNT_PANELQ, 0, sizeof(int), s);  // no strip kernel resets it on this path
         {
             KScope k(K_SWAP_TRSM, s);
             swap_trsm_kernel<<<grid_s, SW_NT, sw_smem, s>>>(a, counters, bins, j, nb, chunks_per);
