@@ -42,7 +42,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
 // CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
 // rows: C3 61.7), 8-warp xgemm CTAs (16 warps: C3 58.3, C5 651 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -133,6 +133,8 @@ int num_sms() {
 struct DeviceStreams {
     cudaStream_t side = nullptr;
     cudaEvent_t fork = nullptr, join = nullptr;
+    cudaStream_t side2 = nullptr;             // the grid tier's second part
+    cudaEvent_t fork2 = nullptr, join2 = nullptr;
 };
 static DeviceStreams g_streams[64];
 
@@ -145,6 +147,9 @@ static DeviceStreams *dev_streams() {
         if (cudaStreamCreateWithFlags(&d.side, cudaStreamNonBlocking) != cudaSuccess) { d.side = nullptr; return nullptr; }
         cudaEventCreateWithFlags(&d.fork, cudaEventDisableTiming);
         cudaEventCreateWithFlags(&d.join, cudaEventDisableTiming);
+        if (cudaStreamCreateWithFlags(&d.side2, cudaStreamNonBlocking) != cudaSuccess) d.side2 = nullptr;
+        cudaEventCreateWithFlags(&d.fork2, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&d.join2, cudaEventDisableTiming);
     }
     return &d;
 }
@@ -171,6 +176,7 @@ struct Work {
     int *keys;  // per-matrix sort keys
     void *plans;  // getrf / partial only: one interchange plan per tier-L slot
     void *outer_plans;  // getrf / partial only: one outer-block plan per tier-L slot (two-level tier)
+    int *part_counters, *part_list, *part_tile_off;  // getrf / partial only: the grid tier's second part
 };
 
 static size_t work_bytes_for(int batch) {
@@ -183,7 +189,8 @@ static size_t work_bytes_for(int batch) {
 // grid-wide tier (written by its panel kernel, read by its strip kernel)
 static size_t work_bytes_getrf(int batch) {
     size_t b = (size_t)(batch > 0 ? batch : 1);
-    return work_bytes_for(batch) + align256(b * SWAP_PLAN_BYTES) + align256(b * OUTER_PLAN_BYTES);
+    return work_bytes_for(batch) + align256(b * SWAP_PLAN_BYTES) + align256(b * OUTER_PLAN_BYTES) +
+           align256(CNT_INTS * sizeof(int)) + align256(b * sizeof(int)) + align256((b + 1) * sizeof(int));
 }
 
 static Work carve(void *work, int batch) {
@@ -203,6 +210,12 @@ static Work carve(void *work, int batch) {
     w.plans = p;  // valid only in a work_bytes_getrf() workspace
     p += align256(b * SWAP_PLAN_BYTES);
     w.outer_plans = p;
+    p += align256(b * OUTER_PLAN_BYTES);
+    w.part_counters = (int *)p;
+    p += align256(CNT_INTS * sizeof(int));
+    w.part_list = (int *)p;
+    p += align256(b * sizeof(int));
+    w.part_tile_off = (int *)p;
     return w;
 }
 
@@ -252,7 +265,12 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
         }
         if (has_large) {
             if (t.l1) launch_lu_l1(a, w.counters, w.bins, w.keys, w.sort, s);
-            if (!t.l1 || a.max_m > t.l1_rows) launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, w.outer_plans, s, w.keys, w.sort);
+            if (!t.l1 || a.max_m > t.l1_rows) {
+                DeviceStreams *ds = dev_streams();
+                PartWork pw{w.part_counters, w.part_list, w.part_tile_off, ds ? ds->side2 : nullptr,
+                            ds ? ds->fork2 : nullptr, ds ? ds->join2 : nullptr};
+                launch_lu_large(a, w.counters, w.bins, w.tile_off, w.plans, w.outer_plans, s, w.keys, w.sort, &pw);
+            }
         }
     }
     if (side != s) {
@@ -334,6 +352,8 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
     else if (!strcmp(key, "nb_outer")) g_tuning.nb_outer = value < 0 ? 0 : (value > NB_OUTER_MAX ? NB_OUTER_MAX : value);
     else if (!strcmp(key, "xgemm_warps")) g_tuning.xgemm_warps = value >= 16 ? 16 : 8;
+    else if (!strcmp(key, "parts")) g_tuning.parts = value >= 2 ? 2 : 1;
+    else if (!strcmp(key, "part_grid")) g_tuning.part_grid = value >= 2 ? 2 : 1;
 }
 
 int irr_get_tuning(const char *key) {
@@ -358,6 +378,8 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) return g_tuning.defer;
     if (!strcmp(key, "nb_outer")) return g_tuning.nb_outer;
     if (!strcmp(key, "xgemm_warps")) return g_tuning.xgemm_warps;
+    if (!strcmp(key, "parts")) return g_tuning.parts;
+    if (!strcmp(key, "part_grid")) return g_tuning.part_grid;
     return -1;
 }
 

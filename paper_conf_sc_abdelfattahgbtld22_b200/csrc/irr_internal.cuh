@@ -35,6 +35,8 @@ struct Tuning {
     int getrs_vec;       // 1: irr_getrs with max_nrhs <= 4 by the CTA-per-system kernel (getrs_vec.cu)
     int nb_outer;        // grid-wide tier: outer block width of the two-level blocking (0 / <= nb: one level)
     int xgemm_warps;     // 8 or 16 warps per 128 x 128 DMMA tile CTA (the two-level trailing GEMM)
+    int parts;           // two-level grid tier: 1, or 2 halves of the LPT list on two streams
+    int part_grid;       // with 2 parts: 1 = full grids per part, 2 = half grids
 };
 Tuning &tuning();
 
@@ -240,8 +242,17 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
 constexpr size_t SWAP_PLAN_BYTES = 1040;  // sizeof(SwapPlan), checked in lu_large.cu
 constexpr int NB_OUTER_MAX = 128;          // widest outer block of the two-level grid tier
 constexpr size_t OUTER_PLAN_BYTES = 2064;  // sizeof(OuterPlan), checked in lu_large.cu
+// second part of the two-level grid tier (tuning parts = 2): its own counters
+// block, list, tile offsets and stream
+struct PartWork {
+    int *counters;  // CNT_INTS ints
+    int *list;      // batch ints
+    int *tile_off;  // batch + 1 ints
+    cudaStream_t side;
+    cudaEvent_t fork, join;
+};
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins, int *tile_off, void *plans, void *outer_plans,
-                     cudaStream_t s, int *keys = nullptr, int *sort_ws = nullptr);
+                     cudaStream_t s, int *keys = nullptr, int *sort_ws = nullptr, PartWork *pw = nullptr);
 void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys, int *sort_ws, cudaStream_t s);
 
 // gemm_vb.cu : DCWI gemm on pointer arrays (irr_gemm semantics)

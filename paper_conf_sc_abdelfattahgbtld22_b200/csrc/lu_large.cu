@@ -1088,15 +1088,32 @@ void launch_lu_l1(const GetrfArgs &a, int *counters, const int *bins, int *keys,
 // the grid-wide tier's list in LPT order (largest first, buckets of 32 in
 // the cube-root key): every kernel of the tier walks slots in this order, so
 // the dynamic queues hand out the biggest panels / strips first
+// With two parts the sorted list is dealt alternately (part p gets the
+// entries t = p, p + 2, ...: both halves LPT-ordered and flop-balanced); each
+// part's count goes to its own counters block.
 __global__ void set_bin_list_kernel(const int *__restrict__ sorted, const int *__restrict__ count_ptr,
-                                    int *__restrict__ dst) {
+                                    int *__restrict__ dst, int *__restrict__ dst_b, int *__restrict__ cnt_a,
+                                    int *__restrict__ cnt_b) {
     const int count = *count_ptr;
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < count; t += gridDim.x * blockDim.x) dst[t] = sorted[t];
+    const int parts = dst_b ? 2 : 1;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < count; t += gridDim.x * blockDim.x) {
+        if (parts == 1 || !(t & 1)) dst[t / parts] = sorted[t];
+        else dst_b[t / 2] = sorted[t];
+    }
+    if (parts == 2 && blockIdx.x == 0 && threadIdx.x == 0) {
+        *cnt_a = (count + 1) / 2;
+        *cnt_b = count / 2;
+    }
 }
 
 void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *tile_off, void *plans_v,
-                     void *outer_plans_v, cudaStream_t s, int *keys, int *sort_ws) {
+                     void *outer_plans_v, cudaStream_t s, int *keys, int *sort_ws, PartWork *pw) {
     int *bins = const_cast<int *>(bins_c);
+    const Tuning &tu = tuning();
+    // two parts (the LPT list dealt alternately) on two streams: one part's
+    // latency-bound panels / strips / interchanges overlap the other part's
+    // trailing GEMMs (two-level path only; see below)
+    const bool two_parts = pw && pw->side && tu.parts == 2 && keys && sort_ws;
     if (keys && sort_ws) {
         cudaMemsetAsync(keys, 0, (size_t)a.batch * sizeof(int), s);
         const int g = (a.batch + 255) / 256;
@@ -1106,12 +1123,13 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
         }
         launch_size_sort(keys, a.batch, sort_ws, s);
         SlotList sl = sorted_slots(sort_ws, a.batch, 31);
+        if (two_parts) cudaMemsetAsync(pw->counters, 0, CNT_INTS * sizeof(int), s);
         KScope k(K_MISC, s);
-        set_bin_list_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(sl.idx, sl.prefix + sl.bucket0,
-                                                                bins + (size_t)BIN_L * a.batch);
+        set_bin_list_kernel<<<g < 1024 ? g : 1024, 256, 0, s>>>(
+            sl.idx, sl.prefix + sl.bucket0, bins + (size_t)BIN_L * a.batch, two_parts ? pw->list : nullptr,
+            counters + CNT_BIN0 + BIN_L, two_parts ? pw->counters + CNT_BIN0 + BIN_L : nullptr);
     }
     SwapPlan *plans = reinterpret_cast<SwapPlan *>(plans_v);
-    const Tuning &tu = tuning();
     const int nb = clamp_nb(tu.nb);
     const int Kmax = a.max_m < a.max_n ? a.max_m : a.max_n;
     // shared-memory panel rows: (rows|1) * nb doubles within the opt-in limit
@@ -1161,47 +1179,75 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 8>, BIG_SMEM);
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 16>, BIG_SMEM);
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
-        const int *cnt_ptr = counters + CNT_BIN0 + BIN_L;
-        for (int J = 0; J < Kmax; J += nbo) {
-            for (int j = J; j < Kmax && j < J + nbo; j += nb) {
-                {
-                    KScope k(K_PANEL, s);
-                    launch_panel_win(a.max_m - j, grid_w, a, counters, bins, j, nb, plans, counters + CNT_STRIPQ, s);
+        // one part = one list of tier-L slots with its own counters block
+        // (count, queues), plan slots, tile offsets and stream
+        auto run_part = [&](int *cnt, int *bns, SwapPlan *pl, OuterPlan *opl, int *toff, cudaStream_t st, int gdiv) {
+            const int *listP = bns + (size_t)BIN_L * a.batch;
+            const int *cnt_ptr = cnt + CNT_BIN0 + BIN_L;
+            const int gs = sms / gdiv > 0 ? sms / gdiv : 1;
+            const int gw = grid_w / gdiv > 0 ? grid_w / gdiv : 1;
+            for (int J = 0; J < Kmax; J += nbo) {
+                for (int j = J; j < Kmax && j < J + nbo; j += nb) {
+                    {
+                        KScope k(K_PANEL, st);
+                        launch_panel_win(a.max_m - j, gw, a, cnt, bns, j, nb, pl, cnt + CNT_STRIPQ, st);
+                    }
+                    KScope k(K_STRIP, st);
+                    if (tu.dmma) strip_kernel<true><<<gs * 3, G_NT, st_smem, st>>>(
+                        a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
+                    else strip_kernel<false><<<gs * 3, G_NT, st_smem, st>>>(
+                        a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
                 }
-                KScope k(K_STRIP, s);
-                if (tu.dmma) strip_kernel<true><<<sms * 3, G_NT, st_smem, s>>>(
-                    a, counters, bins, plans, counters + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
-                else strip_kernel<false><<<sms * 3, G_NT, st_smem, s>>>(
-                    a, counters, bins, plans, counters + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
+                {
+                    KScope k(K_MISC, st);
+                    int g = (a.batch + OP_NT / 32 - 1) / (OP_NT / 32);
+                    if (g > gs * 8) g = gs * 8;
+                    outer_plan_kernel<<<g, OP_NT, 0, st>>>(a, cnt, bns, J, nbo, opl, cnt + CNT_OUTQ);
+                }
+                {
+                    KScope k(K_GEMM_SCAN, st);
+                    scan_units_kernel<OuterStrips><<<1, 1024, 0, st>>>(OuterStrips{a, listP, J, nbo},
+                                                                       SlotList{nullptr, cnt_ptr, 0}, a.batch, toff);
+                }
+                {
+                    KScope k(K_OUTER_TRSM, st);
+                    outer_swap_trsm_kernel<<<gs, OS_NT, OS_SMEM, st>>>(a, cnt, bns, opl, toff, J, nbo);
+                }
+                OuterTrailProb P{a, listP, J, nbo};
+                {
+                    KScope k(K_GEMM_SCAN, st);
+                    xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, st>>>(P, -1, cnt_ptr, toff);
+                }
+                KScope k(K_GEMM_TRAIL, st);
+                if (tu.xgemm_warps == 16)
+                    xgemm_sched_kernel<OuterTrailProb, 0, 0, 16><<<gs * XGEMM_MINB, 512, BIG_SMEM, st>>>(P, -1, cnt_ptr,
+                                                                                                     toff);
+                else
+                    xgemm_sched_kernel<OuterTrailProb, 0, 0, 8><<<gs * XGEMM_MINB, 256, BIG_SMEM, st>>>(P, -1, cnt_ptr,
+                                                                                                    toff);
             }
-            {
-                KScope k(K_MISC, s);
-                int g = (a.batch + OP_NT / 32 - 1) / (OP_NT / 32);
-                if (g > sms * 8) g = sms * 8;
-                outer_plan_kernel<<<g, OP_NT, 0, s>>>(a, counters, bins, J, nbo, oplans, counters + CNT_OUTQ);
+            if (Kmax > nbo) {  // deferred left-block interchanges of this part
+                cudaMemsetAsync(cnt + CNT_LSWQ, 0, sizeof(int), st);
+                KScope k(K_LEFT_SWAPS, st);
+                int grid = 2 * gs;
+                if (grid > a.batch) grid = a.batch;
+                left_swaps_kernel<<<grid, LSW_NT, lsw_smem, st>>>(a, cnt, bns, nbo, a.max_m, lsw_bufd, cnt + CNT_LSWQ);
             }
-            {
-                KScope k(K_GEMM_SCAN, s);
-                scan_units_kernel<OuterStrips><<<1, 1024, 0, s>>>(OuterStrips{a, listL, J, nbo},
-                                                                  SlotList{nullptr, cnt_ptr, 0}, a.batch, tile_off);
-            }
-            {
-                KScope k(K_OUTER_TRSM, s);
-                outer_swap_trsm_kernel<<<sms, OS_NT, OS_SMEM, s>>>(a, counters, bins, oplans, tile_off, J, nbo);
-            }
-            OuterTrailProb P{a, listL, J, nbo};
-            {
-                KScope k(K_GEMM_SCAN, s);
-                xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, s>>>(P, -1, cnt_ptr, tile_off);
-            }
-            KScope k(K_GEMM_TRAIL, s);
-            if (tu.xgemm_warps == 16)
-                xgemm_sched_kernel<OuterTrailProb, 0, 0, 16><<<sms * XGEMM_MINB, 512, BIG_SMEM, s>>>(P, -1, cnt_ptr,
-                                                                                                 tile_off);
-            else
-                xgemm_sched_kernel<OuterTrailProb, 0, 0, 8><<<sms * XGEMM_MINB, 256, BIG_SMEM, s>>>(P, -1, cnt_ptr,
-                                                                                                tile_off);
+        };
+        if (two_parts) {
+            const size_t half = ((size_t)a.batch + 1) / 2;
+            cudaEventRecord(pw->fork, s);
+            cudaStreamWaitEvent(pw->side, pw->fork, 0);
+            const int gdiv = tu.part_grid == 2 ? 2 : 1;
+            run_part(counters, bins, plans, oplans, tile_off, s, gdiv);
+            run_part(pw->counters, pw->list - (size_t)BIN_L * a.batch, plans + half, oplans + half, pw->tile_off,
+                     pw->side, gdiv);
+            cudaEventRecord(pw->join, pw->side);
+            cudaStreamWaitEvent(s, pw->join, 0);
+        } else {
+            run_part(counters, bins, plans, oplans, tile_off, s, 1);
         }
+        return;
     } else
     for (int j = 0; j < Kmax; j += nb) {
         if (tu.panel_win) {

@@ -424,3 +424,22 @@ def test_results_bitwise_identical_across_shard_counts():
             ref = got
         else:
             assert got == ref, f"G = {G} differs from G = 1"
+
+
+@pytest.mark.parametrize("part_grid", [1, 2])
+def test_two_parts_bitwise_equal(part_grid):
+    """The two-level grid tier split into two LPT halves on two streams
+    (tuning parts = 2) factors every matrix bitwise as the single list does
+    (the per-matrix arithmetic does not depend on the part), and matches the
+    oracle."""
+    shapes = [(700, 700), (300, 260), (1024, 900), (520, 520), (2000, 300), (300, 2000), (45, 45), (600, 601),
+              (1500, 1500)]
+    mats = _uniform(shapes, seed=97)
+    one, ip1, inf1, _ = gpu_getrf(mats)
+    irr.irr_set_tuning("parts", 2)
+    irr.irr_set_tuning("part_grid", part_grid)
+    two, ip2, inf2, _ = gpu_getrf(mats)
+    for a, b, p, q in zip(one, two, ip1, ip2):
+        assert np.array_equal(a, b) and np.array_equal(p, q)
+    assert np.array_equal(inf1, inf2)
+    _run_and_check(mats)
