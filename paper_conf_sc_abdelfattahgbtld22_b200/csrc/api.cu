@@ -42,7 +42,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
 // CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
 // rows: C3 61.7), 8-warp xgemm CTAs (16 warps: C3 58.3, C5 651 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1};
+static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1, 64};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -354,6 +354,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "xgemm_warps")) g_tuning.xgemm_warps = value >= 16 ? 16 : 8;
     else if (!strcmp(key, "parts")) g_tuning.parts = value >= 2 ? 2 : 1;
     else if (!strcmp(key, "part_grid")) g_tuning.part_grid = value >= 2 ? 2 : 1;
+    else if (!strcmp(key, "outer_cols")) g_tuning.outer_cols = value <= 32 ? 32 : 64;
 }
 
 int irr_get_tuning(const char *key) {
@@ -380,6 +381,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "xgemm_warps")) return g_tuning.xgemm_warps;
     if (!strcmp(key, "parts")) return g_tuning.parts;
     if (!strcmp(key, "part_grid")) return g_tuning.part_grid;
+    if (!strcmp(key, "outer_cols")) return g_tuning.outer_cols;
     return -1;
 }
 

@@ -29,10 +29,13 @@ namespace irr {
 #ifndef XGEMM_MINB
 #define XGEMM_MINB 1    // resident CTAs per SM
 #endif
-constexpr int XBM = 128, XBN = 128, XBK = 16, X_NT = 256, XST = XGEMM_ST;
+#ifndef XGEMM_BK
+#define XGEMM_BK 16     // K chunk per ring stage
+#endif
+constexpr int XBM = 128, XBN = 128, XBK = XGEMM_BK, X_NT = 256, XST = XGEMM_ST;
 constexpr int XLD_KM = 132;  // [k][m] layout: XBK rows of XBM (+4)
-constexpr int XLD_MK = 20;   // [m][k] layout: XBM rows of XBK (+4)
-constexpr int XSTAGE = 2560; // doubles per operand stage: max(16 * 132, 128 * 20)
+constexpr int XLD_MK = XBK + 4;   // [m][k] layout: XBM rows of XBK (+4)
+constexpr int XSTAGE = (XBK * XLD_KM > XBM * XLD_MK) ? XBK * XLD_KM : XBM * XLD_MK;  // doubles per operand stage
 
 struct BigSmem {
     double A[XST][XSTAGE];

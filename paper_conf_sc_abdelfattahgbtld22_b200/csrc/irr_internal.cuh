@@ -37,6 +37,7 @@ struct Tuning {
     int xgemm_warps;     // 8 or 16 warps per 128 x 128 DMMA tile CTA (the two-level trailing GEMM)
     int parts;           // two-level grid tier: 1, or 2 halves of the LPT list on two streams
     int part_grid;       // with 2 parts: 1 = full grids per part, 2 = half grids
+    int outer_cols;      // two-level interchange + U12 solve strip width: 64 (L11 square, 1 CTA/SM) or 32 (packed, 2/SM)
 };
 Tuning &tuning();
 

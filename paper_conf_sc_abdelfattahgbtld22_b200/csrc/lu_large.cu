@@ -770,9 +770,24 @@ __global__ void __launch_bounds__(OP_NT) outer_plan_kernel(GetrfArgs a, const in
 //      broadcast by shuffle), the rows below it by a rank-32 DMMA update
 //      (m8n8k4, both operands in shared memory);
 //   3. U12 back to rows [J, J + ibo), one thread per row (coalesced).
-constexpr int OS_COLS = 64, OS_NT = 256, OS_TLD = OS_COLS + 1, OS_LDL = 136;
-constexpr size_t OS_SMEM = (size_t)(NB_OUTER_MAX * OS_TLD + NB_OUTER_MAX * OS_LDL) * sizeof(double);
+// Two shapes: 64-column strips with L11 in a padded square (1 CTA / SM,
+// 206 KB), or 32-column strips with L11's strict lower triangle packed by
+// columns (2 CTAs / SM, 101 KB) -- tuning outer_cols.
+constexpr int OS_NT = 256, OS_LDL = 136;
+constexpr int OS_LPACK = NB_OUTER_MAX * (NB_OUTER_MAX - 1) / 2;
+template <int COLS>
+struct OsCfg {
+    static constexpr bool PACK = COLS <= 32;
+    static constexpr int TLD = COLS + 1;
+    static constexpr size_t SMEM =
+        (size_t)(NB_OUTER_MAX * TLD + (PACK ? OS_LPACK : NB_OUTER_MAX * OS_LDL)) * sizeof(double);
+    // L11(r, s), r > s
+    __device__ static __forceinline__ int lidx(int r, int s) {
+        return PACK ? s * (2 * NB_OUTER_MAX - 1 - s) / 2 + (r - s - 1) : s * OS_LDL + r;
+    }
+};
 
+template <int COLS>
 struct OuterStrips {
     GetrfArgs a;
     const int *list;
@@ -783,21 +798,24 @@ struct OuterStrips {
         const int K = mi < ni ? mi : ni;
         if (J >= K) return 0;
         const int c1 = J + imin(NBo, K - J);
-        return c1 < ni ? (ni - c1 + OS_COLS - 1) / OS_COLS : 0;
+        return c1 < ni ? (ni - c1 + COLS - 1) / COLS : 0;
     }
 };
 
-__global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, const int *__restrict__ counters,
-                                                                   const int *__restrict__ bins,
-                                                                   const OuterPlan *__restrict__ plans,
-                                                                   const int *__restrict__ off, int J, int NBo) {
+template <int COLS>
+__global__ void __launch_bounds__(OS_NT, COLS <= 32 ? 2 : 1) outer_swap_trsm_kernel(
+    GetrfArgs a, const int *__restrict__ counters, const int *__restrict__ bins, const OuterPlan *__restrict__ plans,
+    const int *__restrict__ off, int J, int NBo) {
+    using Cfg = OsCfg<COLS>;
+    constexpr int TLD = Cfg::TLD;
     extern __shared__ __align__(16) double os_smem[];
-    double *top = os_smem;                       // U12 rows: top[t * OS_TLD + c]
-    double *Ls = top + NB_OUTER_MAX * OS_TLD;    // L11: Ls[s * OS_LDL + r] (column s, row r)
+    double *top = os_smem;                       // U12 rows: top[t * TLD + c]
+    double *Ls = top + NB_OUTER_MAX * TLD;       // L11 strict lower: Ls[Cfg::lidx(r, s)]
     __shared__ OuterPlan sp;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int g = lane >> 2, t4 = lane & 3;
     constexpr int NWS = OS_NT / 32;
+    constexpr int CPW = COLS / NWS;   // diagonal-solve columns per warp
     const int count = counters[CNT_BIN0 + BIN_L];
     const int *list = bins + (size_t)BIN_L * a.batch;
     int last_slot = -1;
@@ -806,8 +824,8 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
         const int mi = a.m[i], ni = a.n[i];
         const int K = mi < ni ? mi : ni;
         const int ibo = imin(NBo, K - J), c1 = J + ibo;
-        const int cb = c1 + q * OS_COLS;
-        const int W = imin(OS_COLS, ni - cb);
+        const int cb = c1 + q * COLS;
+        const int W = imin(COLS, ni - cb);
         const long ld = a.ld[i];
         double *gA = a.A[i];
         if (slot != last_slot) {
@@ -818,7 +836,7 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
             // strict lower part of L11, column by column (lanes over rows)
             for (int sc = warp; sc < ibo - 1; sc += NWS) {
                 const double *gl = gA + J + (size_t)(J + sc) * ld;
-                for (int r = sc + 1 + lane; r < ibo; r += 32) cp_async8(&Ls[sc * OS_LDL + r], gl + r);
+                for (int r = sc + 1 + lane; r < ibo; r += 32) cp_async8(&Ls[Cfg::lidx(r, sc)], gl + r);
             }
             last_slot = slot;
         }
@@ -826,11 +844,11 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
         const int nbot = sp.nbot;
         // ---- 1. gather: threads [0, 128) the top rows, [128, 256) the rows pushed down
         const double *gcb = gA + (size_t)cb * ld;
-        double bv[OS_COLS];
+        double bv[COLS];
         if (tid < NB_OUTER_MAX) {
             if (tid < ibo) {
                 const double *src = gcb + sp.top_src[tid];
-                double *dst = top + tid * OS_TLD;
+                double *dst = top + tid * TLD;
 #pragma unroll 8
                 for (int c = 0; c < W; ++c) cp_async8(dst + c, src + (size_t)c * ld);
             }
@@ -839,7 +857,7 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
             if (b < nbot) {
                 const double *src = gcb + sp.bot_src[b];
 #pragma unroll
-                for (int c = 0; c < OS_COLS; ++c) bv[c] = c < W ? src[(size_t)c * ld] : 0.0;
+                for (int c = 0; c < COLS; ++c) bv[c] = c < W ? src[(size_t)c * ld] : 0.0;
             }
         }
         cp_async_commit();
@@ -850,7 +868,7 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
             if (b < nbot) {
                 double *dst = gA + (size_t)cb * ld + sp.bot_pos[b];
 #pragma unroll
-                for (int c = 0; c < OS_COLS; ++c)
+                for (int c = 0; c < COLS; ++c)
                     if (c < W) dst[(size_t)c * ld] = bv[c];
             }
         }
@@ -858,24 +876,24 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
         for (int d0 = 0; d0 < ibo; d0 += 32) {
             const int bw = imin(32, ibo - d0);
             const int below = ibo - d0 - bw;
-            {   // diagonal block: warp w solves columns [8w, 8w + 8), lane = row
-                const int c0 = warp * 8;
-                double x[8];
+            {   // diagonal block: warp w solves columns [CPW w, CPW w + CPW), lane = row
+                const int c0 = warp * CPW;
+                double x[CPW];
 #pragma unroll
-                for (int c = 0; c < 8; ++c) x[c] = (lane < bw && c0 + c < W) ? top[(d0 + lane) * OS_TLD + c0 + c] : 0.0;
+                for (int c = 0; c < CPW; ++c) x[c] = (lane < bw && c0 + c < W) ? top[(d0 + lane) * TLD + c0 + c] : 0.0;
                 for (int sc = 0; sc < bw - 1; ++sc) {
-                    const double l = (lane > sc && lane < bw) ? Ls[(d0 + sc) * OS_LDL + d0 + lane] : 0.0;
+                    const double l = (lane > sc && lane < bw) ? Ls[Cfg::lidx(d0 + lane, d0 + sc)] : 0.0;
 #pragma unroll
-                    for (int c = 0; c < 8; ++c) x[c] = fma(-l, __shfl_sync(FULL, x[c], sc), x[c]);
+                    for (int c = 0; c < CPW; ++c) x[c] = fma(-l, __shfl_sync(FULL, x[c], sc), x[c]);
                 }
                 if (lane < bw)
 #pragma unroll
-                    for (int c = 0; c < 8; ++c)
-                        if (c0 + c < W) top[(d0 + lane) * OS_TLD + c0 + c] = x[c];
+                    for (int c = 0; c < CPW; ++c)
+                        if (c0 + c < W) top[(d0 + lane) * TLD + c0 + c] = x[c];
             }
             __syncthreads();
             if (below > 0) {   // rows below: 32 x 32 output tiles per warp (DMMA)
-                const int tiles_m = (below + 31) / 32, tiles = tiles_m * 2;
+                const int tiles_m = (below + 31) / 32, tiles = tiles_m * (COLS / 32);
                 for (int tt = warp; tt < tiles; tt += NWS) {
                     const int rb = (tt % tiles_m) * 32, cbt = (tt / tiles_m) * 32;
                     double acc[4][4][2];
@@ -890,12 +908,12 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
 #pragma unroll
                         for (int mi = 0; mi < 4; ++mi) {
                             const int r = rb + 8 * mi + g;   // row under the diagonal block
-                            av[mi] = (sc < bw && r < below) ? Ls[(d0 + sc) * OS_LDL + d0 + bw + r] : 0.0;
+                            av[mi] = (sc < bw && r < below) ? Ls[Cfg::lidx(d0 + bw + r, d0 + sc)] : 0.0;
                         }
 #pragma unroll
                         for (int n8 = 0; n8 < 4; ++n8) {
                             const int c = cbt + 8 * n8 + g;
-                            bb[n8] = (sc < bw && c < W) ? top[(d0 + sc) * OS_TLD + c] : 0.0;
+                            bb[n8] = (sc < bw && c < W) ? top[(d0 + sc) * TLD + c] : 0.0;
                         }
 #pragma unroll
                         for (int mi = 0; mi < 4; ++mi)
@@ -906,7 +924,7 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
                     for (int mi = 0; mi < 4; ++mi) {
                         const int r = rb + 8 * mi + g;
                         if (r >= below) continue;
-                        double *row = top + (size_t)(d0 + bw + r) * OS_TLD;
+                        double *row = top + (size_t)(d0 + bw + r) * TLD;
 #pragma unroll
                         for (int n8 = 0; n8 < 4; ++n8) {
                             const int c = cbt + 8 * n8 + 2 * t4;
@@ -921,7 +939,7 @@ __global__ void __launch_bounds__(OS_NT, 1) outer_swap_trsm_kernel(GetrfArgs a, 
         // ---- 3. U12 back to rows [J, J + ibo), one thread per row
         if (tid < ibo) {
             double *dst = gA + J + tid + (size_t)cb * ld;
-            const double *src = top + tid * OS_TLD;
+            const double *src = top + tid * TLD;
 #pragma unroll 8
             for (int c = 0; c < W; ++c) dst[(size_t)c * ld] = src[c];
         }
@@ -1175,7 +1193,9 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
     }
     if (outer) {
         OuterPlan *oplans = reinterpret_cast<OuterPlan *>(outer_plans_v);
-        smem_optin(outer_swap_trsm_kernel, OS_SMEM);
+        smem_optin(outer_swap_trsm_kernel<64>, OsCfg<64>::SMEM);
+        smem_optin(outer_swap_trsm_kernel<32>, OsCfg<32>::SMEM);
+        const bool os32 = tu.outer_cols == 32;
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 8>, BIG_SMEM);
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 16>, BIG_SMEM);
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
@@ -1206,12 +1226,19 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
                 }
                 {
                     KScope k(K_GEMM_SCAN, st);
-                    scan_units_kernel<OuterStrips><<<1, 1024, 0, st>>>(OuterStrips{a, listP, J, nbo},
-                                                                       SlotList{nullptr, cnt_ptr, 0}, a.batch, toff);
+                    if (os32)
+                        scan_units_kernel<OuterStrips<32>><<<1, 1024, 0, st>>>(
+                            OuterStrips<32>{a, listP, J, nbo}, SlotList{nullptr, cnt_ptr, 0}, a.batch, toff);
+                    else
+                        scan_units_kernel<OuterStrips<64>><<<1, 1024, 0, st>>>(
+                            OuterStrips<64>{a, listP, J, nbo}, SlotList{nullptr, cnt_ptr, 0}, a.batch, toff);
                 }
                 {
                     KScope k(K_OUTER_TRSM, st);
-                    outer_swap_trsm_kernel<<<gs, OS_NT, OS_SMEM, st>>>(a, cnt, bns, opl, toff, J, nbo);
+                    if (os32)
+                        outer_swap_trsm_kernel<32><<<2 * gs, OS_NT, OsCfg<32>::SMEM, st>>>(a, cnt, bns, opl, toff, J, nbo);
+                    else
+                        outer_swap_trsm_kernel<64><<<gs, OS_NT, OsCfg<64>::SMEM, st>>>(a, cnt, bns, opl, toff, J, nbo);
                 }
                 OuterTrailProb P{a, listP, J, nbo};
                 {

@@ -443,3 +443,16 @@ def test_two_parts_bitwise_equal(part_grid):
         assert np.array_equal(a, b) and np.array_equal(p, q)
     assert np.array_equal(inf1, inf2)
     _run_and_check(mats)
+
+
+@pytest.mark.parametrize("cols", [32, 64])
+def test_outer_strip_widths(cols):
+    """The two-level interchange + U12 solve in 32-column strips (packed L11,
+    2 CTAs / SM) and 64-column strips (square L11, 1 CTA / SM): oracle parity
+    and G1 bit-exactness."""
+    irr.irr_set_tuning("l1", 0)
+    irr.irr_set_tuning("outer_cols", cols)
+    shapes = [(700, 700), (300, 1000), (1000, 300), (513, 513), (1300, 1300), (129, 900)]
+    _run_and_check(_uniform(shapes, seed=101 + cols))
+    mats = [irrgen.g1_exact(17, g, m, n)[0] for g, (m, n) in enumerate([(600, 600), (300, 700), (900, 400)])]
+    _run_and_check(mats, exact=True)
