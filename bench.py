@@ -533,7 +533,7 @@ def run_e2e(args, B, kind, host, flush, stream, world, sm, sn, words, status, ga
     Be, note = B, "whole batch"
     if host is None:
         avail = psutil.virtual_memory().available
-        budget = int(avail * 0.70) // 16          # doubles per host copy (two copies: in, out)
+        budget = int(avail * 0.50) // 16          # doubles per host copy (two pinned copies: in, out)
         i1 = B.batch
         if B.total > budget:
             ends = B.offsets + (B.ld_h * (B.n_h if kind == "getrf" else B.nf_h))

@@ -606,6 +606,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, int *__rest
         if (tid == 0) item_s = atomicAdd(queue, 1);
         __syncthreads();
         const long long w = item_s;
+        __syncthreads();  // every thread has read item_s before thread 0 takes the next item
         if (w >= total) break;
         const int slot = (int)(w / chunks_per), q = (int)(w - (long long)slot * chunks_per);
         const int i = list[slot];

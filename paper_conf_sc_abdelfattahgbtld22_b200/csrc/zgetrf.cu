@@ -126,6 +126,7 @@ __global__ void __launch_bounds__(ZT) zgetrf_kernel(ZArgs a, int *queue, SlotLis
                 const int p = z_iamax(A, ld, k, m, k, skey, srow);
                 if (tid == 0) ip[k] = p + 1;
                 const double2 pv = A[p + (size_t)k * ld];
+                __syncthreads();  // every thread has the pivot before the interchange moves it
                 const bool nz = pv.x != 0.0 || pv.y != 0.0;
                 if (nz) {
                     if (p != k)
