@@ -409,15 +409,21 @@ double oracle_backward_error(int m, int n, const double *A0, int lda0, const dou
                 PA[p + (size_t)j * m] = t;
             }
     }
+    /* the rows of L copied row-major once, so that both operands of the dot
+     * products below are read contiguously (same terms, same order) */
+    double *Lr = (double *)malloc(sizeof(double) * (size_t)(m > 0 ? m : 1) * (size_t)(K > 0 ? K : 1));
+    for (int i = 0; i < m; ++i)
+        for (int l = 0; l < imin(i, K); ++l) Lr[(size_t)i * K + l] = LU[i + (size_t)l * ld];
     long double rn = 0.0L, an = 0.0L;
     for (int j = 0; j < n; ++j)
         for (int i = 0; i < m; ++i) {
             long double s = 0.0L;
             int lim = imin(imin(i, j), K - 1);
+            const double *li = Lr + (size_t)i * K;
+            const double *uj = LU + (size_t)j * ld;
             for (int l = 0; l <= lim; ++l) {
-                long double lv = (l == i) ? 1.0L : (long double)LU[i + (size_t)l * ld];
-                long double uv = (long double)LU[l + (size_t)j * ld];
-                if (l < i || l == i) s += lv * uv;
+                long double lv = (l == i) ? 1.0L : (long double)li[l];
+                s += lv * (long double)uj[l];
             }
             long double d = PA[i + (size_t)j * m] - s;
             rn += d * d;
@@ -425,6 +431,7 @@ double oracle_backward_error(int m, int n, const double *A0, int lda0, const dou
             an += a * a;
         }
     free(PA);
+    free(Lr);
     if (an == 0.0L) return rn == 0.0L ? 0.0 : INFINITY;
     return (double)(sqrtl(rn) / (sqrtl(an) * (long double)imax(1, K) * (long double)DBL_EPSILON));
 }

@@ -32,7 +32,8 @@ from parity import assess_getrf, assess_partial  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200.batch import FrontBatch, MatrixBatch  # noqa: E402
 
-CHUNK = 1 << 27   # doubles of host buffer per checked chunk (1 GiB)
+CHUNK = 1 << 30   # doubles of host buffer per checked chunk (8 GiB: the 47 C4 fronts >= 3072
+                  # fall in one chunk, so the big oracle runs spread over every thread)
 THREADS = len(os.sched_getaffinity(0))
 
 
