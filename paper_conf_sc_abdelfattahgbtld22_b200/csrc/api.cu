@@ -31,7 +31,7 @@ void launch_getrs_vec(int batch, int max_n, int max_nrhs, const int *n, const in
                       cudaStream_t s);
 void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *const *F11, const int *ld11,
                         double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
-                        int *queue, SlotList sl, cudaStream_t s);
+                        int *queue, SlotList sl, cudaStream_t s, int upper = 1);
 
 // defaults chosen by measurement on B200: tier M only up to
 // 48 KB (C2 6.20 -> 6.06 ms against 96 KB, once L1 got faster; C4 100.5 ->
@@ -467,10 +467,11 @@ static int partial_core(int lapack, int batch, int max_n1, int max_n2, const int
     t.max_m = max_n1; t.max_n = max_n2; t.m = n1; t.n = n2; t.alpha = 1.0;
     t.T = (const double *const *)F11; t.Ti = 0; t.Tj = 0; t.ldt = ld11;
     t.B = F12; t.Bi = 0; t.Bj = 0; t.ldb = ld12; t.batch = batch;
-    if (!lapack && tuning().getrs_fused && getrs_strip_ok(max_n1)) {
-        // step 2: F12 <- U^-1 L^-1 P^T F12: one fused strip kernel
+    if (tuning().getrs_fused && getrs_strip_ok(max_n1)) {
+        // step 2: F12 <- U^-1 L^-1 P^T F12 / U12 <- L^-1 P^T F12: one
+        // fused strip kernel (the LAPACK-style variant stops before U^-1)
         launch_getrs_strip(batch, n1, n2, (const double *const *)F11, ld11, F12, ld12, ipiv, info, w.tile_off,
-                           w.counters + CNT_GSQ, sorted_slots(w.sort, batch, 0), s);
+                           w.counters + CNT_GSQ, sorted_slots(w.sort, batch, 0), s, lapack ? 0 : 1);
     } else {
         // irrLASWP + irrTRSM(L, unit) [+ irrTRSM(U)] as the paper composes GETRS
         launch_laswp_masked(max_n2, n2, F12, 0, 0, ld12, 0, max_n1, n1, ipiv, batch, info, s, w.tile_off,

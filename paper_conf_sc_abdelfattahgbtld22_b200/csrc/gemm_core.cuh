@@ -29,10 +29,6 @@ struct GemmDesc {
     double *C; long ldc;
     int m, n, k;
     double alpha, beta;
-    // MAP variants only (the row-map CTA kernel, lu_large.cu): logical row r
-    // of op(A) and C lives at storage row rmap[r]; row k of B at kmap[k]
-    // (shared-memory lists; the pointers above then carry column offsets only)
-    const int *rmap = nullptr, *kmap = nullptr;
 };
 
 constexpr int CPAD = GBM + 2;  // even: 16-byte row pairs of the C stage stay aligned (cp.async16, LDS.128)
@@ -46,33 +42,10 @@ constexpr size_t GEMM_SMEM = sizeof(GemmSmem);
 
 // Issue the cp.async copies of K chunk [k0, k0+16) of tile (r0, c0) into buffer
 // `buf` (out-of-range elements are zero-filled with plain stores).
-template <bool MAP = false, bool BRES = false, bool APAIR = true>
+template <bool BRES = false, bool APAIR = true>
 __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int c0, int k0, GemmSmem &sm, int buf) {
     const int tid = threadIdx.x;
-    if (MAP) {
-        // the row of op(A) (tid & 63) and of B (tid & 15) are fixed per thread:
-        // one map lookup each, all before the cp.async sequence
-        const int r = tid & 63, gr = r0 + r, kb = tid & 15, gkb = k0 + kb;
-        const bool okr = gr < d.m, okb = gkb < d.k;
-        const double *arow = d.A + (okr ? d.rmap[gr] : 0);
-        const double *brow = d.B + (okb ? d.kmap[gkb] : 0);
-#pragma unroll
-        for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
-            const int kk = (tid >> 6) + 2 * q, gk = k0 + kk;
-            double *dst = &sm.As[buf][kk][r];
-            if (okr && gk < d.k) cp_async8(dst, arow + (size_t)gk * d.lda);
-            else *dst = 0.0;
-        }
-#pragma unroll
-        for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
-            const int c = (tid >> 4) + 8 * q, gc = c0 + c;
-            double *dst = &sm.Bs[buf][kb][c];
-            if (okb && gc < d.n) cp_async8(dst, brow + (size_t)gc * d.ldb);
-            else *dst = 0.0;
-        }
-        return;
-    }
-    if (APAIR && !MAP && !d.ta) {
+    if (APAIR && !d.ta) {
         // op(A) = A column-major: row pairs (2p, 2p+1) of column kk, one
         // 16-byte copy where the pair is aligned in global memory, else two
 #pragma unroll
@@ -95,12 +68,11 @@ __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int 
     for (int q = 0; q < (GBM * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int r, kk;
-        if (MAP || !d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
+        if (!d.ta) { r = e & 63; kk = e >> 6; } else { kk = e & 15; r = e >> 4; }
         const int gr = r0 + r, gk = k0 + kk;
         double *dst = &sm.As[buf][kk][r];
         if (gr < d.m && gk < d.k) {
-            if (MAP) cp_async8(dst, d.A + d.rmap[gr] + (size_t)gk * d.lda);
-            else cp_async8(dst, d.ta ? d.A + gk + (size_t)gr * d.lda : d.A + gr + (size_t)gk * d.lda);
+            cp_async8(dst, d.ta ? d.A + gk + (size_t)gr * d.lda : d.A + gr + (size_t)gk * d.lda);
         } else {
             *dst = 0.0;
         }
@@ -111,45 +83,36 @@ __device__ __forceinline__ void gemm_issue_chunk(const GemmDesc &d, int r0, int 
     for (int q = 0; q < (GBN * GBK) / G_NT; ++q) {
         const int e = tid + G_NT * q;
         int c, kk;
-        if (MAP || !d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
+        if (!d.tb) { kk = e & 15; c = e >> 4; } else { c = e & 63; kk = e >> 6; }
         const int gc = c0 + c, gk = k0 + kk;
         double *dst = &sm.Bs[buf][kk][c];
         if (gc < d.n && gk < d.k) {
-            if (MAP) cp_async8(dst, d.B + d.kmap[gk] + (size_t)gc * d.ldb);
-            else cp_async8(dst, d.tb ? d.B + gc + (size_t)gk * d.ldb : d.B + gk + (size_t)gc * d.ldb);
+            cp_async8(dst, d.tb ? d.B + gc + (size_t)gk * d.ldb : d.B + gk + (size_t)gc * d.ldb);
         } else {
             *dst = 0.0;
         }
     }
 }
 
-template <bool MAP = false>
 __device__ __forceinline__ void gemm_issue_c(const GemmDesc &d, int r0, int c0, GemmSmem &sm) {
     if (d.beta == 0.0) return;
     const int tid = threadIdx.x;
     const int mr = imin(GBM, d.m - r0), nc = imin(GBN, d.n - c0);
-    if (!MAP) {
-        // row pair (2p, 2p+1) per thread: one 16-byte copy where the column's
-        // pair is 16-byte aligned in global memory (parity of r0 + c ldc), else two
-        const int p2 = 2 * (tid & 31);
-        if (p2 >= mr) return;
-        const bool two = p2 + 1 < mr;
-        for (int c = tid >> 5; c < nc; c += G_NT / 32) {
-            const double *src = d.C + r0 + p2 + (size_t)(c0 + c) * d.ldc;
-            double *dst = &sm.Cs[c][p2];
-            if (two && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
-                cp_async16(dst, src);
-            } else {
-                cp_async8(dst, src);
-                if (two) cp_async8(dst + 1, src + 1);
-            }
+    // row pair (2p, 2p+1) per thread: one 16-byte copy where the column's
+    // pair is 16-byte aligned in global memory (parity of r0 + c ldc), else two
+    const int p2 = 2 * (tid & 31);
+    if (p2 >= mr) return;
+    const bool two = p2 + 1 < mr;
+    for (int c = tid >> 5; c < nc; c += G_NT / 32) {
+        const double *src = d.C + r0 + p2 + (size_t)(c0 + c) * d.ldc;
+        double *dst = &sm.Cs[c][p2];
+        if (two && ((reinterpret_cast<uintptr_t>(src) & 15) == 0)) {
+            cp_async16(dst, src);
+        } else {
+            cp_async8(dst, src);
+            if (two) cp_async8(dst + 1, src + 1);
         }
-        return;
     }
-    const int r = tid & 63;  // fixed per thread (G_NT = 2 x 64)
-    if (r >= mr) return;
-    const double *cr = d.C + (MAP ? d.rmap[r0 + r] : r0 + r);
-    for (int c = tid >> 6; c < nc; c += G_NT / 64) cp_async8(&sm.Cs[c][r], cr + (size_t)(c0 + c) * d.ldc);
 }
 
 // ---- DFMA path: thread (tx, ty) owns rows tx + 8q (q < 8), cols ty + 16p (p < 4);
@@ -252,7 +215,7 @@ __device__ __forceinline__ void gemm_epilogue_creg(const GemmDesc &d, int r0, in
     }
 }
 
-template <bool DMMA, bool MAP = false>
+template <bool DMMA>
 __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0, const GemmSmem &sm,
                                               const double (&acc)[32]) {
     const int tid = threadIdx.x;
@@ -262,14 +225,13 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
         for (int q = 0; q < 8; ++q) {
             const int rl = tx + 8 * q, r = r0 + rl;
             if (r >= d.m) continue;
-            const int rs = MAP ? d.rmap[r] : r;
 #pragma unroll
             for (int p = 0; p < 4; ++p) {
                 const int cl = ty + 16 * p, c = c0 + cl;
                 if (c >= d.n) continue;
                 double v = d.alpha * acc[q * 4 + p];
                 if (d.beta != 0.0) v += d.beta * sm.Cs[cl][rl];
-                d.C[rs + (size_t)c * d.ldc] = v;
+                d.C[r + (size_t)c * d.ldc] = v;
             }
         }
     } else {
@@ -293,17 +255,12 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
                     v0 = fma(d.beta, cv.x, v0);
                     v1 = fma(d.beta, cv.y, v1);
                 }
-                if (MAP) {
-                    d.C[d.rmap[r] + (size_t)c * d.ldc] = v0;
-                    if (r + 1 < d.m) d.C[d.rmap[r + 1] + (size_t)c * d.ldc] = v1;
+                double *dst = d.C + r + (size_t)c * d.ldc;
+                if (r + 1 < d.m && ((reinterpret_cast<uintptr_t>(dst) & 15) == 0)) {
+                    *reinterpret_cast<double2 *>(dst) = make_double2(v0, v1);
                 } else {
-                    double *dst = d.C + r + (size_t)c * d.ldc;
-                    if (r + 1 < d.m && ((reinterpret_cast<uintptr_t>(dst) & 15) == 0)) {
-                        *reinterpret_cast<double2 *>(dst) = make_double2(v0, v1);
-                    } else {
-                        dst[0] = v0;
-                        if (r + 1 < d.m) dst[1] = v1;
-                    }
+                    dst[0] = v0;
+                    if (r + 1 < d.m) dst[1] = v1;
                 }
             }
         }
@@ -317,20 +274,20 @@ __device__ __forceinline__ void gemm_epilogue(const GemmDesc &d, int r0, int c0,
 // stream -- chunk c reads Bs[c] -- and is never loaded (the strip kernel's
 // U12, solved in place there).
 // APAIR: 16-byte row-pair copies of op(A) (off where the extra registers spill).
-template <bool DMMA, class Next, bool MAP = false, bool CREG_OK = false, bool BRES = false, bool APAIR = true>
+template <bool DMMA, class Next, bool CREG_OK = false, bool BRES = false, bool APAIR = true>
 __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
     GemmDesc d, dn;
     int r0, c0, rn, cn;
     if (!next(d, r0, c0)) return;
     int buf = 0;
-    if (d.k > 0) gemm_issue_chunk<MAP, BRES, APAIR>(d, r0, c0, 0, sm, buf);
+    if (d.k > 0) gemm_issue_chunk<BRES, APAIR>(d, r0, c0, 0, sm, buf);
     cp_async_commit();
     bool have = true;
-    constexpr bool CREG = DMMA && !MAP && CREG_OK;  // C in registers (the commit below is then an empty group)
+    constexpr bool CREG = DMMA && CREG_OK;  // C in registers (the commit below is then an empty group)
     while (have) {
         double cr[32];
         if (CREG) gemm_load_c_regs(d, r0, c0, cr);
-        else gemm_issue_c<MAP>(d, r0, c0, sm);
+        else gemm_issue_c(d, r0, c0, sm);
         cp_async_commit();
         double acc[32];
 #pragma unroll
@@ -339,10 +296,10 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         bool has_next_tile = false;
         for (int c = 0; c < (nchunks > 0 ? nchunks : 1); ++c) {
             if (c + 1 < nchunks) {
-                gemm_issue_chunk<MAP, BRES, APAIR>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
+                gemm_issue_chunk<BRES, APAIR>(d, r0, c0, (c + 1) * GBK, sm, buf ^ 1);
             } else {
                 has_next_tile = next(dn, rn, cn);
-                if (has_next_tile && dn.k > 0) gemm_issue_chunk<MAP, BRES, APAIR>(dn, rn, cn, 0, sm, buf ^ 1);
+                if (has_next_tile && dn.k > 0) gemm_issue_chunk<BRES, APAIR>(dn, rn, cn, 0, sm, buf ^ 1);
             }
             cp_async_commit();
             if (c == 0) cp_async_wait<2>(); else cp_async_wait<1>();
@@ -359,7 +316,7 @@ __device__ __forceinline__ void gemm_tile_stream(Next next, GemmSmem &sm) {
         } else {
             cp_async_wait<1>();
             __syncthreads();
-            gemm_epilogue<DMMA, MAP>(d, r0, c0, sm, acc);
+            gemm_epilogue<DMMA>(d, r0, c0, sm, acc);
             __syncthreads();
         }
         have = has_next_tile;
@@ -471,7 +428,7 @@ __global__ void __launch_bounds__(G_NT, 3) gemm_sched_kernel(Prob P, int count, 
         ++local;
         return true;
     };
-    gemm_tile_stream<DMMA, decltype(next), false, gemm_creg_ok<Prob>::value>(next, sm);
+    gemm_tile_stream<DMMA, decltype(next), gemm_creg_ok<Prob>::value>(next, sm);
 }
 
 // DCWI-grid fallback (no workspace): virtual tiles over the required dims,

@@ -58,6 +58,7 @@ struct GsArgs {
     double *const *F12; const int *ld12;
     int *const *ipiv;
     const int *info;  // fronts with info < 0 (bad arguments) are skipped
+    int upper;        // 0: stop after L^-1 (U12 of the LAPACK-style partial)
 };
 
 struct GsUnits {
@@ -317,6 +318,7 @@ __global__ void __launch_bounds__(GS_NT, 2) getrs_strip_kernel(GsArgs g, SlotLis
             // ---- 2. L^-1 (unit lower), blocks top to bottom
         for (int r0 = 0; r0 < n1; r0 += GS_BR) gs_block<true>(F11, ld11, X, ld12, n1, c0, W, r0, rg, sv);
         // ---- 3. U^-1 (non-unit upper), blocks bottom to top
+        if (!g.upper) return;
         const int last = ((n1 - 1) / GS_BR) * GS_BR;
         for (int r0 = last; r0 >= 0; r0 -= GS_BR) gs_block<false>(F11, ld11, X, ld12, n1, c0, W, r0, rg, sv);
     };
@@ -348,8 +350,8 @@ bool getrs_strip_ok(int max_n1) { return max_n1 <= GS_N1MAX; }
 
 void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *const *F11, const int *ld11,
                         double *const *F12, const int *ld12, int *const *ipiv, const int *info, int *units_off,
-                        int *queue, SlotList sl, cudaStream_t s) {
-    GsArgs g{batch, n1, n2, F11, ld11, F12, ld12, ipiv, info};
+                        int *queue, SlotList sl, cudaStream_t s, int upper) {
+    GsArgs g{batch, n1, n2, F11, ld11, F12, ld12, ipiv, info, upper};
     smem_optin(getrs_strip_kernel, GS_SMEM);
     {
         KScope k(K_GEMM_SCAN, s);

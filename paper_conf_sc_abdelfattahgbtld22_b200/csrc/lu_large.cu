@@ -427,7 +427,7 @@ __global__ void __launch_bounds__(L1_NT, 3) lu_l1_kernel(GetrfArgs a, int *__res
                     ++tt;
                     return true;
                 };
-                gemm_tile_stream<DMMA, decltype(next), false, false, false, false>(next, gsm);
+                gemm_tile_stream<DMMA, decltype(next), false, false, false>(next, gsm);
             }
             __syncthreads();
             if (phase_timing && tid == 0) { long long t1 = clock64(); atomicAdd(ph + 2, (unsigned long long)(t1 - t0)); t0 = t1; }
@@ -668,7 +668,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, int *__rest
                 if (ib < 2 * GBK)
                     for (int e = tid; e < (2 * GBK - ib) * GPAD; e += G_NT) top[ib * GPAD + e] = 0.0;
                 __syncthreads();
-                gemm_tile_stream<DMMA, decltype(next), false, false, true>(next, gsm);
+                gemm_tile_stream<DMMA, decltype(next), false, true>(next, gsm);
             } else {
                 gemm_tile_stream<DMMA>(next, gsm);
             }

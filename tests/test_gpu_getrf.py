@@ -456,3 +456,13 @@ def test_outer_strip_widths(cols):
     _run_and_check(_uniform(shapes, seed=101 + cols))
     mats = [irrgen.g1_exact(17, g, m, n)[0] for g, (m, n) in enumerate([(600, 600), (300, 700), (900, 400)])]
     _run_and_check(mats, exact=True)
+
+
+def test_outer_update_vs_oracle():
+    """The two-level outer update against the oracle on shapes with ragged
+    outer tails, wide / tall, several strips and row tiles, pivots from below
+    and from the block."""
+    irr.irr_set_tuning("l1", 0)
+    shapes = [(700, 700), (300, 1000), (1000, 300), (513, 513), (1300, 1300), (129, 900), (2048, 2048),
+              (1500, 1100), (260, 2000), (640, 129), (2000, 640)]
+    _run_and_check(_uniform(shapes, seed=303))

@@ -83,11 +83,14 @@ LAPACK_SHAPES = [(1, 1), (5, 7), (16, 3), (31, 1), (32, 40), (33, 65), (64, 200)
                  (300, 200), (3, 0), (0, 5)]
 
 
-@pytest.mark.parametrize("tier", ["default", "L"])
+@pytest.mark.parametrize("tier", ["default", "L", "unfused"])
 def test_lapack_partial_exact(tier):
     """G1'' fronts through irr_getrf_partial_lapack:
     F12 -> U12 = X, F21 -> L21 = Y, F22 -> S, F11 -> the chosen L\\U, all
-    bit-exact (the construction, no oracle needed)."""
+    bit-exact (the construction, no oracle needed).  "unfused": U12 through
+    irrLASWP + irrTRSM instead of the strip kernel stopped before U^-1."""
+    if tier == "unfused":
+        irr.irr_set_tuning("getrs_fused", 0)
     if tier == "L":
         irr.irr_set_tuning("tier_s", 0)
         irr.irr_set_tuning("tier_m_max", 0)
@@ -107,12 +110,14 @@ def test_lapack_partial_exact(tier):
         assert np.array_equal(Fg[n1:, n1:], f["S"]), (n1, F.shape)
 
 
-def test_lapack_partial_vs_oracle():
+@pytest.mark.parametrize("fused", [1, 0])
+def test_lapack_partial_vs_oracle(fused):
     """Uniform fronts against oracle.getrf_partial_lapack: ipiv / info equal
     (well-separated pivots), F11 / U12 / L21 within 1e-10 normwise-max
     relative, F22 within 1e-10 of sigma = max(|F22_in| + |L21_o| |U12_o|)."""
     from gpu_util import rel_dev
     import oracle
+    irr.irr_set_tuning("getrs_fused", fused)
     shapes = [(1, 0), (7, 0), (3, 4), (10, 10), (17, 40), (50, 80), (97, 31), (129, 257), (400, 500), (33, 700)]
     fronts = [(irrgen.front_values(88, g, n1 + n2), n1) for g, (n1, n2) in enumerate(shapes)]
     out, ipivs, info = gpu_partial(fronts, lapack=True)

@@ -1,3 +1,12 @@
-# sanitizers over every tier + the every-front C5 parity check (long)
-bash tools/gpu_runs/r2_sanitize.sh 2>&1 | tee gpurun_out/sanitizer/summary.txt
-IRR_PARITY_C5_ALL=1 timeout 3000 python -m pytest tests/test_gpu_fullconfig.py -q -s -p no:randomly -k c5 > gpurun_out/parity_c5_all.log 2>&1; echo c5all rc $?; grep "parity C5" gpurun_out/parity_c5_all.log; tail -2 gpurun_out/parity_c5_all.log
+# outer_swap_trsm3 (outer_kernel=2) + xgemm negc A/B
+export PATH=/usr/local/cuda/bin:$PATH
+timeout 900 python -m pytest tests/test_gpu_getrf.py tests/test_gpu_partial.py -q -m "gpu and not full" -p no:randomly > gpurun_out/pytest_gpu_k.log 2>&1; echo pytest rc $?; tail -3 gpurun_out/pytest_gpu_k.log; grep -E "^FAILED|^ERROR" gpurun_out/pytest_gpu_k.log | head
+run() { c=$1; shift; timeout 400 python bench.py --config $c --no-cpu-baseline --no-e2e "$@" > /tmp/b.json 2>/tmp/b.err; tail -2 /tmp/b.err
+cp /tmp/b.json gpurun_out/bench_${c}_$(echo "$*" | tr -c 'a-z0-9\n' '_').json
+python -c "import json,sys; d=json.load(open('/tmp/b.json')); print('$c $*', round(d['ms_per_step'],3), round(d['value'],1), {k:round(v,3) for k,v in d['kernel_ms_per_step'].items()}, d['roofline']['kernel'], round(d['roofline']['frac'],3))"; }
+run C3 --tune outer_kernel=2
+run C3 --tune xgemm_negc=1
+run C3 --tune outer_kernel=2 --tune xgemm_negc=1
+run C5 --steps 3 --tune outer_kernel=2 --tune xgemm_negc=1
+run C5 --steps 3 --tune xgemm_negc=1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:outer_swap_trsm3 -s 3 -c 1 -o gpurun_out/prof_outer3_C5 python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e --tune outer_kernel=2 > gpurun_out/ncu_outer3.log 2>&1; echo ncu rc $?
