@@ -288,7 +288,8 @@ int irr_extend_add(int batch, int max_n2, const int *n2, const double *const *F2
 /* ------------------------------------------------------------------------
  * Tuning (tests and experiments; defaults are fixed by measurement and are
  * process-global, not thread-safe).  Keys: "nb" (tier-L panel width, 1..64),
- * "tier_s" (1 = enable the warp-per-matrix tier), "tier_m_max" (max padded
+ * "tier_s" (1 = enable the warp-per-matrix tier, 2 = also pack 4 / 2 matrices
+ * per warp when m, n <= 8 / 16; default 2), "tier_m_max" (max padded
  * m*n of the shared-memory tier, 0 disables it), "l1" (1 = CTA-per-matrix
  * tier for m <= 256), "l1_ctas_per_sm" (1..3), "panel_rows" (max rows of a
  * grid-wide panel staged in shared memory), "trsm_nb" (TRSM recursion leaf),

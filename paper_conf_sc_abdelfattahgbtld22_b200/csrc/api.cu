@@ -42,7 +42,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
 // CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
 // rows: C3 61.7), 8-warp xgemm CTAs (16 warps: C3 58.3, C5 651 ms).
-static Tuning g_default = {32, 1, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1, 64};
+static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1, 64};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -333,7 +333,7 @@ long long irr_launch_count(int reset) {
 void irr_set_tuning(const char *key, int value) {
     if (!key) return;
     if (!strcmp(key, "nb")) g_tuning.nb = value < 1 ? 1 : (value > 64 ? 64 : value);
-    else if (!strcmp(key, "tier_s")) g_tuning.tier_s = value ? 1 : 0;
+    else if (!strcmp(key, "tier_s")) g_tuning.tier_s = value < 0 ? 0 : (value > 2 ? 2 : value);
     else if (!strcmp(key, "tier_m_max")) g_tuning.tier_m_max = value < 0 ? 0 : (value > TIER_M_MAX_DEFAULT ? TIER_M_MAX_DEFAULT : value);
     else if (!strcmp(key, "panel_rows")) g_tuning.panel_rows = value < 0 ? 0 : value;
     else if (!strcmp(key, "trsm_nb")) g_tuning.trsm_nb = value < 1 ? 1 : (value > 32 ? 32 : value);

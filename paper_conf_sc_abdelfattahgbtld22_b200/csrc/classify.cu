@@ -29,7 +29,9 @@ __global__ void __launch_bounds__(256) classify_kernel(GetrfArgs a, int *counter
         a.info[i] = e;
         if (e == 0 && mi > 0 && ni > 0) {
             const long long el = (long long)mid_lds(mi) * ni;
-            if (tier_s && mi <= 32 && ni <= 32) bin = ni <= 8 ? BIN_S8 : (ni <= 16 ? BIN_S16 : BIN_S);
+            if (tier_s >= 2 && mi <= 8 && ni <= 8) bin = BIN_S8G;  // four matrices per warp
+            else if (tier_s >= 2 && mi <= 16 && ni <= 16) bin = BIN_S16G;  // two per warp
+            else if (tier_s && mi <= 32 && ni <= 32) bin = ni <= 8 ? BIN_S8 : (ni <= 16 ? BIN_S16 : BIN_S);
             else if (el <= M1_ELEMS && el <= tier_m_max) bin = BIN_M1;
             else if (el <= M2_ELEMS && el <= tier_m_max) bin = BIN_M2;
             else if (el <= tier_m_max) bin = BIN_M3;

@@ -15,7 +15,7 @@ constexpr unsigned FULL = 0xffffffffu;
 // ---------------------------------------------------------------- tuning
 struct Tuning {
     int nb;          // tier-L panel width ("typically 16-32 columns")
-    int tier_s;      // 1: warp-per-matrix tier for m, n <= 32
+    int tier_s;      // 1: warp-per-matrix tier for m, n <= 32; 2: + several matrices per warp for m, n <= 16
     int tier_m_max;  // max padded m*n (doubles) of the shared-memory tier
     int panel_rows;  // max rows of a tier-L panel staged in shared memory
     int trsm_nb;     // TRSM recursion leaf (<= 32)
@@ -74,7 +74,9 @@ struct KScope {
 // L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
 // kernels per panel iteration.
 enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, BIN_S16 = 6, BIN_S8 = 7, BIN_L1T = 8,
-           NBINS = 9 };  // L1T: CTA-per-matrix tier, 257..l1_rows rows (tall-panel kernel variant)
+           BIN_S16G = 9, BIN_S8G = 10, NBINS = 11 };
+// L1T: CTA-per-matrix tier, 257..l1_rows rows (tall-panel kernel variant);
+// S16G / S8G: m, n <= 16 / 8, several matrices per warp (tuning tier_s = 2)
 constexpr int L1_MAX_ROWS = 256;    // panels up to this many rows are staged in shared memory
 constexpr int L1_TALL_ROWS = 1024;  // taller L1 panels: panel_win in global memory (128 threads x 8 rows)
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM
@@ -87,8 +89,9 @@ __host__ __device__ inline int mid_lds(int m) { return m | 1; }
 
 // counters block at the head of every workspace (ints)
 constexpr int CNT_INTS = 64;
-enum CounterSlot { CNT_BIN0 = 0, CNT_TILES = 8, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15, CNT_ZQ = 16, CNT_PANELQ = 17,
+enum CounterSlot { CNT_BIN0 = 48 /* NBINS ints */, CNT_MAXM = 9, CNT_MAXN = 10, CNT_L1_NEXT = 11, CNT_STRIPQ = 12, CNT_GSQ = 13, CNT_LSWQ = 14, CNT_OUTQ = 15, CNT_ZQ = 16, CNT_PANELQ = 17,
                    CNT_PHASE0 = 32 /* 8 x u64 phase-cycle accumulators (tuning phase_timing) */ };
+static_assert(CNT_BIN0 + NBINS <= CNT_INTS && CNT_PHASE0 + 16 <= CNT_BIN0, "counter slots overlap");
 
 inline size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 

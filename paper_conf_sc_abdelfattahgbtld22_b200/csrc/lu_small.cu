@@ -111,12 +111,15 @@ __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &m
     if (pos == k) pos = pmin;
     if (lane == w) pos = k;
     const bool below = valid && pos > k;
-    double l = a[0];
-    if (pv != 0.0) {
-        if (rc != 0.0) l = l * rc;
-        else l = l / pv;  // |pv| < DBL_MIN or 1/pv subnormal (LAPACK divides below sfmin)
-    } else if (info == 0) {
-        info = k + 1;  // exact zero pivot: every candidate is 0, pmin == k, no scaling
+    // common case branch-free (pv and rc are loaded together, the multiply
+    // does not wait behind a branch on pv); divide / zero pivot are the rare paths
+    double l = a[0] * rc;
+    if (rc == 0.0) {
+        if (pv != 0.0) l = a[0] / pv;  // |pv| < DBL_MIN or 1/pv subnormal (LAPACK divides below sfmin)
+        else {
+            l = a[0];
+            if (info == 0) info = k + 1;  // exact zero pivot: every candidate is 0, pmin == k, no scaling
+        }
     }
     if (below) sm.L[k * 32 + lane] = l;
     // ---- rank-1 update fused with the shift, u streamed in 16-byte loads
@@ -183,6 +186,194 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     __syncwarp();  // sm is rewritten by the next matrix
 }
 
+// ------------------------------------------------------------------ grouped
+// Matrices with m, n <= GS (GS = 8 or 16): G = 32 / GS matrices per warp, one
+// per lane group of GS lanes (lane = group * GS + row).  Same row-relabel
+// shift form as lu_warp, but every warp instruction of a step now serves G
+// matrices: the publish, the pivot-row loads, the multiplier stores and the
+// FMAs are shared; only the pivot search is per group (G high-word reduxes,
+// one ballot split by group).  The step loop runs to the largest K of the
+// warp's matrices and the width class follows their largest n; a group whose
+// matrix has no step k left sits the step out (no publish, no info, no L).
+template <int GS>
+struct __align__(16) GroupWarpSmem {
+    static constexpr int G = 32 / GS;
+    double L[GS * 32];               // L[k*32 + lane]
+    double U[G][s_ucap<GS>()];       // per group: row k of U at urow[k], W(k) slots
+    double rcp[G][2];                // per group: reciprocal of the pivot of step k in rcp[g][k & 1]
+    int urow[GS];                    // warp-uniform packed offsets
+};
+static_assert(sizeof(GroupWarpSmem<8>) % 16 == 0 && sizeof(GroupWarpSmem<16>) % 16 == 0,
+              "per-warp slots must stay 16-byte aligned");
+
+template <int GS, int W>
+__device__ __forceinline__ void g_step(double (&a)[GS], int k, int &pos, int &my_piv, int &info, bool valid,
+                                       bool act, int lane, int uo, GroupWarpSmem<GS> &sm) {
+    constexpr int G = 32 / GS;
+    const int g = lane / GS, glane = lane & (GS - 1);
+    const bool cand = valid && act && pos >= k;
+    const double myr = fast_rcp(a[0]);
+    // ---- per-group arg-max of |a[0]|: G reduxes on the high word, one ballot
+    const unsigned long long key = (unsigned long long)__double_as_longlong(fabs(a[0]));
+    const unsigned hi = cand ? (unsigned)(key >> 32) : 0u;
+    unsigned mhi = 0;
+#pragma unroll
+    for (int q = 0; q < G; ++q) {
+        const unsigned r = __reduce_max_sync(FULL, g == q ? hi : 0u);
+        if (g == q) mhi = r;
+    }
+    const bool e1 = cand && hi == mhi;
+    constexpr unsigned GM = GS == 32 ? 0xffffffffu : ((1u << GS) - 1u);
+    unsigned gm = (__ballot_sync(FULL, e1) >> (g * GS)) & GM;
+    if (__any_sync(FULL, (gm & (gm - 1)) != 0)) {  // a high-word tie in some group (rare)
+        unsigned mlo = 0;
+#pragma unroll
+        for (int q = 0; q < G; ++q) {
+            const unsigned r = __reduce_max_sync(FULL, (g == q && e1) ? (unsigned)key : 0u);
+            if (g == q) mlo = r;
+        }
+        const bool e2 = e1 && (unsigned)key == mlo;
+        unsigned pm = 0xffffffffu;
+#pragma unroll
+        for (int q = 0; q < G; ++q) {
+            const unsigned r = __reduce_min_sync(FULL, (g == q && e2) ? (unsigned)pos : 0xffffffffu);
+            if (g == q) pm = r;
+        }
+        gm = (__ballot_sync(FULL, e2 && pos == (int)pm) >> (g * GS)) & GM;
+    }
+    const int w = gm ? g * GS + __ffs(gm) - 1 : lane;  // winner lane of this group
+    const int pmin = __shfl_sync(FULL, pos, w);
+    // ---- publish the pivot rows (one lane per group)
+    double *urow = sm.U[g] + uo;
+    if (gm && lane == w) {
+#pragma unroll
+        for (int c = 0; c < W; c += 2) *reinterpret_cast<double2 *>(urow + c) = make_double2(a[c], a[c + 1]);
+        sm.rcp[g][k & 1] = myr;
+    }
+    if (lane == 0) sm.urow[k] = uo;
+    if (act && glane == k) my_piv = pmin + 1;
+    __syncwarp();
+    const double pv = urow[0];
+    const double rc = sm.rcp[g][k & 1];
+    if (act) {
+        if (pos == k) pos = pmin;
+        if (lane == w) pos = k;
+    }
+    const bool below = valid && act && pos > k;
+    double l = a[0] * rc;
+    if (rc == 0.0) {
+        if (pv != 0.0) l = a[0] / pv;
+        else {
+            l = a[0];
+            if (act && info == 0) info = k + 1;
+        }
+    }
+    if (below) sm.L[k * 32 + lane] = l;
+    constexpr int CH = W < 4 ? W : 4;
+#pragma unroll
+    for (int e0 = 0; e0 < W; e0 += CH) {
+        double uu[CH];
+#pragma unroll
+        for (int q = 0; q < CH; q += 2) {
+            const double2 v = *reinterpret_cast<const double2 *>(urow + e0 + q);
+            uu[q] = v.x;
+            uu[q + 1] = v.y;
+        }
+#pragma unroll
+        for (int q = 0; q < CH; ++q)
+            if (e0 + q >= 1) a[e0 + q - 1] = fma(-l, uu[q], a[e0 + q]);
+    }
+    a[W - 1] = 0.0;
+    (void)glane;
+}
+
+template <int GS>
+constexpr int group_ctas() { return GS == 8 ? 8 : 6; }  // 64 / 80 registers
+
+template <int GS>
+__global__ void __launch_bounds__(32 * S_WARPS, group_ctas<GS>()) lu_group_kernel(GetrfArgs a,
+                                                                             const int *__restrict__ counters,
+                                                                             const int *__restrict__ bins, int bin) {
+    constexpr int G = 32 / GS;
+    extern __shared__ __align__(16) double s_small[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int g = lane / GS, glane = lane & (GS - 1);
+    GroupWarpSmem<GS> &sm = reinterpret_cast<GroupWarpSmem<GS> *>(s_small)[warp];
+    const int count = counters[CNT_BIN0 + bin];
+    const int *list = bins + (size_t)bin * a.batch;
+    const int items = (count + G - 1) / G;
+    const int stride = gridDim.x * S_WARPS;
+    for (int t = blockIdx.x * S_WARPS + warp; t < items; t += stride) {
+        const int slot = t * G + g;
+        int m = 0, n = 0, ld = 1, i = -1;
+        if (slot < count) {
+            i = list[slot];
+            m = a.m[i];
+            n = a.n[i];
+            ld = a.ld[i];
+        }
+        // next item of this warp into L2, one lane group per matrix
+        const int sn = (t + stride) * G + g;
+        if (t + stride < items && sn < count) {
+            const int i2 = list[sn];
+            const char *p2 = reinterpret_cast<const char *>(a.A[i2]);
+            const long bytes = ((long)(a.n[i2] - 1) * a.ld[i2] + a.m[i2]) * 8;
+            for (long o = (long)glane * 128; o < bytes; o += GS * 128)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(p2 + o));
+        }
+        const bool valid = glane < m;
+        double a_[GS];
+        {
+            const double *gr = i >= 0 ? a.A[i] + glane : nullptr;
+#pragma unroll
+            for (int c = 0; c < GS; ++c) {
+                a_[c] = (valid && c < n) ? gr[(size_t)c * ld] : 0.0;
+            }
+        }
+        const int K = m < n ? m : n;
+        const int Kmax = (int)__reduce_max_sync(FULL, (unsigned)K);
+        const int nmax = (int)__reduce_max_sync(FULL, (unsigned)n);
+        int pos = glane, my_piv = 0, info = 0, k = 0, uo = 0;
+        if (GS >= 16) {
+            for (; k < Kmax && nmax - k > 12; ++k, uo += 16)
+                g_step<GS, 16>(a_, k, pos, my_piv, info, valid, k < K, lane, uo, sm);
+            for (; k < Kmax && nmax - k > 8; ++k, uo += 12)
+                g_step<GS, 12>(a_, k, pos, my_piv, info, valid, k < K, lane, uo, sm);
+        }
+        for (; k < Kmax && nmax - k > 4; ++k, uo += 8) g_step<GS, 8>(a_, k, pos, my_piv, info, valid, k < K, lane, uo, sm);
+        for (; k < Kmax; ++k, uo += 4) g_step<GS, 4>(a_, k, pos, my_piv, info, valid, k < K, lane, uo, sm);
+        __syncwarp();
+        if (valid) {
+            double *go = a.A[i] + pos;
+            const double *ur = sm.U[g] + sm.urow[pos < K ? pos : 0] - pos;
+            for (int c = 0; c < n; ++c) {
+                double v;
+                if (c < pos) v = sm.L[c * 32 + lane];
+                else v = ur[c];
+                go[(size_t)c * ld] = v;
+            }
+        }
+        if (i >= 0) {
+            if (glane < K) a.ipiv[i][glane] = my_piv;
+            if (glane == 0) a.info[i] = info;
+        }
+        __syncwarp();
+    }
+}
+
+template <int GS>
+static void launch_group(const GetrfArgs &a, const int *counters, const int *bins, int bin, cudaStream_t s) {
+    const size_t smem = (size_t)S_WARPS * sizeof(GroupWarpSmem<GS>);
+    smem_optin(lu_group_kernel<GS>, smem);
+    constexpr int G = 32 / GS;
+    int grid = num_sms() * group_ctas<GS>();
+    int need = (a.batch + S_WARPS * G - 1) / (S_WARPS * G);
+    if (grid > need) grid = need;
+    if (grid < 1) grid = 1;
+    KScope k(K_LU_SMALL, s);
+    lu_group_kernel<GS><<<grid, 32 * S_WARPS, smem, s>>>(a, counters, bins, bin);
+}
+
 // Each warp walks its share of the width class's list (static stride); the
 // next matrix of the warp is prefetched into L2 before the current one is
 // loaded.
@@ -228,10 +419,17 @@ static void launch_class(const GetrfArgs &a, const int *counters, const int *bin
 // widest class first: it has the most work per matrix, the narrow kernels
 // fill in behind it
 void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
-    launch_class<32>(a, counters, bins, s);
+    const bool grouped = tuning().tier_s >= 2;
+    if (a.max_n > 16 || a.max_m > 16 || !grouped) launch_class<32>(a, counters, bins, s);
     if (a.max_n > 0) {
-        launch_class<16>(a, counters, bins, s);
-        launch_class<8>(a, counters, bins, s);
+        if (a.max_m > 16 || !grouped) {
+            launch_class<16>(a, counters, bins, s);
+            launch_class<8>(a, counters, bins, s);
+        }
+        if (grouped) {
+            if (a.max_m > 8 || a.max_n > 8) launch_group<16>(a, counters, bins, BIN_S16G, s);
+            launch_group<8>(a, counters, bins, BIN_S8G, s);
+        }
     }
 }
 

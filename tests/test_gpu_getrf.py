@@ -466,3 +466,33 @@ def test_outer_update_vs_oracle():
     shapes = [(700, 700), (300, 1000), (1000, 300), (513, 513), (1300, 1300), (129, 900), (2048, 2048),
               (1500, 1100), (260, 2000), (640, 129), (2000, 640)]
     _run_and_check(_uniform(shapes, seed=303))
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_grouped_tier_s_bitwise_and_oracle(seed):
+    """tier_s = 2 packs 4 (m, n <= 8) or 2 (m, n <= 16) matrices per warp.
+    Each row sees the same FMA sequence as the warp-per-matrix kernel
+    (tier_s = 1): results bitwise identical, and every matrix matches the
+    oracle.  Mixed shapes so a warp's matrices differ in K and n (groups that
+    sit steps out), rectangular both ways, tall n <= 8 with m > 16 (stays on
+    the warp-per-matrix kernels), and a batch that is not a multiple of the
+    group count."""
+    rng = np.random.default_rng(seed)
+    shapes = [(int(rng.integers(1, 9)), int(rng.integers(1, 9))) for _ in range(203)]
+    shapes += [(int(rng.integers(1, 17)), int(rng.integers(1, 17))) for _ in range(151)]
+    shapes += [(int(rng.integers(17, 33)), int(rng.integers(1, 9))) for _ in range(23)]
+    shapes += [(m, n) for m in (1, 2, 7, 8, 9, 15, 16) for n in (1, 2, 7, 8, 9, 15, 16)]
+    mats = _uniform(shapes, seed=100 + seed)
+    sing = [irrgen.g1_singular(5, g, 8, 8, c)[0] for g, c in enumerate((0, 3, 7))]
+    sing += [irrgen.g1_singular(6, g, 16, 16, c)[0] for g, c in enumerate((1, 12, 15))]
+    mats += sing
+    irr.irr_set_tuning("tier_s", 2)
+    LU2, ip2, info2, _ = gpu_getrf(mats)
+    irr.irr_set_tuning("tier_s", 1)
+    LU1, ip1, info1, _ = gpu_getrf(mats)
+    assert np.array_equal(info1, info2)
+    for a, b, p, q in zip(LU1, LU2, ip1, ip2):
+        assert np.array_equal(p, q)
+        assert np.array_equal(a.view(np.int64), b.view(np.int64))
+    for g, (A, LU, ip, inf) in enumerate(zip(mats, LU2, ip2, info2)):
+        check_getrf(A, LU, ip, int(inf), exact=g >= len(mats) - len(sing), label=f"grouped #{g} {A.shape}")
