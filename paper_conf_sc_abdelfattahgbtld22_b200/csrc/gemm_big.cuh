@@ -208,13 +208,9 @@ __device__ __forceinline__ void xgemm_prefetch_c(const GemmDesc &d, int r0, int 
     }
 }
 
-// One tile: the whole K loop through the 4-deep ring, then the epilogue.
-template <int TA, int TB, int NWG = 8>
-__device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, BigSmem &sm) {
-    constexpr int NT = 32 * NWG, ACC = XWarp<NWG>::ACC;
-    double acc[ACC];
-#pragma unroll
-    for (int q = 0; q < ACC; ++q) acc[q] = 0.0;
+// Ring prologue of a tile: its C tile towards L2 and its first XST-1 K chunks.
+template <int TA, int TB, int NT>
+__device__ __forceinline__ void xgemm_prologue(const GemmDesc &d, int r0, int c0, BigSmem &sm) {
     const int nk = (d.k + XBK - 1) / XBK;
     xgemm_prefetch_c<NT>(d, r0, c0);
 #pragma unroll
@@ -222,6 +218,17 @@ __device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, Bi
         if (s < nk) xgemm_issue<TA, TB, NT>(d, r0, c0, s * XBK, sm, s);
         cp_async_commit();
     }
+}
+
+// The K loop of a tile whose prologue has been issued.  Ends with the ring
+// free (every chunk consumed, barrier passed), the product in acc.
+template <int TA, int TB, int NWG = 8>
+__device__ __forceinline__ void xgemm_main(const GemmDesc &d, int r0, int c0, BigSmem &sm,
+                                           double (&acc)[XWarp<NWG>::ACC]) {
+    constexpr int NT = 32 * NWG, ACC = XWarp<NWG>::ACC;
+#pragma unroll
+    for (int q = 0; q < ACC; ++q) acc[q] = 0.0;
+    const int nk = (d.k + XBK - 1) / XBK;
     for (int kc = 0; kc < nk; ++kc) {
         cp_async_wait<XST - 2>();
         __syncthreads();
@@ -232,6 +239,14 @@ __device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, Bi
     }
     cp_async_wait<0>();
     __syncthreads();  // the ring is refilled by the next tile's prologue
+}
+
+// One tile: prologue, K loop, epilogue (no overlap with a next tile).
+template <int TA, int TB, int NWG = 8>
+__device__ __forceinline__ void xgemm_tile(const GemmDesc &d, int r0, int c0, BigSmem &sm) {
+    double acc[XWarp<NWG>::ACC];
+    xgemm_prologue<TA, TB, 32 * NWG>(d, r0, c0, sm);
+    xgemm_main<TA, TB, NWG>(d, r0, c0, sm, acc);
     xgemm_epilogue<NWG>(d, r0, c0, acc);
 }
 
@@ -309,20 +324,40 @@ __global__ void __launch_bounds__(32 * NWG, XGEMM_MINB) xgemm_sched_kernel(Prob 
     int w = xgemm_tile_weight(cur), off_b = tile_off[b];
     int nt_b = (tile_off[b + 1] - off_b) / w;
     int local = u_begin > off_b ? (u_begin - off_b + w - 1) / w : 0;
-    while (true) {
+    // next tile of this CTA's share (false: done)
+    auto advance = [&]() -> bool {
         while (local >= nt_b) {
-            if (++b >= count) return;
+            if (++b >= count) return false;
             off_b = tile_off[b];
-            if (off_b >= u_end) return;
+            if (off_b >= u_end) return false;
             P.get(b, cur);
             w = xgemm_tile_weight(cur);
             nt_b = (tile_off[b + 1] - off_b) / w;
             local = 0;
         }
-        if (off_b + local * w >= u_end) return;
-        const int ntm = (cur.m + XBM - 1) / XBM;
-        xgemm_tile<TA, TB, NWG>(cur, (local % ntm) * XBM, (local / ntm) * XBN, sm);
+        return off_b + local * w < u_end;
+    };
+    if (!advance()) return;
+    int ntm = (cur.m + XBM - 1) / XBM;
+    int r0 = (local % ntm) * XBM, c0 = (local / ntm) * XBN;
+    xgemm_prologue<TA, TB, 32 * NWG>(cur, r0, c0, sm);
+    double acc[XWarp<NWG>::ACC];
+    while (true) {
+        xgemm_main<TA, TB, NWG>(cur, r0, c0, sm, acc);
+        // the next tile's C prefetch and first K chunks go out before this
+        // tile's epilogue, so their latency hides behind it
+        const GemmDesc done = cur;
+        const int dr0 = r0, dc0 = c0;
         ++local;
+        const bool more = advance();
+        if (more) {
+            ntm = (cur.m + XBM - 1) / XBM;
+            r0 = (local % ntm) * XBM;
+            c0 = (local / ntm) * XBN;
+            xgemm_prologue<TA, TB, 32 * NWG>(cur, r0, c0, sm);
+        }
+        xgemm_epilogue<NWG>(done, dr0, dc0, acc);
+        if (!more) return;
     }
 }
 

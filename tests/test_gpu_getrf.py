@@ -481,18 +481,23 @@ def test_grouped_tier_s_bitwise_and_oracle(seed):
     shapes = [(int(rng.integers(1, 9)), int(rng.integers(1, 9))) for _ in range(203)]
     shapes += [(int(rng.integers(1, 17)), int(rng.integers(1, 17))) for _ in range(151)]
     shapes += [(int(rng.integers(17, 33)), int(rng.integers(1, 9))) for _ in range(23)]
+    shapes += [(int(rng.integers(1, 33)), int(rng.integers(17, 33))) for _ in range(97)]
+    shapes += [(int(rng.integers(17, 33)), int(rng.integers(1, 33))) for _ in range(61)]
     shapes += [(m, n) for m in (1, 2, 7, 8, 9, 15, 16) for n in (1, 2, 7, 8, 9, 15, 16)]
     mats = _uniform(shapes, seed=100 + seed)
     sing = [irrgen.g1_singular(5, g, 8, 8, c)[0] for g, c in enumerate((0, 3, 7))]
     sing += [irrgen.g1_singular(6, g, 16, 16, c)[0] for g, c in enumerate((1, 12, 15))]
+    sing += [irrgen.g1_singular(7, g, 32, 32, c)[0] for g, c in enumerate((0, 16, 31))]
+    sing += [irrgen.g1_exact(8, g, m, n)[0] for g, (m, n) in enumerate(((32, 32), (17, 32), (32, 17), (31, 25)))]
     mats += sing
-    irr.irr_set_tuning("tier_s", 2)
-    LU2, ip2, info2, _ = gpu_getrf(mats)
     irr.irr_set_tuning("tier_s", 1)
     LU1, ip1, info1, _ = gpu_getrf(mats)
-    assert np.array_equal(info1, info2)
-    for a, b, p, q in zip(LU1, LU2, ip1, ip2):
-        assert np.array_equal(p, q)
-        assert np.array_equal(a.view(np.int64), b.view(np.int64))
+    for ts in (2,):
+        irr.irr_set_tuning("tier_s", ts)
+        LU2, ip2, info2, _ = gpu_getrf(mats)
+        assert np.array_equal(info1, info2), ts
+        for a, b, p, q in zip(LU1, LU2, ip1, ip2):
+            assert np.array_equal(p, q), ts
+            assert np.array_equal(a.view(np.int64), b.view(np.int64)), ts
     for g, (A, LU, ip, inf) in enumerate(zip(mats, LU2, ip2, info2)):
         check_getrf(A, LU, ip, int(inf), exact=g >= len(mats) - len(sing), label=f"grouped #{g} {A.shape}")
