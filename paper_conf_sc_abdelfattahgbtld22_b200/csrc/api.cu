@@ -41,8 +41,9 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // left-block interchanges (6.80 -> 6.53 ms), two-level grid tier with outer
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
 // CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
-// rows: C3 61.7), 8-warp xgemm CTAs (16 warps: C3 58.3, C5 651 ms).
-static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 8, 1, 1, 64};
+// rows: C3 61.7), warp-specialised xgemm (8 DMMA warps + a producer warpgroup on an
+// mbarrier ring: C5 616 -> 572 ms, C3 54.8 -> 52.0, C4 91.8 -> 87.0; 16 warps: C3 58.3, C5 651 ms).
+static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -351,7 +352,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "l1_rows")) g_tuning.l1_rows = value < 1 ? 1 : (value > L1_TALL_ROWS ? L1_TALL_ROWS : value);
     else if (!strcmp(key, "defer") || !strcmp(key, "l1_defer")) g_tuning.defer = value ? 1 : 0;
     else if (!strcmp(key, "nb_outer")) g_tuning.nb_outer = value < 0 ? 0 : (value > NB_OUTER_MAX ? NB_OUTER_MAX : value);
-    else if (!strcmp(key, "xgemm_warps")) g_tuning.xgemm_warps = value >= 16 ? 16 : 8;
+    else if (!strcmp(key, "xgemm_warps")) g_tuning.xgemm_warps = value >= 16 ? 16 : (value == 9 ? 9 : 8);
     else if (!strcmp(key, "parts")) g_tuning.parts = value >= 2 ? 2 : 1;
     else if (!strcmp(key, "part_grid")) g_tuning.part_grid = value >= 2 ? 2 : 1;
     else if (!strcmp(key, "outer_cols")) g_tuning.outer_cols = value <= 32 ? 32 : 64;

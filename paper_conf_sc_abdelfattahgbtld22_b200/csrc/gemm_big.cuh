@@ -67,8 +67,9 @@ __device__ __forceinline__ void x_pair(double *dst, const double *src, bool ok0,
 // A^T, k for B, n for B^T): both shared layouts keep such pairs 16-byte
 // aligned (even leading dimensions 132 / 20).
 template <int TA, int TB, int NT = X_NT>
-__device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st) {
-    const int tid = threadIdx.x;
+__device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st,
+                                            int tid = -1) {
+    if (tid < 0) tid = threadIdx.x;
     double *As = sm.A[st];
     double *Bs = sm.B[st];
 #pragma unroll
@@ -361,6 +362,136 @@ __global__ void __launch_bounds__(32 * NWG, XGEMM_MINB) xgemm_sched_kernel(Prob 
     }
 }
 
+// ---------------------------------------------------------------------------
+// Warp-specialised variant (tuning xgemm_ws = 1): the 8 DMMA warps never wait
+// at a CTA barrier.  A 9th warp is the producer: it fills the 4-stage ring
+// with cp.async and signals each stage's mbarrier (cp.async.mbarrier.arrive:
+// the arrival fires when the copies have landed); the DMMA warps wait on the
+// stage's `full` barrier, compute, and release it through its `empty`
+// barrier (one arrival per warp).  The producer runs up to 4 chunks ahead,
+// across tile boundaries, so the next tile's operands stream in while the
+// DMMA warps run this tile's epilogue.  384 threads = 3 warpgroups launched
+// at 168 registers (64,512 for the CTA); setmaxnreg moves registers from the
+// producer group (56) to the DMMA groups (216) inside that allocation:
+// 128 x 56 + 256 x 216 = 62,464 (an increase beyond the CTA's launch
+// allocation never completes).  9 warps at 224 cannot launch at all: 3 warps
+// of one SM sub-partition would need 21,504 of its 16,384 registers.
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned long long *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cp_async(unsigned long long *bar) {
+    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "XW_WAIT%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        " @!p bra XW_WAIT%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+constexpr int XWS_NT = 384;  // 8 DMMA warps + a producer warpgroup
+
+template <class Prob, int TA, int TB>
+__global__ void __launch_bounds__(XWS_NT, 1) xgemm_ws_kernel(Prob P, int count, const int *count_ptr,
+                                                         const int *__restrict__ tile_off) {
+    extern __shared__ __align__(16) unsigned char x_smem[];
+    BigSmem &sm = *reinterpret_cast<BigSmem *>(x_smem);
+    __shared__ __align__(8) unsigned long long full_b[XST], empty_b[XST];
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < XST; ++s) {
+            mbar_init(&full_b[s], 128);  // the producer threads (cp.async arrivals)
+            mbar_init(&empty_b[s], 8);  // one arrival per DMMA warp
+        }
+    }
+    __syncthreads();
+    if (count < 0) count = *count_ptr;
+    if (count <= 0) return;
+    const int total = tile_off[count];
+    const long long G = gridDim.x;
+    const int u_begin = (int)((long long)blockIdx.x * total / G);
+    const int u_end = (int)((long long)(blockIdx.x + 1) * total / G);
+    if (u_begin >= u_end) return;
+    int lo = 0, hi = count - 1;
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (tile_off[mid] <= u_begin) lo = mid; else hi = mid - 1;
+    }
+    int b = lo;
+    GemmDesc cur;
+    P.get(b, cur);
+    int w = xgemm_tile_weight(cur), off_b = tile_off[b];
+    int nt_b = (tile_off[b + 1] - off_b) / w;
+    int local = u_begin > off_b ? (u_begin - off_b + w - 1) / w : 0;
+    auto advance = [&]() -> bool {
+        while (local >= nt_b) {
+            if (++b >= count) return false;
+            off_b = tile_off[b];
+            if (off_b >= u_end) return false;
+            P.get(b, cur);
+            w = xgemm_tile_weight(cur);
+            nt_b = (tile_off[b + 1] - off_b) / w;
+            local = 0;
+        }
+        return off_b + local * w < u_end;
+    };
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned q = 0;  // chunk counter over this CTA's tiles: stage q % XST, phase (q / XST) & 1
+    if (warp >= 8) {
+        // ---- producer warpgroup
+        asm volatile("setmaxnreg.dec.sync.aligned.u32 56;\n" ::: "memory");
+        const int ptid = threadIdx.x - 256;
+        while (advance()) {
+            const int ntm = (cur.m + XBM - 1) / XBM;
+            const int r0 = (local % ntm) * XBM, c0 = (local / ntm) * XBN;
+            if (cur.beta != 0.0) {  // C tile towards L2 (4 columns x 8 lines per lane)
+                for (int c = ptid; c < XBN; c += 128) {
+                    if (c0 + c >= cur.n) break;
+                    for (int r = 0; r < XBM; r += 16)
+                        if (r0 + r < cur.m)
+                            asm volatile("prefetch.global.L2 [%0];" ::"l"(cur.C + r0 + r + (size_t)(c0 + c) * cur.ldc));
+                }
+            }
+            const int nk = (cur.k + XBK - 1) / XBK;
+            for (int kc = 0; kc < nk; ++kc, ++q) {
+                const int st = q % XST;
+                mbar_wait(&empty_b[st], ((q / XST) & 1) ^ 1);
+                xgemm_issue<TA, TB, 128>(cur, r0, c0, kc * XBK, sm, st, ptid);
+                mbar_arrive_cp_async(&full_b[st]);
+            }
+            ++local;
+        }
+        asm volatile("cp.async.wait_all;\n" ::: "memory");
+        return;
+    }
+    // ---- DMMA warps
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 216;\n" ::: "memory");
+    double acc[XWarp<8>::ACC];
+    while (advance()) {
+        const int ntm = (cur.m + XBM - 1) / XBM;
+        const int r0 = (local % ntm) * XBM, c0 = (local / ntm) * XBN;
+#pragma unroll
+        for (int i = 0; i < XWarp<8>::ACC; ++i) acc[i] = 0.0;
+        const int nk = (cur.k + XBK - 1) / XBK;
+        for (int kc = 0; kc < nk; ++kc, ++q) {
+            const int st = q % XST;
+            mbar_wait(&full_b[st], (q / XST) & 1);
+            xgemm_compute<TA, TB, 8>(sm, st, acc);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty_b[st]);
+        }
+        xgemm_epilogue<8>(cur, r0, c0, acc);
+        ++local;
+    }
+}
+
 // Wraps a problem and keeps only the slots one of the two cores should run:
 // the big core takes products whose tile would be mostly full and whose K
 // amortises the pipeline fill.
@@ -378,6 +509,11 @@ struct SizeFilter {
 
 template <class Prob, int TA, int TB>
 inline void xgemm_launch_t(const Prob &P, int cnt, const int *cnt_ptr, const int *tile_off, cudaStream_t s) {
+    if (tuning().xgemm_warps == 9) {
+        smem_optin(xgemm_ws_kernel<Prob, TA, TB>, BIG_SMEM);
+        xgemm_ws_kernel<Prob, TA, TB><<<num_sms(), XWS_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+        return;
+    }
     smem_optin(xgemm_sched_kernel<Prob, TA, TB>, BIG_SMEM);
     xgemm_sched_kernel<Prob, TA, TB><<<num_sms() * XGEMM_MINB, X_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
 }

@@ -34,7 +34,7 @@ struct Tuning {
     int defer;           // 1: left-block interchanges applied once at the end, coalesced (L1 and grid tiers)
     int getrs_vec;       // 1: irr_getrs with max_nrhs <= 4 by the CTA-per-system kernel (getrs_vec.cu)
     int nb_outer;        // grid-wide tier: outer block width of the two-level blocking (0 / <= nb: one level)
-    int xgemm_warps;     // 8 or 16 warps per 128 x 128 DMMA tile CTA (the two-level trailing GEMM)
+    int xgemm_warps;     // 8 or 16 warps per 128 x 128 DMMA tile CTA, or 9 = 8 DMMA warps + 1 producer warp (mbarrier ring)
     int parts;           // two-level grid tier: 1, or 2 halves of the LPT list on two streams
     int part_grid;       // with 2 parts: 1 = full grids per part, 2 = half grids
     int outer_cols;      // two-level interchange + U12 solve strip width: 64 (L11 square, 1 CTA/SM) or 32 (packed, 2/SM)

@@ -1199,6 +1199,7 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
         const bool os32 = tu.outer_cols == 32;
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 8>, BIG_SMEM);
         smem_optin(xgemm_sched_kernel<OuterTrailProb, 0, 0, 16>, BIG_SMEM);
+        smem_optin(xgemm_ws_kernel<OuterTrailProb, 0, 0>, BIG_SMEM);
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
         // one part = one list of tier-L slots with its own counters block
         // (count, queues), plan slots, tile offsets and stream
@@ -1247,7 +1248,9 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
                     xgemm_scan_kernel<OuterTrailProb><<<1, 1024, 0, st>>>(P, -1, cnt_ptr, toff);
                 }
                 KScope k(K_GEMM_TRAIL, st);
-                if (tu.xgemm_warps == 16)
+                if (tu.xgemm_warps == 9)
+                    xgemm_ws_kernel<OuterTrailProb, 0, 0><<<gs, XWS_NT, BIG_SMEM, st>>>(P, -1, cnt_ptr, toff);
+                else if (tu.xgemm_warps == 16)
                     xgemm_sched_kernel<OuterTrailProb, 0, 0, 16><<<gs * XGEMM_MINB, 512, BIG_SMEM, st>>>(P, -1, cnt_ptr,
                                                                                                      toff);
                 else

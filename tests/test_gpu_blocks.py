@@ -17,6 +17,12 @@ from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200.batch import MatrixBatch  # noqa: E402
 
 
+@pytest.fixture(autouse=True)
+def _reset_tuning():
+    yield
+    irr.irr_reset_tuning()
+
+
 def _upload(mats):
     B = MatrixBatch([a.shape[0] for a in mats], [a.shape[1] for a in mats], with_ipiv=False)
     host = np.zeros(B.total)
@@ -68,11 +74,14 @@ def test_gemm_dcwi_exact(ta, tb, use_work):
         assert np.array_equal(got[i], exp), i
 
 
+@pytest.mark.parametrize("warps", [8, 9])
 @pytest.mark.parametrize("ta,tb", list(itertools.product((0, 1), (0, 1))))
-def test_gemm_big_core_exact(ta, tb):
+def test_gemm_big_core_exact(ta, tb, warps):
     """Products large enough for the 128 x 128 DMMA core (several tiles, ragged
     edges, K not a multiple of the 16-chunk) mixed with small ones that stay
-    on the 64 x 64 core; integer data, so every entry is exact."""
+    on the 64 x 64 core; integer data, so every entry is exact.  warps = 9:
+    the warp-specialised core (producer warp + mbarrier ring)."""
+    irr.irr_set_tuning("xgemm_warps", warps)
     rng = np.random.default_rng(100 + ta * 2 + tb)
     m = np.array([300, 97, 5, 260, 130, 64]); n = np.array([257, 140, 200, 96, 7, 64])
     k = np.array([201, 48, 300, 77, 130, 40])

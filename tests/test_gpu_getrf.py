@@ -501,3 +501,21 @@ def test_grouped_tier_s_bitwise_and_oracle(seed):
             assert np.array_equal(a.view(np.int64), b.view(np.int64)), ts
     for g, (A, LU, ip, inf) in enumerate(zip(mats, LU2, ip2, info2)):
         check_getrf(A, LU, ip, int(inf), exact=g >= len(mats) - len(sing), label=f"grouped #{g} {A.shape}")
+
+
+@pytest.mark.parametrize("warps", [8, 16])
+def test_xgemm_variants_bitwise_equal(warps):
+    """The two-level trailing GEMM on the 8-warp or the 16-warp core gives
+    bitwise the factors of the default warp-specialised core (9: 8 DMMA warps
+    + a producer warpgroup on an mbarrier ring; same DMMA sequence per
+    accumulator), and matches the oracle."""
+    irr.irr_set_tuning("l1", 0)
+    shapes = [(700, 700), (300, 1000), (1000, 300), (1300, 1300), (2048, 2048), (129, 900), (2000, 640)]
+    mats = _uniform(shapes, seed=404)
+    one, ip1, inf1, _ = gpu_getrf(mats)
+    irr.irr_set_tuning("xgemm_warps", warps)
+    two, ip2, inf2, _ = gpu_getrf(mats)
+    for a, b, p, q in zip(one, two, ip1, ip2):
+        assert np.array_equal(a.view(np.int64), b.view(np.int64)) and np.array_equal(p, q)
+    assert np.array_equal(inf1, inf2)
+    _run_and_check(mats)
