@@ -31,7 +31,8 @@ __global__ void __launch_bounds__(256) classify_kernel(GetrfArgs a, int *counter
             const long long el = (long long)mid_lds(mi) * ni;
             if (tier_s >= 2 && mi <= 8 && ni <= 8) bin = BIN_S8G;  // four matrices per warp
             else if (tier_s >= 2 && mi <= 16 && ni <= 16) bin = BIN_S16G;  // two per warp
-            else if (tier_s && mi <= 32 && ni <= 32) bin = ni <= 8 ? BIN_S8 : (ni <= 16 ? BIN_S16 : BIN_S);
+            else if (tier_s && mi <= 32 && ni <= 32)
+                bin = ni <= 8 ? BIN_S8 : (ni <= 16 ? BIN_S16 : ((tier_s >= 2 && ni <= 24) ? BIN_S24 : BIN_S));
             else if (el <= M1_ELEMS && el <= tier_m_max) bin = BIN_M1;
             else if (el <= M2_ELEMS && el <= tier_m_max) bin = BIN_M2;
             else if (el <= tier_m_max) bin = BIN_M3;
@@ -39,17 +40,14 @@ __global__ void __launch_bounds__(256) classify_kernel(GetrfArgs a, int *counter
             else bin = BIN_L;
         }
     }
-    // warp-aggregated append to the bin lists (one atomic per warp and bin)
-#pragma unroll
-    for (int b = 0; b < NBINS; ++b) {
-        unsigned mask = __ballot_sync(FULL, bin == b);
-        if (!mask) continue;
-        int leader = __ffs(mask) - 1;
-        int base = 0;
-        if (lane == leader) base = atomicAdd(&counters[CNT_BIN0 + b], __popc(mask));
-        base = __shfl_sync(FULL, base, leader);
-        if (bin == b) bins[(size_t)b * a.batch + base + __popc(mask & ((1u << lane) - 1))] = i;
-    }
+    // warp-aggregated append to the bin lists: lanes of equal bin found with
+    // one match, one atomic per distinct bin of the warp (leader lane)
+    const unsigned mask = __match_any_sync(FULL, bin);
+    const int leader = __ffs(mask) - 1;
+    int base = 0;
+    if (lane == leader && bin >= 0) base = atomicAdd(&counters[CNT_BIN0 + bin], __popc(mask));
+    base = __shfl_sync(FULL, base, leader);
+    if (bin >= 0) bins[(size_t)bin * a.batch + base + __popc(mask & ((1u << lane) - 1))] = i;
 }
 
 void launch_classify(const GetrfArgs &a, int *counters, int *bins, int keep_neg_info, cudaStream_t s) {

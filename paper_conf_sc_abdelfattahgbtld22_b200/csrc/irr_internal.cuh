@@ -74,9 +74,10 @@ struct KScope {
 // L1 = tier L with m <= L1_MAX_ROWS, one CTA per matrix; L = the rest, grid-wide
 // kernels per panel iteration.
 enum Bin { BIN_S = 0, BIN_M1 = 1, BIN_M2 = 2, BIN_M3 = 3, BIN_L = 4, BIN_L1 = 5, BIN_S16 = 6, BIN_S8 = 7, BIN_L1T = 8,
-           BIN_S16G = 9, BIN_S8G = 10, NBINS = 11 };
+           BIN_S16G = 9, BIN_S8G = 10, BIN_S24 = 11, NBINS = 12 };
 // L1T: CTA-per-matrix tier, 257..l1_rows rows (tall-panel kernel variant);
-// S16G / S8G: m, n <= 16 / 8, several matrices per warp (tuning tier_s = 2)
+// S16G / S8G: m, n <= 16 / 8, several matrices per warp; S24: m <= 32, 16 < n <= 24
+// on its own register budget (tuning tier_s = 2)
 constexpr int L1_MAX_ROWS = 256;    // panels up to this many rows are staged in shared memory
 constexpr int L1_TALL_ROWS = 1024;  // taller L1 panels: panel_win in global memory (128 threads x 8 rows)
 constexpr int M1_ELEMS = 6144;    // 48 KB  -> 4 CTAs / SM

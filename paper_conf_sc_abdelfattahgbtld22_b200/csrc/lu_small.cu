@@ -40,6 +40,11 @@ template <int NC>
 struct SmallCfg;
 template <>
 struct SmallCfg<32> { static constexpr int ctas = 4, bin = BIN_S; };    // 128 regs, 16 warps / SM
+#ifndef IRR_S24_CTAS
+#define IRR_S24_CTAS 5
+#endif
+template <>
+struct SmallCfg<24> { static constexpr int ctas = IRR_S24_CTAS, bin = BIN_S24; };  // 96 regs, 20 warps / SM (tier_s = 2)
 template <>
 struct SmallCfg<16> { static constexpr int ctas = 6, bin = BIN_S16; };  // 80 regs, 24 warps / SM
 template <>
@@ -51,7 +56,7 @@ struct SmallCfg<8> { static constexpr int ctas = 8, bin = BIN_S8; };    // 64 re
 // touches another row's slots.  Capacity = the widths summed at n = NC.
 template <int NC>
 __host__ __device__ constexpr int s_width(int rem) {
-    return (NC >= 32 && rem > 24) ? 32 : (NC >= 32 && rem > 16) ? 24 : (NC >= 16 && rem > 12) ? 16
+    return (NC >= 32 && rem > 24) ? 32 : (NC >= 24 && rem > 16) ? 24 : (NC >= 16 && rem > 12) ? 16
          : (NC >= 16 && rem > 8) ? 12 : (rem > 4) ? (NC >= 8 ? 8 : NC) : 4;
 }
 template <int NC>
@@ -68,10 +73,11 @@ struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 s
     double rcp[2];                 // reciprocal of the pivot of step k in rcp[k & 1] (0: divide)
     int urow[NC];                  // offset of U row k
 };
-static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<16>) % 16 == 0 &&
-                  sizeof(SmallWarpSmem<8>) % 16 == 0,
+static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<24>) % 16 == 0 &&
+                  sizeof(SmallWarpSmem<16>) % 16 == 0 && sizeof(SmallWarpSmem<8>) % 16 == 0,
               "per-warp slots must stay 16-byte aligned");
-static_assert(s_ucap<32>() == 608 && s_ucap<16>() == 160 && s_ucap<8>() == 48, "packed U capacity");
+static_assert(s_ucap<32>() == 608 && s_ucap<24>() == 352 && s_ucap<16>() == 160 && s_ucap<8>() == 48,
+              "packed U capacity");
 
 template <int NC, int W>
 __device__ __forceinline__ void s_step(double (&a)[NC], int &k, int &pos, int &my_piv, int &info, bool valid,
@@ -158,10 +164,10 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     const int K = m < n ? m : n;
     // active width W >= n - k in steps of 32 / 24 / 16 / 12 / 8 / 4 (the
     // FMAs, pivot-row loads and publish stores of a step scale with W)
-    if (NC >= 32) {
+    if (NC >= 32)
         while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
-        while (k < K && n - k > 16) s_step<NC, (NC >= 32 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
-    }
+    if (NC >= 24)
+        while (k < K && n - k > 16) s_step<NC, (NC >= 24 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
     if (NC >= 16) {
         while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
         while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
@@ -420,7 +426,10 @@ static void launch_class(const GetrfArgs &a, const int *counters, const int *bin
 // fill in behind it
 void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
     const bool grouped = tuning().tier_s >= 2;
-    if (a.max_n > 16 || a.max_m > 16 || !grouped) launch_class<32>(a, counters, bins, s);
+    if (a.max_n > 16 || a.max_m > 16 || !grouped) {
+        launch_class<32>(a, counters, bins, s);
+        if (grouped && a.max_n > 16) launch_class<24>(a, counters, bins, s);
+    }
     if (a.max_n > 0) {
         if (a.max_m > 16 || !grouped) {
             launch_class<16>(a, counters, bins, s);
