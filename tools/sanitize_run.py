@@ -19,6 +19,10 @@ import oracle  # noqa: E402
 from paper_conf_sc_abdelfattahgbtld22_b200 import irr  # noqa: E402
 
 what = sys.argv[1]
+# extra tuning for the run: IRR_TUNE="key=value,key=value"
+for kv in filter(None, os.environ.get("IRR_TUNE", "").split(",")):
+    k, v = kv.split("=")
+    irr.irr_set_tuning(k, int(v))
 
 
 def getrf_check(shapes, **tune):
@@ -41,7 +45,7 @@ elif what == "L1":
 elif what == "grid1":
     getrf_check([(300, 300), (520, 400), (400, 520), (700, 90)], l1=0, nb_outer=0)
 elif what == "grid2":
-    getrf_check([(300, 300), (520, 400), (400, 520), (700, 90), (90, 700)], l1=0, nb_outer=128)
+    getrf_check([(300, 300), (520, 400), (400, 520), (700, 90), (90, 700), (401, 333)], l1=0, nb_outer=128)
 elif what in ("partial", "partial_lapack"):
     from gpu_util import check_partial, gpu_partial
     shapes = [(3, 4), (17, 40), (50, 80), (129, 200), (300, 150)]
