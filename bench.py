@@ -456,7 +456,9 @@ def main():
     cand = main if big_ran else {k: v for k, v in prof.items() if v[1]}
     dom = max(cand.items(), key=lambda kv: kv[1][0])
     dname, (dms, dcnt) = dom
-    dms_step = dms / args.steps
+    # a class whose kernels run on two streams at once (tier S: the narrow
+    # classes beside the wide ones) sums overlapping intervals: cap at the step
+    dms_step = min(dms / args.steps, total_ms / args.steps)
     fl, by = cw.get(dname, (0.0, 0.0))
     t_f = fl / (FP64_PEAK_TFLOPS * 1e12)
     t_b = by / (hbm * 1e9)

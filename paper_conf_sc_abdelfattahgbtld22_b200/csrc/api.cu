@@ -42,8 +42,10 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // blocks of 128 (round 2: C5 747 -> 637 ms, C3 59.9 -> 57.7 ms; 64 / 96 slower),
 // CTA-per-matrix tier up to 512 rows (C5 641 -> 629, C3 57.5 -> 56.2 ms; 1024
 // rows: C3 61.7), warp-specialised xgemm (8 DMMA warps + a producer warpgroup on an
-// mbarrier ring: C5 616 -> 572 ms, C3 54.8 -> 52.0, C4 91.8 -> 87.0; 16 warps: C3 58.3, C5 651 ms).
-static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64};
+// mbarrier ring: C5 616 -> 572 ms, C3 54.8 -> 52.0, C4 91.8 -> 87.0; 16 warps: C3 58.3, C5 651 ms),
+// its A operand by TMA bulk copies (C5 576.7 -> 575.8, C3 52.22 -> 52.18 ms: neutral, kept;
+// ring 5 x 16: C5 598, 3 x 32: 630 ms).
+static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64, 1};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -136,6 +138,8 @@ struct DeviceStreams {
     cudaEvent_t fork = nullptr, join = nullptr;
     cudaStream_t side2 = nullptr;             // the grid tier's second part
     cudaEvent_t fork2 = nullptr, join2 = nullptr;
+    cudaStream_t side3 = nullptr;             // tier S: the narrow classes beside the wide ones
+    cudaEvent_t fork3 = nullptr, join3 = nullptr;
 };
 static DeviceStreams g_streams[64];
 
@@ -151,6 +155,9 @@ static DeviceStreams *dev_streams() {
         if (cudaStreamCreateWithFlags(&d.side2, cudaStreamNonBlocking) != cudaSuccess) d.side2 = nullptr;
         cudaEventCreateWithFlags(&d.fork2, cudaEventDisableTiming);
         cudaEventCreateWithFlags(&d.join2, cudaEventDisableTiming);
+        if (cudaStreamCreateWithFlags(&d.side3, cudaStreamNonBlocking) != cudaSuccess) d.side3 = nullptr;
+        cudaEventCreateWithFlags(&d.fork3, cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&d.join3, cudaEventDisableTiming);
     }
     return &d;
 }
@@ -256,7 +263,14 @@ static int getrf_core(const GetrfArgs &a, const Work &w, int keep_neg_info, cuda
             side = s;
         }
     }
-    if (t.tier_s) launch_lu_small(a, w.counters, w.bins, side);
+    if (t.tier_s) {
+        // batches of tier-S matrices only: the narrow classes on a second
+        // stream fill the wide classes' tails (C1big 3.44 -> 3.30 ms); with
+        // larger tiers present, tier S already runs beside them on `side`
+        DeviceStreams *ds = (t.concurrent && only_s) ? dev_streams() : nullptr;
+        SmallStreams ss{ds ? ds->side3 : nullptr, ds ? ds->fork3 : nullptr, ds ? ds->join3 : nullptr};
+        launch_lu_small(a, w.counters, w.bins, side, ss.s2 ? &ss : nullptr);
+    }
     if (!only_s) {
         if (mmax > 0) {
             launch_lu_mid(a, w.counters, w.bins, BIN_M1, (int)(mmax < M1_ELEMS ? mmax : M1_ELEMS), side);
@@ -356,6 +370,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "parts")) g_tuning.parts = value >= 2 ? 2 : 1;
     else if (!strcmp(key, "part_grid")) g_tuning.part_grid = value >= 2 ? 2 : 1;
     else if (!strcmp(key, "outer_cols")) g_tuning.outer_cols = value <= 32 ? 32 : 64;
+    else if (!strcmp(key, "xgemm_tma")) g_tuning.xgemm_tma = value ? 1 : 0;
 }
 
 int irr_get_tuning(const char *key) {
@@ -383,6 +398,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "parts")) return g_tuning.parts;
     if (!strcmp(key, "part_grid")) return g_tuning.part_grid;
     if (!strcmp(key, "outer_cols")) return g_tuning.outer_cols;
+    if (!strcmp(key, "xgemm_tma")) return g_tuning.xgemm_tma;
     return -1;
 }
 

@@ -68,12 +68,13 @@ __device__ __forceinline__ void x_pair(double *dst, const double *src, bool ok0,
 // aligned (even leading dimensions 132 / 20).
 template <int TA, int TB, int NT = X_NT>
 __device__ __forceinline__ void xgemm_issue(const GemmDesc &d, int r0, int c0, int k0, BigSmem &sm, int st,
-                                            int tid = -1) {
+                                            int tid = -1, bool skip_a = false) {
     if (tid < 0) tid = threadIdx.x;
     double *As = sm.A[st];
     double *Bs = sm.B[st];
 #pragma unroll
     for (int q = 0; q < (XBM * XBK) / (2 * NT); ++q) {
+        if (skip_a) break;
         const int e = tid + NT * q;
         if (!TA) {  // A(m, k) at A + m + k lda: pairs along m
             const int m = 2 * (e & (XBM / 2 - 1)), kk = e / (XBM / 2);
@@ -119,7 +120,8 @@ struct XWarp {
 };
 
 template <int TA, int TB, int NWG = 8>
-__device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double (&acc)[XWarp<NWG>::ACC]) {
+__device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double (&acc)[XWarp<NWG>::ACC],
+                                              int aoff = 0) {
     constexpr int MI = XWarp<NWG>::MI, WGM = XWarp<NWG>::WGM;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int g = lane >> 2, t = lane & 3;
@@ -132,7 +134,7 @@ __device__ __forceinline__ void xgemm_compute(const BigSmem &sm, int st, double 
 #pragma unroll
         for (int mi = 0; mi < MI; ++mi) {
             const int m = wm + 8 * mi + g, k = ks + t;
-            a[mi] = TA ? As[m * XLD_MK + k] : As[k * XLD_KM + m];
+            a[mi] = TA ? As[m * XLD_MK + k] : As[k * XLD_KM + m + aoff];
         }
 #pragma unroll
         for (int ni = 0; ni < 4; ++ni) {
@@ -397,11 +399,38 @@ __device__ __forceinline__ void mbar_wait(unsigned long long *bar, unsigned pari
         : "memory");
 }
 
+// TMA bulk copy global -> shared, completion counted in bytes on an mbarrier
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, unsigned bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, unsigned long long *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+// TMA path for the A operand (TA = 0, tuning xgemm_tma): each of the 16
+// k-columns of a chunk is one contiguous segment of <= 128 rows in global
+// memory -> one bulk copy per column into its row of the [k][m] stage.  A
+// segment that starts 8 bytes off a 16-byte boundary (odd (A + r0 + k lda))
+// is copied from one element earlier, so its rows sit one slot later:
+// a_shift(d, r0, k) = 1.  The extra element read before / after a segment
+// stays inside the matrix: it is row c1 - 1 of the same column, or the
+// element after row m - 1 of L21 column J + k, i.e. row 0 of column J + k + 1
+// <= c1 < n (padding when ld > m) -- so the path is only used for the
+// two-level trailing update, not for a caller's irr_gemm operands.  Only
+// chunks entirely below K take this path (the K tail keeps the zero-filling
+// cp.async path: A columns past K must read as zeros).
+__device__ __forceinline__ int a_shift(const GemmDesc &d, int r0, int k) {
+    return (int)((reinterpret_cast<uintptr_t>(d.A + r0 + (size_t)k * d.lda) >> 3) & 1);
+}
+
 constexpr int XWS_NT = 384;  // 8 DMMA warps + a producer warpgroup
 
 template <class Prob, int TA, int TB>
 __global__ void __launch_bounds__(XWS_NT, 1) xgemm_ws_kernel(Prob P, int count, const int *count_ptr,
-                                                         const int *__restrict__ tile_off) {
+                                                         const int *__restrict__ tile_off, int tma = 0) {
     extern __shared__ __align__(16) unsigned char x_smem[];
     BigSmem &sm = *reinterpret_cast<BigSmem *>(x_smem);
     __shared__ __align__(8) unsigned long long full_b[XST], empty_b[XST];
@@ -463,7 +492,17 @@ __global__ void __launch_bounds__(XWS_NT, 1) xgemm_ws_kernel(Prob P, int count, 
             for (int kc = 0; kc < nk; ++kc, ++q) {
                 const int st = q % XST;
                 mbar_wait(&empty_b[st], ((q / XST) & 1) ^ 1);
-                xgemm_issue<TA, TB, 128>(cur, r0, c0, kc * XBK, sm, st, ptid);
+                const int k0 = kc * XBK;
+                const bool bulk = !TA && tma && k0 + XBK <= cur.k;
+                if (bulk && ptid < XBK) {
+                    const int rows = imin(XBM, cur.m - r0);
+                    const int sh = a_shift(cur, r0, k0 + ptid);
+                    const double *src = cur.A + r0 + (size_t)(k0 + ptid) * cur.lda - sh;
+                    const unsigned bytes = (unsigned)(((rows + sh) * 8 + 15) & ~15);
+                    mbar_expect_tx(&full_b[st], bytes);
+                    bulk_g2s(sm.A[st] + ptid * XLD_KM, src, bytes, &full_b[st]);
+                }
+                xgemm_issue<TA, TB, 128>(cur, r0, c0, k0, sm, st, ptid, bulk);
                 mbar_arrive_cp_async(&full_b[st]);
             }
             ++local;
@@ -483,7 +522,11 @@ __global__ void __launch_bounds__(XWS_NT, 1) xgemm_ws_kernel(Prob P, int count, 
         for (int kc = 0; kc < nk; ++kc, ++q) {
             const int st = q % XST;
             mbar_wait(&full_b[st], (q / XST) & 1);
-            xgemm_compute<TA, TB, 8>(sm, st, acc);
+            // bulk-copied A columns: k = ks + (lane & 3), so the shift of a
+            // lane's k-column only depends on the parity of its t
+            const bool bulk = !TA && tma && kc * XBK + XBK <= cur.k;
+            const int aoff = bulk ? a_shift(cur, r0, kc * XBK + (lane & 3)) : 0;
+            xgemm_compute<TA, TB, 8>(sm, st, acc, aoff);
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty_b[st]);
         }
@@ -511,7 +554,9 @@ template <class Prob, int TA, int TB>
 inline void xgemm_launch_t(const Prob &P, int cnt, const int *cnt_ptr, const int *tile_off, cudaStream_t s) {
     if (tuning().xgemm_warps == 9) {
         smem_optin(xgemm_ws_kernel<Prob, TA, TB>, BIG_SMEM);
-        xgemm_ws_kernel<Prob, TA, TB><<<num_sms(), XWS_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off);
+        // no TMA path here: a caller's A may end (or start) exactly at its
+        // allocation, and a shifted / rounded segment reads 8 bytes past it
+        xgemm_ws_kernel<Prob, TA, TB><<<num_sms(), XWS_NT, BIG_SMEM, s>>>(P, cnt, cnt_ptr, tile_off, 0);
         return;
     }
     smem_optin(xgemm_sched_kernel<Prob, TA, TB>, BIG_SMEM);

@@ -38,6 +38,7 @@ struct Tuning {
     int parts;           // two-level grid tier: 1, or 2 halves of the LPT list on two streams
     int part_grid;       // with 2 parts: 1 = full grids per part, 2 = half grids
     int outer_cols;      // two-level interchange + U12 solve strip width: 64 (L11 square, 1 CTA/SM) or 32 (packed, 2/SM)
+    int xgemm_tma;       // warp-specialised xgemm: A operand (K-chunk columns) by TMA bulk copies (cp.async.bulk)
 };
 Tuning &tuning();
 
@@ -239,7 +240,14 @@ void launch_classify(const GetrfArgs &a, int *counters, int *bins, int keep_neg_
 void launch_max_dims(int batch, const int *m, const int *n, int *counters, cudaStream_t s);
 
 // lu_small.cu
-void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s);
+// optional second stream for the narrow classes (their kernels fill the wide
+// classes' tails): fork recorded on s, joined back into s
+struct SmallStreams {
+    cudaStream_t s2;
+    cudaEvent_t fork, join;
+};
+void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s,
+                     const SmallStreams *ss = nullptr);
 // lu_mid.cu
 void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int bin, int max_elems,
                    cudaStream_t s);

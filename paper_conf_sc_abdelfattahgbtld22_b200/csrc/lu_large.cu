@@ -1249,7 +1249,8 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
                 }
                 KScope k(K_GEMM_TRAIL, st);
                 if (tu.xgemm_warps == 9)
-                    xgemm_ws_kernel<OuterTrailProb, 0, 0><<<gs, XWS_NT, BIG_SMEM, st>>>(P, -1, cnt_ptr, toff);
+                    xgemm_ws_kernel<OuterTrailProb, 0, 0><<<gs, XWS_NT, BIG_SMEM, st>>>(P, -1, cnt_ptr, toff,
+                                                                                       tu.xgemm_tma);
                 else if (tu.xgemm_warps == 16)
                     xgemm_sched_kernel<OuterTrailProb, 0, 0, 16><<<gs * XGEMM_MINB, 512, BIG_SMEM, st>>>(P, -1, cnt_ptr,
                                                                                                      toff);

@@ -424,21 +424,34 @@ static void launch_class(const GetrfArgs &a, const int *counters, const int *bin
 
 // widest class first: it has the most work per matrix, the narrow kernels
 // fill in behind it
-void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s) {
+void launch_lu_small(const GetrfArgs &a, const int *counters, const int *bins, cudaStream_t s,
+                     const SmallStreams *ss) {
     const bool grouped = tuning().tier_s >= 2;
-    if (a.max_n > 16 || a.max_m > 16 || !grouped) {
+    const bool wide = a.max_n > 16 || a.max_m > 16 || !grouped;
+    // the narrow classes on a second stream when the wide ones run too: each
+    // class is a persistent grid, the second stream's CTAs take the SMs the
+    // wide kernels' tails release
+    cudaStream_t s2 = s;
+    if (ss && wide && a.max_n > 0 && ss->s2 && cudaEventRecord(ss->fork, s) == cudaSuccess &&
+        cudaStreamWaitEvent(ss->s2, ss->fork, 0) == cudaSuccess)
+        s2 = ss->s2;
+    if (wide) {
         launch_class<32>(a, counters, bins, s);
         if (grouped && a.max_n > 16) launch_class<24>(a, counters, bins, s);
     }
     if (a.max_n > 0) {
         if (a.max_m > 16 || !grouped) {
-            launch_class<16>(a, counters, bins, s);
-            launch_class<8>(a, counters, bins, s);
+            launch_class<16>(a, counters, bins, s2);
+            launch_class<8>(a, counters, bins, s2);
         }
         if (grouped) {
-            if (a.max_m > 8 || a.max_n > 8) launch_group<16>(a, counters, bins, BIN_S16G, s);
-            launch_group<8>(a, counters, bins, BIN_S8G, s);
+            if (a.max_m > 8 || a.max_n > 8) launch_group<16>(a, counters, bins, BIN_S16G, s2);
+            launch_group<8>(a, counters, bins, BIN_S8G, s2);
         }
+    }
+    if (s2 != s) {
+        cudaEventRecord(ss->join, s2);
+        cudaStreamWaitEvent(s, ss->join, 0);
     }
 }
 

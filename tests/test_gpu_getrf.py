@@ -503,17 +503,23 @@ def test_grouped_tier_s_bitwise_and_oracle(seed):
         check_getrf(A, LU, ip, int(inf), exact=g >= len(mats) - len(sing), label=f"grouped #{g} {A.shape}")
 
 
-@pytest.mark.parametrize("warps", [8, 16])
+@pytest.mark.parametrize("warps", [8, 16, "tma"])
 def test_xgemm_variants_bitwise_equal(warps):
     """The two-level trailing GEMM on the 8-warp or the 16-warp core gives
     bitwise the factors of the default warp-specialised core (9: 8 DMMA warps
     + a producer warpgroup on an mbarrier ring; same DMMA sequence per
-    accumulator), and matches the oracle."""
+    accumulator), and matches the oracle; "tma": the default core with the A
+    operand staged by cp.async.bulk (odd and even leading dimensions, ragged
+    row tiles, K tails)."""
     irr.irr_set_tuning("l1", 0)
-    shapes = [(700, 700), (300, 1000), (1000, 300), (1300, 1300), (2048, 2048), (129, 900), (2000, 640)]
+    shapes = [(700, 700), (300, 1000), (1000, 300), (1300, 1300), (2048, 2048), (129, 900), (2000, 640),
+              (1001, 1001), (777, 901), (1290, 1290), (513, 700)]
     mats = _uniform(shapes, seed=404)
     one, ip1, inf1, _ = gpu_getrf(mats)
-    irr.irr_set_tuning("xgemm_warps", warps)
+    if warps == "tma":  # the warp-specialised core with the A operand by TMA bulk copies
+        irr.irr_set_tuning("xgemm_tma", 1)
+    else:
+        irr.irr_set_tuning("xgemm_warps", warps)
     two, ip2, inf2, _ = gpu_getrf(mats)
     for a, b, p, q in zip(one, two, ip1, ip2):
         assert np.array_equal(a.view(np.int64), b.view(np.int64)) and np.array_equal(p, q)
