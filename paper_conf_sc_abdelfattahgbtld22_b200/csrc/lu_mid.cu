@@ -10,17 +10,74 @@
 // TRSM of the U12 row block, register-tiled GEMM update of the trailing
 // matrix, all in shared memory.
 #include "panel.cuh"
+#include "gemm_core.cuh"  // dmma_8x8x4
 
 namespace irr {
 
 constexpr int NBM = 16;
+
+// A22 -= L21 U12 in shared memory on the FP64 tensor core (tuning mid_dmma):
+// warp tiles of 32 x 32 = 4 x 4 mma.sync.m8n8k4 tiles, the C fragments read
+// from and written back to the resident matrix, K = ib <= NBM in steps of 4
+// (A = -L21 so that D = C + A B).  Fragment layout of m8n8k4.f64 row.col:
+// lane (g = lane / 4, t = lane % 4) holds A[g][t], B[t][g], C[g][2t, 2t + 1].
+template <int NW>
+__device__ __forceinline__ void mid_update_dmma(double *s, int lds, int j, int ib, int c1, int mi, int ni) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, g = lane >> 2, t = lane & 3;
+    const int Mr = mi - c1, Nc = ni - c1;
+    const int tm = (Mr + 31) >> 5, tn = (Nc + 31) >> 5;
+    for (int item = warp; item < tm * tn; item += NW) {
+        const int rb = c1 + (item % tm) * 32, cb = c1 + (item / tm) * 32;
+        double acc[4][4][2];
+#pragma unroll
+        for (int a4 = 0; a4 < 4; ++a4) {
+            const int r = rb + 8 * a4 + g;
+#pragma unroll
+            for (int b4 = 0; b4 < 4; ++b4) {
+                const int c = cb + 8 * b4 + 2 * t;
+                acc[a4][b4][0] = (r < mi && c < ni) ? s[r + c * lds] : 0.0;
+                acc[a4][b4][1] = (r < mi && c + 1 < ni) ? s[r + (c + 1) * lds] : 0.0;
+            }
+        }
+        for (int kk = 0; kk < ib; kk += 4) {
+            const bool kv = kk + t < ib;
+            const int k = j + kk + t;
+            double a[4], b[4];
+#pragma unroll
+            for (int a4 = 0; a4 < 4; ++a4) {
+                const int r = rb + 8 * a4 + g;
+                a[a4] = (kv && r < mi) ? -s[r + k * lds] : 0.0;
+            }
+#pragma unroll
+            for (int b4 = 0; b4 < 4; ++b4) {
+                const int c = cb + 8 * b4 + g;
+                b[b4] = (kv && c < ni) ? s[k + c * lds] : 0.0;
+            }
+#pragma unroll
+            for (int a4 = 0; a4 < 4; ++a4)
+#pragma unroll
+                for (int b4 = 0; b4 < 4; ++b4) dmma_8x8x4(acc[a4][b4][0], acc[a4][b4][1], a[a4], b[b4]);
+        }
+#pragma unroll
+        for (int a4 = 0; a4 < 4; ++a4) {
+            const int r = rb + 8 * a4 + g;
+            if (r >= mi) continue;
+#pragma unroll
+            for (int b4 = 0; b4 < 4; ++b4) {
+                const int c = cb + 8 * b4 + 2 * t;
+                if (c < ni) s[r + c * lds] = acc[a4][b4][0];
+                if (c + 1 < ni) s[r + (c + 1) * lds] = acc[a4][b4][1];
+            }
+        }
+    }
+}
 
 // M_NT threads, MINB CTAs per SM (registers capped so the footprint-limited
 // occupancy is reachable: M1 48 KB -> 4 CTAs, M2 96 KB -> 2, M3 192 KB -> 1)
 template <int M_NT, int MINB>
 __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const int *__restrict__ counters,
                                                       const int *__restrict__ bins, int bin,
-                                                      unsigned long long *ph) {
+                                                      unsigned long long *ph, int dmma) {
     extern __shared__ __align__(16) double s[];
     long long t0 = 0;
 #define MID_PHASE(k)                                                                    \
@@ -98,10 +155,12 @@ __global__ void __launch_bounds__(M_NT, MINB) lu_mid_kernel(GetrfArgs a, const i
             }
             __syncthreads();
             MID_PHASE(5)
-            // ---- A22 -= L21 * U12 : warp tiles of 64 rows x 4 columns,
-            //      lane owns rows (lane, lane + 32) of the tile
+            // ---- A22 -= L21 * U12 : DMMA warp tiles (mid_dmma), or warp tiles
+            //      of 64 rows x 4 columns with the lane owning rows (lane, lane + 32)
             const int Mr = mi - c1, Nc = ni - c1;
-            if (Mr > 0) {
+            if (Mr > 0 && dmma) {
+                mid_update_dmma<NW>(s, lds, j, ib, c1, mi, ni);
+            } else if (Mr > 0) {
                 const int nrt = (Mr + 63) >> 6, nct = (Nc + 3) >> 2;
                 for (int item = warp; item < nrt * nct; item += NW) {
                     const int tr = item % nrt, tc = item / nrt;
@@ -149,19 +208,20 @@ void launch_lu_mid(const GetrfArgs &a, const int *counters, const int *bins, int
     int grid = num_sms() * per_sm;
     if (grid > a.batch) grid = a.batch;
     if (grid < 1) grid = 1;
+    const int dm = tuning().mid_dmma;
     KScope k(K_LU_MID, s);
     unsigned long long *ph =
         tuning().phase_timing ? reinterpret_cast<unsigned long long *>(const_cast<int *>(counters) + CNT_PHASE0)
                               : nullptr;
     if (per_sm >= 4) {
         smem_optin(lu_mid_kernel<128, 4>, smem);
-        lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin, ph);
+        lu_mid_kernel<128, 4><<<grid, 128, smem, s>>>(a, counters, bins, bin, ph, dm);
     } else if (per_sm >= 2) {
         smem_optin(lu_mid_kernel<256, 2>, smem);
-        lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
+        lu_mid_kernel<256, 2><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph, dm);
     } else {
         smem_optin(lu_mid_kernel<256, 1>, smem);
-        lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph);
+        lu_mid_kernel<256, 1><<<grid, 256, smem, s>>>(a, counters, bins, bin, ph, dm);
     }
 }
 

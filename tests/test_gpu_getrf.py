@@ -57,12 +57,15 @@ def test_edge_shapes_all_tiers():
     assert st.get("match", 0) + st.get("empty", 0) >= len(shapes) - 2
 
 
+@pytest.mark.parametrize("mid_dmma", [0, 1])
 @pytest.mark.parametrize("tier_m_max", [None, 12288, 24576])
-def test_tier_m_boundary_and_extreme_shapes(tier_m_max):
+def test_tier_m_boundary_and_extreme_shapes(tier_m_max, mid_dmma):
     # m * n around the tier-M limits (48 / 96 / 192 KB footprints) and very
-    # thin shapes, at the default limit and with the two larger bins enabled
+    # thin shapes, at the default limit and with the two larger bins enabled;
+    # mid_dmma = 1: the in-shared-memory trailing update on the DMMA core
     if tier_m_max is not None:
         irr.irr_set_tuning("tier_m_max", tier_m_max)
+    irr.irr_set_tuning("mid_dmma", mid_dmma)
     shapes = [(151, 162), (151, 163), (153, 160), (160, 153), (96, 256), (256, 96), (97, 256),
               (77, 79), (78, 78), (79, 78), (110, 111), (111, 110), (64, 96), (95, 64),
               (1, 1024), (1024, 1), (33, 1), (1, 33), (300, 7), (7, 300), (1000, 30), (30, 1000)]
@@ -106,11 +109,12 @@ def test_panel_in_global_memory():
     _run_and_check(mats)
 
 
-@pytest.mark.parametrize("tier", ["default", "M", "L", "L2", "L2two", "Ltall"])
+@pytest.mark.parametrize("tier", ["default", "M", "Mdmma", "L", "L2", "L2two", "Ltall"])
 def test_g1_exact_bitexact(tier):
     """G1: bit-exact L, U, ipiv in any arithmetic order."""
-    if tier == "M":
+    if tier in ("M", "Mdmma"):
         irr.irr_set_tuning("tier_m_max", 24576)
+        irr.irr_set_tuning("mid_dmma", 1 if tier == "Mdmma" else 0)
     if tier == "Ltall":
         irr.irr_set_tuning("l1_rows", 1024)
     if tier == "L2two":
