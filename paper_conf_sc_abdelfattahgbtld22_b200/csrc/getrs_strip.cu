@@ -25,11 +25,20 @@
 
 namespace irr {
 
-constexpr int GS_SW = 64;     // strip width (right-hand sides per unit)
+#ifndef IRR_GS_SW
+#define IRR_GS_SW 64
+#endif
+// strip width (right-hand sides per unit), 64 or 128 (build switch): 128
+// halves the re-reads of F11 per front and gives each warp a 32 x 32 tile,
+// but needs a 3-deep ring for 2 CTAs / SM and was measured slower (C4 a5.2
+// 30.15 vs 29.33 ms, profiles/r02/s2/r3m_*)
+constexpr int GS_SW = IRR_GS_SW;
+constexpr int GS_NI = GS_SW / 32;  // 8-column DMMA tiles per warp (warps: 2 along m x 4 along n)
+constexpr int GS_CPQ = GS_SW / 64; // columns per 4-lane group in the substitution
 constexpr int GS_BR = 64;     // row block of the blocked solve
 constexpr int GS_NT = 256;
 constexpr int GS_BK = 16;     // K chunk of the update GEMM
-constexpr int GS_ST = 4;      // cp.async ring depth (3 chunks in flight: L2 latency)
+constexpr int GS_ST = GS_SW > 64 ? 3 : 4;  // cp.async ring depth (2 CTAs / SM must fit)
 constexpr int GS_LDA = GS_BR + 4;  // [k][m] layout, conflict-free fragments
 constexpr int GS_LDB = GS_BK + 4;  // [n][k] layout
 constexpr int GS_LDT = GS_BR + 1;
@@ -111,12 +120,12 @@ __device__ __forceinline__ void gs_issue(const double *T, long ldt, int r0, int 
     (void)kbeg;
 }
 
-__device__ __forceinline__ void gs_update(double (&acc)[16], const double *T, long ldt, int r0, int rb,
+__device__ __forceinline__ void gs_update(double (&acc)[8 * GS_NI], const double *T, long ldt, int r0, int rb,
                                           const double *X, long ldx, int c0, int W, int kbeg, int kend, GsRing &rg) {
     if (kend <= kbeg) return;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int g = lane >> 2, t = lane & 3;
-    const int wm = (warp & 1) * 32, wn = (warp >> 1) * 16;
+    const int wm = (warp & 1) * 32, wn = (warp >> 1) * (8 * GS_NI);
     const int nk = (kend - kbeg + GS_BK - 1) / GS_BK;
 #pragma unroll
     for (int st = 0; st < GS_ST - 1; ++st) {
@@ -133,17 +142,17 @@ __device__ __forceinline__ void gs_update(double (&acc)[16], const double *T, lo
         const double *Bs = rg.B[kc % GS_ST];
 #pragma unroll
         for (int ks = 0; ks < GS_BK; ks += 4) {
-            double a[4], b[2];
+            double a[4], b[GS_NI];
 #pragma unroll
-            for (int mi = 0; mi < 4; ++mi) a[mi] = As[(ks + t) * GS_LDA + wm + 8 * mi + g];
+            for (int mi = 0; mi < 4; ++mi) a[mi] = -As[(ks + t) * GS_LDA + wm + 8 * mi + g];
 #pragma unroll
-            for (int ni = 0; ni < 2; ++ni) b[ni] = Bs[(wn + 8 * ni + g) * GS_LDB + ks + t];
+            for (int ni = 0; ni < GS_NI; ++ni) b[ni] = Bs[(wn + 8 * ni + g) * GS_LDB + ks + t];
 #pragma unroll
             for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-                for (int ni = 0; ni < 2; ++ni) {
-                    // acc -= a b : negate one operand (exact)
-                    dmma_8x8x4(acc[(mi * 2 + ni) * 2], acc[(mi * 2 + ni) * 2 + 1], -a[mi], b[ni]);
+                for (int ni = 0; ni < GS_NI; ++ni) {
+                    // acc -= a b : one operand negated (exact)
+                    dmma_8x8x4(acc[(mi * GS_NI + ni) * 2], acc[(mi * GS_NI + ni) * 2 + 1], a[mi], b[ni]);
                 }
         }
     }
@@ -159,17 +168,17 @@ __device__ __forceinline__ void gs_block(const double *T, long ldt, double *X, l
                                          int r0, GsRing &rg, GsSolve &sv) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int g = lane >> 2, t = lane & 3;
-    const int wm = (warp & 1) * 32, wn = (warp >> 1) * 16;
+    const int wm = (warp & 1) * 32, wn = (warp >> 1) * (8 * GS_NI);
     const int rb = imin(GS_BR, n1 - r0);
-    double acc[16];
+    double acc[8 * GS_NI];
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
+        for (int ni = 0; ni < GS_NI; ++ni)
 #pragma unroll
             for (int i = 0; i < 2; ++i) {
                 const int r = wm + 8 * mi + g, c = wn + 8 * ni + 2 * t + i;
-                acc[(mi * 2 + ni) * 2 + i] = (r < rb && c < W) ? X[r0 + r + (size_t)(c0 + c) * ldx] : 0.0;
+                acc[(mi * GS_NI + ni) * 2 + i] = (r < rb && c < W) ? X[r0 + r + (size_t)(c0 + c) * ldx] : 0.0;
             }
     if (LOWER) gs_update(acc, T, ldt, r0, rb, X, ldx, c0, W, 0, r0, rg);
     else gs_update(acc, T, ldt, r0, rb, X, ldx, c0, W, r0 + rb, n1, rg);
@@ -185,11 +194,11 @@ __device__ __forceinline__ void gs_block(const double *T, long ldt, double *X, l
 #pragma unroll
     for (int mi = 0; mi < 4; ++mi)
 #pragma unroll
-        for (int ni = 0; ni < 2; ++ni)
+        for (int ni = 0; ni < GS_NI; ++ni)
 #pragma unroll
             for (int i = 0; i < 2; ++i) {
                 const int r = wm + 8 * mi + g, c = wn + 8 * ni + 2 * t + i;
-                sv.X[c * GS_LDT + r] = acc[(mi * 2 + ni) * 2 + i];
+                sv.X[c * GS_LDT + r] = acc[(mi * GS_NI + ni) * 2 + i];
             }
     cp_async_wait<0>();
     __syncthreads();
@@ -200,11 +209,14 @@ __device__ __forceinline__ void gs_block(const double *T, long ldt, double *X, l
         if (tid < GS_BR) sv.rd[tid] = 1.0 / sv.T[tid * GS_LDT + tid];
         __syncthreads();
     }
-    // substitution: column c = tid >> 2; lane q4 = tid & 3 owns rows q4 + 4k
-    // (interleaved, so the four lanes of a column read four consecutive T
-    // entries: conflict-free); x_s comes from lane s & 3 by shuffle
-    {
-        const int c = tid >> 2, q4 = tid & 3;
+    // substitution: columns c = tid >> 2 (and c + 64 when the strip is 128
+    // wide, one after the other: two live chains spill at 128 registers);
+    // lane q4 = tid & 3 owns rows q4 + 4k (interleaved, so the four lanes of
+    // a column read four consecutive T entries: conflict-free); x_s comes
+    // from lane s & 3 by shuffle
+#pragma unroll 1
+    for (int h = 0; h < GS_CPQ; ++h) {
+        const int c = (tid >> 2) + 64 * h, q4 = tid & 3;
         const int base = lane & ~3;
         double x[16];
 #pragma unroll
