@@ -299,7 +299,14 @@ int irr_extend_add(int batch, int max_n2, const int *n2, const double *const *F2
  * shared-memory / global-memory panels), "strip" (1 = grid-wide tier fuses
  * interchange + TRSM + trailing GEMM per 64-column strip; needs panel_win),
  * "phase_timing" (1 = per-phase cycle
- * counters in the workspace).  Unknown keys are ignored;
+ * counters in the workspace), "nb_outer" (outer block of the two-level grid
+ * tier, 0 = one level), "l1_rows" (max rows of the CTA-per-matrix tier),
+ * "xgemm_warps" (trailing GEMM core: 8 or 16 warps, 9 = 8 DMMA warps + a
+ * producer warpgroup on an mbarrier ring; default 9), "xgemm_tma" (1 = the
+ * warp-specialised core's L21 operand by TMA bulk copies; default 1),
+ * "mid_dmma" (1 = tier M's trailing update on the FP64 tensor core; default
+ * 0), "outer_cols", "parts", "part_grid", "defer", "getrs_fused",
+ * "getrs_vec".  Unknown keys are ignored;
  * irr_get_tuning returns the current value (-1 for an unknown key).
  * ---------------------------------------------------------------------- */
 void irr_set_tuning(const char *key, int value);
