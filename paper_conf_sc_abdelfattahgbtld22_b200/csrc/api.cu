@@ -45,7 +45,7 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // mbarrier ring: C5 616 -> 572 ms, C3 54.8 -> 52.0, C4 91.8 -> 87.0; 16 warps: C3 58.3, C5 651 ms),
 // its A operand by TMA bulk copies (C5 576.7 -> 575.8, C3 52.22 -> 52.18 ms: neutral, kept;
 // ring 5 x 16: C5 598, 3 x 32: 630 ms).
-static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64, 1, 0};
+static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64, 1, 0, 0};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
@@ -372,6 +372,7 @@ void irr_set_tuning(const char *key, int value) {
     else if (!strcmp(key, "outer_cols")) g_tuning.outer_cols = value <= 32 ? 32 : 64;
     else if (!strcmp(key, "xgemm_tma")) g_tuning.xgemm_tma = value ? 1 : 0;
     else if (!strcmp(key, "mid_dmma")) g_tuning.mid_dmma = value ? 1 : 0;
+    else if (!strcmp(key, "split_strip")) g_tuning.split_strip = value < 0 ? 0 : (value > 2 ? 2 : value);
 }
 
 int irr_get_tuning(const char *key) {
@@ -401,6 +402,7 @@ int irr_get_tuning(const char *key) {
     if (!strcmp(key, "outer_cols")) return g_tuning.outer_cols;
     if (!strcmp(key, "xgemm_tma")) return g_tuning.xgemm_tma;
     if (!strcmp(key, "mid_dmma")) return g_tuning.mid_dmma;
+    if (!strcmp(key, "split_strip")) return g_tuning.split_strip;
     return -1;
 }
 

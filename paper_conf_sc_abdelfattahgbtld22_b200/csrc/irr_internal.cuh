@@ -40,6 +40,7 @@ struct Tuning {
     int outer_cols;      // two-level interchange + U12 solve strip width: 64 (L11 square, 1 CTA/SM) or 32 (packed, 2/SM)
     int xgemm_tma;       // warp-specialised xgemm: A operand (K-chunk columns) by TMA bulk copies (cp.async.bulk)
     int mid_dmma;        // tier M: trailing update in shared memory on the FP64 tensor core (mma.sync DMMA)
+    int split_strip;     // two-level inner steps: 1 = trailing update as a grid-wide GEMM, 2 = auto (few matrices)
 };
 Tuning &tuning();
 

@@ -568,13 +568,14 @@ static void launch_panel_win(int max_rows, int grid, const GetrfArgs &a, int *co
 // no other CTA can observe a half-swapped column.  Items come from a dynamic
 // queue (reset by the panel kernel).
 constexpr int ST_COLS = GBN;
+constexpr int SPLIT_BATCH = 32;  // split_strip = 2: batches up to this many matrices
 static_assert(sizeof(SwapPlan) <= SWAP_PLAN_BYTES, "plan slot");
 template <bool DMMA>
 __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, int *__restrict__ counters,
                                                         const int *__restrict__ bins,
                                                         const SwapPlan *__restrict__ plans, int *queue, int j,
                                                         int nb, int chunks_per, unsigned long long *ph, int defer,
-                                                        int J, int cmax) {
+                                                        int J, int cmax, int do_gemm = 1) {
     extern __shared__ __align__(16) double st_smem[];
     GemmSmem &gsm = *reinterpret_cast<GemmSmem *>(st_smem);
     const int ldl = nb + 1;
@@ -645,7 +646,7 @@ __global__ void __launch_bounds__(G_NT, 3) strip_kernel(GetrfArgs a, int *__rest
         if (ph && tid == 0) t0 = clock64();
         // trailing GEMM on the strip's right-of-panel columns
         const int cbeg = (v0 > j ? v0 : j) + ib, cend = v0 + W + ib;
-        if (cbeg < cend && c1 < mi) {
+        if (do_gemm && cbeg < cend && c1 < mi) {
             GemmDesc d0;
             d0.A = gA + c1 + (size_t)j * ld; d0.lda = ld; d0.ta = 0;
             d0.B = gA + j + (size_t)cbeg * ld; d0.ldb = ld; d0.tb = 0;
@@ -1032,6 +1033,38 @@ struct TrailingProb {
 template <>
 struct gemm_creg_ok<TrailingProb> { static constexpr bool value = false; };  // measured: staged C is faster
 
+// Few-large batches (tuning split_strip): the inner step's trailing update
+// inside the outer block, C(c1:m, c1:ce) -= L21 U12, as its own grid-wide
+// GEMM over 64 x 64 tiles.  The fused strip kernel streams a strip's whole
+// column range in ONE CTA, so a batch of one or a few large matrices runs
+// its inner steps on one or two CTAs; here every row tile is its own CTA.
+struct InnerTrailProb {
+    GetrfArgs a;
+    const int *list;
+    int j, nb, J, cmax;
+    __device__ bool get(int slot, GemmDesc &d) const {
+        const int i = list[slot];
+        const int mi = a.m[i], ni = a.n[i];
+        const int K = mi < ni ? mi : ni;
+        d.m = 0; d.n = 0; d.k = 0;
+        if (j >= K) return false;
+        const int ib = K - j < nb ? K - j : nb;
+        const int c1 = j + ib;
+        const int ce = imin(imin(ni, cmax), K);
+        if (c1 >= mi || c1 >= ce) return false;
+        const long ld = a.ld[i];
+        double *A = a.A[i];
+        d.A = A + c1 + (size_t)j * ld; d.lda = ld; d.ta = 0;
+        d.B = A + j + (size_t)c1 * ld; d.ldb = ld; d.tb = 0;
+        d.C = A + c1 + (size_t)c1 * ld; d.ldc = ld;
+        d.m = mi - c1; d.n = ce - c1; d.k = ib;
+        d.alpha = -1.0; d.beta = 1.0;
+        return true;
+    }
+};
+template <>
+struct gemm_creg_ok<InnerTrailProb> { static constexpr bool value = false; };
+
 
 static int clamp_nb(int nb) { return nb < 1 ? 1 : (nb > NBMAX ? NBMAX : nb); }
 
@@ -1203,6 +1236,14 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
         const int in_chunks = (nbo + ST_COLS - 1) / ST_COLS;
         // one part = one list of tier-L slots with its own counters block
         // (count, queues), plan slots, tile offsets and stream
+        // few-large batches: the inner trailing update as a grid-wide GEMM
+        // (tuning split_strip: 1 = always, 2 = auto when the batch has at most
+        // SPLIT_BATCH matrices, 0 = never)
+        const bool split = tu.split_strip == 1 || (tu.split_strip == 2 && a.batch <= SPLIT_BATCH);
+        if (split) {
+            gemm_smem_optin(gemm_sched_kernel<InnerTrailProb, true>);
+            gemm_smem_optin(gemm_sched_kernel<InnerTrailProb, false>);
+        }
         auto run_part = [&](int *cnt, int *bns, SwapPlan *pl, OuterPlan *opl, int *toff, cudaStream_t st, int gdiv) {
             const int *listP = bns + (size_t)BIN_L * a.batch;
             const int *cnt_ptr = cnt + CNT_BIN0 + BIN_L;
@@ -1214,11 +1255,26 @@ void launch_lu_large(const GetrfArgs &a, int *counters, const int *bins_c, int *
                         KScope k(K_PANEL, st);
                         launch_panel_win(a.max_m - j, gw, a, cnt, bns, j, nb, pl, cnt + CNT_STRIPQ, st);
                     }
-                    KScope k(K_STRIP, st);
-                    if (tu.dmma) strip_kernel<true><<<gs * 3, G_NT, st_smem, st>>>(
-                        a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
-                    else strip_kernel<false><<<gs * 3, G_NT, st_smem, st>>>(
-                        a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo);
+                    {
+                        KScope k(K_STRIP, st);
+                        const int dg = split ? 0 : 1;
+                        if (tu.dmma) strip_kernel<true><<<gs * 3, G_NT, st_smem, st>>>(
+                            a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo, dg);
+                        else strip_kernel<false><<<gs * 3, G_NT, st_smem, st>>>(
+                            a, cnt, bns, pl, cnt + CNT_STRIPQ, j, nb, in_chunks, ph, 1, J, J + nbo, dg);
+                    }
+                    if (split) {
+                        InnerTrailProb IP{a, listP, j, nb, J, J + nbo};
+                        {
+                            KScope k(K_GEMM_SCAN, st);
+                            gemm_scan_kernel<InnerTrailProb><<<1, 1024, 0, st>>>(IP, -1, cnt_ptr, toff);
+                        }
+                        KScope k(K_STRIP, st);
+                        if (tu.dmma)
+                            gemm_sched_kernel<InnerTrailProb, true><<<gs * 3, G_NT, GEMM_SMEM, st>>>(IP, -1, cnt_ptr, toff);
+                        else
+                            gemm_sched_kernel<InnerTrailProb, false><<<gs * 3, G_NT, GEMM_SMEM, st>>>(IP, -1, cnt_ptr, toff);
+                    }
                 }
                 {
                     KScope k(K_MISC, st);

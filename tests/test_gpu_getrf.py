@@ -364,8 +364,9 @@ def test_pipelined_host_entry_points(chunks):
     assert np.array_equal(fo[2].numpy(), F.info.cpu().numpy())
 
 
+@pytest.mark.parametrize("split", [0, 1])
 @pytest.mark.parametrize("nb,nbo", [(32, 128), (32, 64), (16, 64), (32, 96), (16, 128)])
-def test_two_level_grid_tier(nb, nbo):
+def test_two_level_grid_tier(nb, nbo, split):
     """Grid-wide tier with two-level blocking: inner panels of nb confined to
     outer blocks of nbo, then one interchange + U12 solve + K = nbo GEMM
     update of the rest per outer block.  Ragged outer / inner tails, tall,
@@ -373,6 +374,7 @@ def test_two_level_grid_tier(nb, nbo):
     irr.irr_set_tuning("l1", 0)
     irr.irr_set_tuning("nb", nb)
     irr.irr_set_tuning("nb_outer", nbo)
+    irr.irr_set_tuning("split_strip", split)  # 1: inner trailing update as a grid-wide GEMM
     shapes = [(700, 90), (1024, 64), (1025, 40), (1500, 33), (2048, 70), (513, 513), (90, 700), (600, 600),
               (300, 17), (257, 257), (1000, 1000), (129, 400), (400, 129), (2000, 1300), (nbo + 1, nbo + 1),
               (3 * nbo - 1, 3 * nbo + 5)]

@@ -27,9 +27,12 @@ def _reset_tuning():
     irr.irr_reset_tuning()
 
 
-@pytest.mark.parametrize("nbo", [0, 128])
-def test_large_g1_exact(nbo):
+@pytest.mark.parametrize("nbo,split", [(0, 0), (128, 0), (128, 1)])
+def test_large_g1_exact(nbo, split):
+    """split = 1: the two-level inner steps' trailing update as a grid-wide
+    GEMM (tuning split_strip, the few-large path)."""
     irr.irr_set_tuning("nb_outer", nbo)
+    irr.irr_set_tuning("split_strip", split)
     shapes = [(4096, 4096), (5000, 3000), (3000, 5000), (8192, 700), (40, 40), (300, 300)]
     mats = [irrgen.g1_exact(61, g, m, n)[0] for g, (m, n) in enumerate(shapes)]
     refs = [irrgen.g1_exact(61, g, m, n) for g, (m, n) in enumerate(shapes)]

@@ -113,10 +113,12 @@ def bench_large(reps):
         pristine = torch.rand(B.total, dtype=torch.float64, device="cuda") * 2 - 1
         fl = float(F.getrf_flops([n] * cnt, [n] * cnt).sum())
         res = {}
-        for nbo in (0, 128):
+        for nbo, split in ((0, 0), (128, 0), (128, 1)):
+            irr.irr_reset_tuning()
             irr.irr_set_tuning("nb_outer", nbo)
+            irr.irr_set_tuning("split_strip", split)
             ms = timed(lambda: B.data.copy_(pristine), lambda: B.getrf(), reps)
-            res[f"nb_outer={nbo}"] = {"ms": ms, "gflops": fl / ms / 1e6}
+            res[f"nb_outer={nbo}" + (",split_strip=1" if split else "")] = {"ms": ms, "gflops": fl / ms / 1e6}
         irr.irr_reset_tuning()
         A = pristine[: n * n].view(n, n).clone()
         ms_ref = timed(lambda: None, lambda: torch.linalg.lu_factor(A), reps) * cnt
