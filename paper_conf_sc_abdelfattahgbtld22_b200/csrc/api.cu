@@ -44,8 +44,9 @@ void launch_getrs_strip(int batch, const int *n1, const int *n2, const double *c
 // rows: C3 61.7), warp-specialised xgemm (8 DMMA warps + a producer warpgroup on an
 // mbarrier ring: C5 616 -> 572 ms, C3 54.8 -> 52.0, C4 91.8 -> 87.0; 16 warps: C3 58.3, C5 651 ms),
 // its A operand by TMA bulk copies (C5 576.7 -> 575.8, C3 52.22 -> 52.18 ms: neutral, kept;
-// ring 5 x 16: C5 598, 3 x 32: 630 ms).
-static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64, 1, 0, 0};
+// ring 5 x 16: C5 598, 3 x 32: 630 ms); few-large batches (<= 32 matrices) with the
+// inner trailing update as a grid-wide GEMM (one 4096^2 matrix 50.7 -> 41.1 ms, 8 of them 72.4 -> 58.2).
+static Tuning g_default = {32, 2, M1_ELEMS, 768, 32, 1, 0, 3, 1, 1, 1, 1, 1, 1, 0, 1, 512, 1, 1, NB_OUTER_MAX, 9, 1, 1, 64, 1, 0, 2};
 static Tuning g_tuning = g_default;
 Tuning &tuning() { return g_tuning; }
 
