@@ -1,6 +1,6 @@
-# end-of-session check of HEAD -> gpurun_out/final3 (copied to profiles/r02/final3)
+# end-of-session check of HEAD -> gpurun_out/final4 (copied to profiles/r02/final4)
 export PATH=/usr/local/cuda/bin:$PATH
-O=gpurun_out/final3; mkdir -p $O
+O=gpurun_out/final4; mkdir -p $O
 nvidia-smi --query-gpu=name,driver_version,clocks.max.sm --format=csv > $O/smi.txt
 ( time timeout 1800 python -m pytest tests -q -m gpu -s -p no:randomly ) > $O/pytest_gpu.log 2>&1; echo pytest rc $?; tail -4 $O/pytest_gpu.log | head -2; grep "\[parity" $O/pytest_gpu.log | cut -c1-160
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo smoke rc $?; tail -1 $O/smoke.log
