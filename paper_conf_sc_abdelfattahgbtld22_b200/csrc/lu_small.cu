@@ -56,7 +56,8 @@ struct SmallCfg<8> { static constexpr int ctas = 8, bin = BIN_S8; };    // 64 re
 // touches another row's slots.  Capacity = the widths summed at n = NC.
 template <int NC>
 __host__ __device__ constexpr int s_width(int rem) {
-    return (NC >= 32 && rem > 24) ? 32 : (NC >= 24 && rem > 16) ? 24 : (NC >= 16 && rem > 12) ? 16
+    return (NC >= 32 && rem > 28) ? 32 : (NC >= 32 && rem > 24) ? 28 : (NC >= 24 && rem > 20) ? 24
+         : (NC >= 24 && rem > 16) ? 20 : (NC >= 16 && rem > 12) ? 16
          : (NC >= 16 && rem > 8) ? 12 : (rem > 4) ? (NC >= 8 ? 8 : NC) : 4;
 }
 template <int NC>
@@ -76,7 +77,7 @@ struct __align__(16) SmallWarpSmem {  // 16-byte multiple: U rows take double2 s
 static_assert(sizeof(SmallWarpSmem<32>) % 16 == 0 && sizeof(SmallWarpSmem<24>) % 16 == 0 &&
                   sizeof(SmallWarpSmem<16>) % 16 == 0 && sizeof(SmallWarpSmem<8>) % 16 == 0,
               "per-warp slots must stay 16-byte aligned");
-static_assert(s_ucap<32>() == 608 && s_ucap<24>() == 352 && s_ucap<16>() == 160 && s_ucap<8>() == 48,
+static_assert(s_ucap<32>() == 576 && s_ucap<24>() == 336 && s_ucap<16>() == 160 && s_ucap<8>() == 48,
               "packed U capacity");
 
 template <int NC, int W>
@@ -162,12 +163,16 @@ __device__ __forceinline__ void lu_warp(double *__restrict__ gA, int m, int n, i
     }
     int pos = lane, my_piv = 0, info = 0, k = 0, uo = 0;
     const int K = m < n ? m : n;
-    // active width W >= n - k in steps of 32 / 24 / 16 / 12 / 8 / 4 (the
+    // active width W >= n - k in steps of 32 / 28 / 24 / 20 / 16 / 12 / 8 / 4 (the
     // FMAs, pivot-row loads and publish stores of a step scale with W)
-    if (NC >= 32)
-        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
-    if (NC >= 24)
-        while (k < K && n - k > 16) s_step<NC, (NC >= 24 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+    if (NC >= 32) {
+        while (k < K && n - k > 28) s_step<NC, (NC >= 32 ? 32 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+        while (k < K && n - k > 24) s_step<NC, (NC >= 32 ? 28 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+    }
+    if (NC >= 24) {
+        while (k < K && n - k > 20) s_step<NC, (NC >= 24 ? 24 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+        while (k < K && n - k > 16) s_step<NC, (NC >= 24 ? 20 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
+    }
     if (NC >= 16) {
         while (k < K && n - k > 12) s_step<NC, (NC >= 16 ? 16 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
         while (k < K && n - k > 8) s_step<NC, (NC >= 16 ? 12 : NC)>(a, k, pos, my_piv, info, valid, lane, uo, sm);
