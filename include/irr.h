@@ -329,6 +329,12 @@ long long irr_launch_count(int reset);
  * ---------------------------------------------------------------------- */
 int irr_profile_enable(int max_launches);
 int irr_profile_collect(double *ms, long long *launches, int nclass);
+/* Per class, the length of the UNION of its launches' [start, end] intervals
+ * (ms) since the last collect -- differs from irr_profile_collect's sum when
+ * kernels of one class run concurrently on several streams.  Does not clear
+ * the record; call it before irr_profile_collect.  Returns the number of
+ * launches read, -1 on a CUDA error. */
+int irr_profile_busy(double *busy_ms, int nclass);
 int irr_profile_num_classes(void);
 const char *irr_profile_class_name(int c);
 

@@ -5,6 +5,7 @@
 // expanded interface exists so that no pointer/size arithmetic runs on the
 // host).  The only host loop is over panel ITERATIONS of the largest matrix
 // (P:L167, L179).
+#include <algorithm>
 #include <cstring>
 #include <cstdlib>
 #include <map>
@@ -334,6 +335,39 @@ int irr_profile_collect(double *ms, long long *launches, int nclass) {
     g_open.clear();
     g_ev_used = 0;
     return n;
+}
+
+int irr_profile_busy(double *busy_ms, int nclass) {
+    for (int c = 0; c < nclass; ++c) busy_ms[c] = 0.0;
+    int base = -1;
+    std::vector<std::pair<int, std::pair<double, double>>> iv;  // (class, [t0, t1]) in ms from the first launch
+    for (const ProfRec &r : g_recs) {
+        if (r.ev1 < 0 || r.cls >= nclass) continue;
+        if (cudaEventSynchronize(g_events[r.ev1]) != cudaSuccess) return -1;
+        if (base < 0) base = r.ev0;
+        float t0 = 0.f, t1 = 0.f;
+        if (cudaEventElapsedTime(&t0, g_events[base], g_events[r.ev0]) != cudaSuccess) return -1;
+        if (cudaEventElapsedTime(&t1, g_events[base], g_events[r.ev1]) != cudaSuccess) return -1;
+        iv.push_back({r.cls, {(double)t0, (double)t1}});
+    }
+    std::sort(iv.begin(), iv.end());
+    for (size_t a = 0; a < iv.size();) {  // merge the overlapping intervals of each class
+        const int c = iv[a].first;
+        double lo = iv[a].second.first, hi = iv[a].second.second;
+        size_t b = a + 1;
+        for (; b < iv.size() && iv[b].first == c; ++b) {
+            if (iv[b].second.first > hi) {
+                busy_ms[c] += hi - lo;
+                lo = iv[b].second.first;
+                hi = iv[b].second.second;
+            } else if (iv[b].second.second > hi) {
+                hi = iv[b].second.second;
+            }
+        }
+        busy_ms[c] += hi - lo;
+        a = b;
+    }
+    return (int)iv.size();
 }
 
 int irr_profile_num_classes(void) { return NKCLASS; }

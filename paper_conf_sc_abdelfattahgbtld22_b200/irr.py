@@ -31,6 +31,7 @@ EXPORTED = (
     "irr_getrs_workspace_size", "irr_getrs", "irr_status_words", "irr_extend_add",
     "irr_set_tuning", "irr_get_tuning", "irr_reset_tuning", "irr_launch_count", "irr_version",
     "irr_profile_enable", "irr_profile_collect", "irr_profile_num_classes", "irr_profile_class_name",
+    "irr_profile_busy",
 )
 
 _lib = None
@@ -103,6 +104,8 @@ def load(path: str | None = None):
     L.irr_profile_collect.argtypes = [C.POINTER(C.c_double), C.POINTER(C.c_longlong), i]
     L.irr_profile_collect.restype = i
     L.irr_profile_num_classes.restype = i
+    L.irr_profile_busy.argtypes = [C.POINTER(C.c_double), i]
+    L.irr_profile_busy.restype = i
     L.irr_profile_class_name.argtypes = [i]
     L.irr_profile_class_name.restype = C.c_char_p
     _lib = L
@@ -264,6 +267,18 @@ def irr_version() -> str:
 
 def irr_profile_enable(max_launches: int):
     return _check(load().irr_profile_enable(int(max_launches)), "irr_profile_enable")
+
+
+def irr_profile_busy():
+    """{class name: ms} -- per class the union of its launch intervals since the
+    last collect (overlapping launches on several streams counted once); call
+    before irr_profile_collect."""
+    L = load()
+    nc = L.irr_profile_num_classes()
+    ms = (C.c_double * nc)()
+    if L.irr_profile_busy(ms, nc) < 0:
+        raise IrrError("irr_profile_busy failed")
+    return {L.irr_profile_class_name(c).decode(): ms[c] for c in range(nc)}
 
 
 def irr_profile_collect():
