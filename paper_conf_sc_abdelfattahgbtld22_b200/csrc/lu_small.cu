@@ -31,6 +31,9 @@
 namespace irr {
 
 constexpr int S_WARPS = 4;
+#ifndef IRR_S_PF
+#define IRR_S_PF 1  // L2 prefetch distance of the warp-per-matrix kernels (items ahead)
+#endif
 
 // Width classes n <= 8 / 16 / 32 are separate bins and separate kernels
 // (classify.cu), so the narrow ones run at their own register and
@@ -402,7 +405,7 @@ __global__ void __launch_bounds__(32 * S_WARPS, SmallCfg<NC>::ctas) lu_small_ker
         const int i = list[t];
         const int m = a.m[i], n = a.n[i], ld = a.ld[i];
         double *gA = a.A[i];
-        const int tn = t + stride;
+        const int tn = t + IRR_S_PF * stride;  // prefetch distance in items of this warp
         if (tn < count) {
             const int i2 = list[tn];
             const int m2 = a.m[i2], n2 = a.n[i2], ld2 = a.ld[i2];
